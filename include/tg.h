@@ -1,0 +1,192 @@
+/*
+ * tg.h -- C-ABI of the B200-native TempGraph temporal-path query engine.
+ *
+ * Paper: "TempGraph: An Efficient Chain-driven Temporal Graph Computing
+ * Framework on the GPU" (ASPLOS '25), /root/reference/PAPER.md, cited P:L<line>.
+ *
+ * Model (§2.1): a temporal graph is a list of edges e = (u, v, t, t')
+ * with t' = t + duration, optionally weighted (w).  A path e_1..e_k is legal iff
+ * t'_i <= t_{i+1}.  A query from x in the window [t_alpha, t_omega]
+ * admits paths with t_alpha <= start(P) and end(P) <= t_omega, i.e. an edge can
+ * be used iff t >= t_alpha and t + duration <= t_omega (both ends inclusive).
+ *
+ * Pipeline (§3.2 and Fig. 6):
+ *   tg_graph_create  -- copy + validate the edge list (the input of the
+ *                       "Chain-based Temporal Graph Transformer")
+ *   tg_build_chains  -- transformation into time-dependent chains (Alg. 1,
+ *                       P:L229-264) and shortcut generation (Alg. 2)
+ *   tg_query         -- Generate-Activate-Compute execution (Alg. 3)
+ *
+ * Conventions
+ *   - Every call returns tg_status; no C++ exception crosses the ABI.  On error
+ *     tg_last_error() returns a thread-local message; output buffers are then
+ *     unspecified.
+ *   - All integers are unsigned 32-bit: vertex ids < n_vertices, times and
+ *     durations with t + duration <= TG_TMAX, weights, edge ids (= input index).
+ *   - Pointers may be host or device (CUDA) pointers unless stated otherwise;
+ *     the library detects which with cudaPointerGetAttributes.  Input arrays are
+ *     copied; the caller keeps ownership of everything it passes in.
+ *   - A tg_graph is not thread-safe; distinct handles are independent.
+ *   - All device work runs on the CUDA device given at create time.
+ */
+#ifndef TG_H
+#define TG_H
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define TG_API __attribute__((visibility("default")))
+#else
+#define TG_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tg_graph tg_graph; /* opaque; owned by the caller; free with tg_graph_destroy */
+
+typedef enum {
+    TG_OK = 0,
+    TG_ERR_INVALID = 1, /* bad argument: NULL pointer, duration 0, alpha > omega, bad problem */
+    TG_ERR_RANGE = 2,   /* id >= n, t + duration > TG_TMAX, source >= n, SP distance overflow */
+    TG_ERR_NOMEM = 3,   /* device or host allocation failed */
+    TG_ERR_CUDA = 4,    /* any other CUDA runtime error (message in tg_last_error) */
+    TG_ERR_STATE = 5,   /* call out of order (e.g. tg_query before tg_build_chains) */
+    TG_ERR_NCCL = 6     /* multi-GPU communicator error */
+} tg_status;
+
+/* Problems.  TG_LD is not in the paper: it is the north star's
+ * latest-departure problem, read as single-TARGET (reading A5). */
+typedef enum {
+    TG_EAT = 0,      /* earliest arrival time end(P)                         */
+    TG_LD = 1,       /* latest departure from v of a path reaching the target by omega */
+    TG_FASTEST = 2,  /* min duration(P) = end(P) - start(P), P:L114 (reading A6)       */
+    TG_SHORTEST = 3, /* min dist(P) = sum of w_e, P:L115 / P:L185 (reading A7)         */
+    TG_REACH = 4     /* reachability P(u,v) != {}: out = 1 or 0                */
+} tg_problem;
+
+typedef struct {
+    uint32_t t_alpha; /* earliest allowed departure of the first edge (inclusive) */
+    uint32_t t_omega; /* latest allowed arrival of the last edge (inclusive)      */
+} tg_window;
+
+#define TG_UNREACHED 0xFFFFFFFFu /* value and pred sentinel                                     */
+#define TG_TMAX 0x7FFFFFFEu      /* max t + duration; keeps (time << 32 | id) words below 2^63  */
+
+/*
+ * tg_graph_create -- copy and validate a temporal edge list.
+ *   n_vertices  >= 1.
+ *   n_edges     number of edges m (0 allowed; m < 2^32 - 1).
+ *   u, v        uint32[m] endpoints, each < n_vertices           (else TG_ERR_RANGE)
+ *   t_start     uint32[m] departure times t
+ *   duration    uint32[m] lambda = t' - t >= 1                    (else TG_ERR_INVALID, reading A2)
+ *               t + duration <= TG_TMAX                            (else TG_ERR_RANGE)
+ *   weight      uint32[m] or NULL; NULL means weight = duration (reading A7)
+ *   device      CUDA device ordinal on which the graph lives.
+ *   out_graph   receives the handle.
+ * The edge id of edge i is i; predecessors returned by tg_query are edge ids.
+ */
+TG_API tg_status tg_graph_create(uint32_t n_vertices, uint64_t n_edges,
+                          const uint32_t *u, const uint32_t *v, const uint32_t *t_start,
+                          const uint32_t *duration, const uint32_t *weight,
+                          int device, tg_graph **out_graph);
+
+/*
+ * tg_build_chains -- transform the graph (Alg. 1) into disjoint
+ * time-dependent chains (Def. 1) of the transformed DAG whose vertices
+ * are departure nodes (v, tau) (reading A11), with hubs per Def. 2 (P:L174,
+ * P:L225); generate one shortcut per chain (Alg. 2); build the vertex ->
+ * occurrence index that replaces the paper's GPU hash table.  The same
+ * is done for the time-mirrored graph used by TG_LD (reading A5).  Idempotent.
+ * Runs on the legacy default stream and returns when finished.
+ */
+TG_API tg_status tg_build_chains(tg_graph *g);
+
+/*
+ * tg_query -- n_sources independent single-source queries (a batch; reading A10).
+ *   p           problem.
+ *   sources     HOST uint32[n_sources], each < n_vertices.  For TG_LD they are
+ *               targets (reading A5).
+ *   n_sources   >= 1.
+ *   w           window, t_alpha <= t_omega (else TG_ERR_INVALID).
+ *   out         uint32[n_sources * n_vertices], row r = query sources[r]
+ *               (host or device).  EAT: arrival time (source: t_alpha);
+ *               LD: latest departure (target: t_omega); FASTEST / SHORTEST:
+ *               min duration / distance (source: 0); REACH: 1 or 0.
+ *               Unreached vertices read TG_UNREACHED (REACH: 0).
+ *   pred        NULL or uint32[n_sources * n_vertices] (host or device), only
+ *               for TG_EAT / TG_LD / TG_REACH (else TG_ERR_INVALID).  EAT/REACH: the smallest
+ *               edge id among valid edges e=(u->v) with EAT(u) <= t_e and
+ *               t_e + duration_e = EAT(v); LD: the smallest id among first
+ *               edges of latest-departure paths (reading A9).  Source/target
+ *               and unreached vertices: TG_UNREACHED.
+ *   cuda_stream cudaStream_t to run on (NULL = legacy default stream).  The
+ *               call returns when the results are in `out` / `pred`.
+ * TG_SHORTEST returns TG_ERR_RANGE when the graph's weights could overflow a
+ * uint32 distance (max path length x max weight >= 2^32 - 1).
+ */
+TG_API tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t n_sources,
+                   tg_window w, uint32_t *out, uint32_t *pred, void *cuda_stream);
+
+TG_API void tg_graph_destroy(tg_graph *g); /* NULL-safe */
+
+TG_API const char *tg_status_string(tg_status s);
+TG_API const char *tg_last_error(void); /* thread-local detail of the last error ("" if none) */
+
+/* ---------------------------------------------------------------- introspection */
+typedef struct {
+    uint32_t n_vertices;
+    uint64_t n_edges;
+    uint64_t n_nodes;        /* departure nodes N_X = distinct (u, t)                      */
+    uint64_t n_chains;       /* time-dependent chains (forward graph)                       */
+    uint64_t n_long_chains;  /* chains with >= 2 edges (they carry a computed shortcut)     */
+    uint32_t max_chain_len;
+    uint32_t c_mirror;       /* C = max(t + duration), the LD mirror constant (reading A5)  */
+    uint64_t device_bytes;   /* bytes of device memory held by the graph                    */
+    double build_ms;         /* last tg_build_chains wall time                              */
+    int built;
+    uint64_t n_chains_mirror; /* chains of the LD mirror graph                              */
+} tg_info;
+
+TG_API tg_status tg_graph_info(const tg_graph *g, tg_info *info);
+
+/*
+ * tg_export_chains -- copy the forward chain structure to HOST arrays (tests).
+ *   chain_off   uint64[n_chains + 1]: chain c is slots [chain_off[c], chain_off[c+1])
+ *   chain_edges uint32[n_edges]: edge id at each slot (chain order)
+ *   sc_*        uint32/uint64[n_chains] shortcut per chain (Alg. 2): tail vertex,
+ *               tail arrival, sum of w (uint64), elapsed = arr_last - t_first.
+ *               Any of the sc_* pointers may be NULL.
+ *   mirrored    0 = forward graph, 1 = the LD mirror graph.
+ */
+TG_API tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off, uint32_t *chain_edges,
+                           uint32_t *sc_tail_v, uint32_t *sc_arr, uint64_t *sc_sum_w, uint32_t *sc_elapsed);
+
+typedef struct {
+    uint32_t rounds;          /* GAC rounds of the last tg_query (max over sub-batches)     */
+    uint32_t sub_batches;
+    uint64_t slots_relaxed;   /* relaxations performed (when stats are enabled)              */
+    uint64_t kernel_launches; /* kernels launched by the last tg_query                       */
+} tg_query_stats;
+
+/* Statistics of the last tg_query on this handle.  If per_query_relax is not
+ * NULL and stats are enabled it receives uint64[n_sources]: slots relaxed per
+ * query (equals the one-pass work count W for EAT/LD: each valid usable edge is
+ * relaxed exactly once, "first touch"). */
+TG_API tg_status tg_last_query_stats(const tg_graph *g, tg_query_stats *st, uint64_t *per_query_relax);
+
+/* Tuning / debugging knobs (key, value):
+ *   "sub_batch"  sources processed concurrently (0 = automatic)
+ *   "stats"      1 = count relaxations per query (slower), 0 = off
+ *   "shortcuts"  1 = relax chain tails through shortcuts on first entry (default), 0 = off
+ *   "round_group" rounds launched between host convergence checks (default 4) */
+TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
+
+/* Total kernels this library has launched in this process (all handles). */
+TG_API uint64_t tg_kernel_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TG_H */

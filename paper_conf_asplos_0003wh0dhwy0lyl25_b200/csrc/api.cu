@@ -1,0 +1,267 @@
+// api.cu -- the C-ABI entry points of include/tg.h.
+#include <chrono>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "tg_internal.cuh"
+
+uint64_t g_tg_launches = 0;
+static thread_local std::string t_err;
+
+void tg_set_error(const std::string &msg) { t_err = msg; }
+
+tg_status DevArena::alloc(void **p, size_t bytes) {
+    *p = nullptr;
+    if (nb >= (int)(sizeof(blks) / sizeof(blks[0]))) {
+        tg_set_error("DevArena: too many blocks");
+        return TG_ERR_NOMEM;
+    }
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        tg_set_error(std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+        return TG_ERR_NOMEM;
+    }
+    blks[nb++] = {*p, bytes};
+    total += bytes;
+    return TG_OK;
+}
+
+void DevArena::free_all() {
+    for (int i = 0; i < nb; i++) cudaFree(blks[i].p);
+    nb = 0;
+    total = 0;
+}
+
+tg_status tg_validate_edges(tg_graph *g, cudaStream_t s);
+tg_status tg_build_mirror(tg_graph *g, cudaStream_t s);
+tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
+                            uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
+tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
+                      bool out_dev, cudaStream_t s);
+
+static bool is_device_ptr(const void *p) {
+    if (!p) return false;
+    cudaPointerAttributes a;
+    cudaError_t e = cudaPointerGetAttributes(&a, p);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+namespace {
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+}  // namespace
+
+extern "C" {
+
+const char *tg_status_string(tg_status s) {
+    switch (s) {
+        case TG_OK: return "TG_OK";
+        case TG_ERR_INVALID: return "TG_ERR_INVALID";
+        case TG_ERR_RANGE: return "TG_ERR_RANGE";
+        case TG_ERR_NOMEM: return "TG_ERR_NOMEM";
+        case TG_ERR_CUDA: return "TG_ERR_CUDA";
+        case TG_ERR_STATE: return "TG_ERR_STATE";
+        case TG_ERR_NCCL: return "TG_ERR_NCCL";
+    }
+    return "TG_ERR_UNKNOWN";
+}
+
+const char *tg_last_error(void) { return t_err.c_str(); }
+
+uint64_t tg_kernel_launch_count(void) { return g_tg_launches; }
+
+tg_status tg_graph_create(uint32_t n_vertices, uint64_t n_edges, const uint32_t *u, const uint32_t *v,
+                          const uint32_t *t_start, const uint32_t *duration, const uint32_t *weight, int device,
+                          tg_graph **out_graph) {
+    t_err.clear();
+    if (!out_graph) { tg_set_error("out_graph is NULL"); return TG_ERR_INVALID; }
+    *out_graph = nullptr;
+    if (n_vertices == 0) { tg_set_error("n_vertices must be >= 1"); return TG_ERR_INVALID; }
+    if (n_edges >= 0xFFFFFFFFull) { tg_set_error("n_edges must be < 2^32 - 1"); return TG_ERR_RANGE; }
+    if (n_edges > 0 && (!u || !v || !t_start || !duration)) { tg_set_error("edge array is NULL"); return TG_ERR_INVALID; }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        tg_set_error("no CUDA device");
+        return TG_ERR_CUDA;
+    }
+    if (device < 0 || device >= ndev) { tg_set_error("bad device ordinal"); return TG_ERR_INVALID; }
+    DeviceGuard dg(device);
+    tg_graph *g = new tg_graph();
+    g->device = device;
+    g->n = n_vertices;
+    g->m = n_edges;
+    const size_t bytes = n_edges * 4;
+    tg_status st = TG_OK;
+    auto fail = [&](tg_status s) { g->arena.free_all(); delete g; return s; };
+    uint32_t **dst[5] = {&g->d_u, &g->d_v, &g->d_t, &g->d_dur, &g->d_w};
+    const uint32_t *src[5] = {u, v, t_start, duration, weight};
+    for (int i = 0; i < 5; i++) {
+        if (i == 4 && !weight) { g->d_w = g->d_dur; break; }  // reading A7: w = duration
+        if ((st = g->arena.alloc((void **)dst[i], bytes)) != TG_OK) return fail(st);
+        if (n_edges) {
+            cudaError_t e = cudaMemcpy(*dst[i], src[i], bytes, cudaMemcpyDefault);
+            if (e != cudaSuccess) { tg_set_error(cudaGetErrorString(e)); cudaGetLastError(); return fail(TG_ERR_CUDA); }
+        }
+    }
+    if ((st = tg_validate_edges(g, 0)) != TG_OK) return fail(st);
+    *out_graph = g;
+    return TG_OK;
+}
+
+tg_status tg_build_chains(tg_graph *g) {
+    t_err.clear();
+    if (!g) { tg_set_error("graph is NULL"); return TG_ERR_INVALID; }
+    if (g->built) return TG_OK;
+    DeviceGuard dg(g->device);
+    auto t0 = std::chrono::steady_clock::now();
+    TG_TRY(tg_build_direction(g, &g->fwd, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, 0));
+    TG_TRY(tg_build_mirror(g, 0));
+    TG_TRY_CUDA(cudaDeviceSynchronize());
+    g->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    g->built = true;
+    return TG_OK;
+}
+
+tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t n_sources, tg_window w, uint32_t *out,
+                   uint32_t *pred, void *cuda_stream) {
+    t_err.clear();
+    if (!g) { tg_set_error("graph is NULL"); return TG_ERR_INVALID; }
+    if (!g->built) { tg_set_error("tg_query before tg_build_chains"); return TG_ERR_STATE; }
+    if (!sources || !out || n_sources == 0) { tg_set_error("sources/out NULL or n_sources == 0"); return TG_ERR_INVALID; }
+    if ((int)p < 0 || (int)p > TG_REACH) { tg_set_error("unknown problem"); return TG_ERR_INVALID; }
+    if (pred && !(p == TG_EAT || p == TG_LD || p == TG_REACH)) {
+        tg_set_error("pred is only defined for TG_EAT / TG_LD / TG_REACH");
+        return TG_ERR_INVALID;
+    }
+    if (w.t_alpha > w.t_omega) { tg_set_error("t_alpha > t_omega"); return TG_ERR_INVALID; }
+    if (is_device_ptr(sources)) { tg_set_error("sources must be a host pointer"); return TG_ERR_INVALID; }
+    for (uint32_t i = 0; i < n_sources; i++)
+        if (sources[i] >= g->n) { tg_set_error("source >= n_vertices"); return TG_ERR_RANGE; }
+    if (p == TG_SHORTEST && !g->sp_ok) {
+        tg_set_error("shortest-path distances could overflow uint32 for this graph's weights");
+        return TG_ERR_RANGE;
+    }
+    DeviceGuard dg(g->device);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    const bool out_dev = is_device_ptr(out);
+    const bool pred_dev = is_device_ptr(pred);
+    if (p == TG_EAT || p == TG_LD || p == TG_REACH)
+        return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
+    return tg_run_spfp(g, p, sources, n_sources, w, out, out_dev, s);
+}
+
+void tg_graph_destroy(tg_graph *g) {
+    if (!g) return;
+    DeviceGuard dg(g->device);
+    cudaDeviceSynchronize();
+    g->qs.arena.free_all();
+    if (g->qs.h_ctr) cudaFreeHost(g->qs.h_ctr);
+    g->arena.free_all();
+    delete[] g->last_relax;
+    delete g;
+}
+
+tg_status tg_graph_info(const tg_graph *g, tg_info *info) {
+    if (!g || !info) { tg_set_error("NULL argument"); return TG_ERR_INVALID; }
+    std::memset(info, 0, sizeof(*info));
+    info->n_vertices = g->n;
+    info->n_edges = g->m;
+    info->n_nodes = g->fwd.nnodes;
+    info->n_chains = g->fwd.nchains;
+    info->n_long_chains = g->fwd.nlong;
+    info->max_chain_len = g->fwd.maxlen;
+    info->c_mirror = g->max_arr;
+    info->device_bytes = g->arena.total + g->qs.arena.total;
+    info->build_ms = g->build_ms;
+    info->built = g->built ? 1 : 0;
+    info->n_chains_mirror = g->mir.nchains;
+    return TG_OK;
+}
+
+tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off, uint32_t *chain_edges,
+                           uint32_t *sc_tail_v, uint32_t *sc_arr, uint64_t *sc_sum_w, uint32_t *sc_elapsed) {
+    if (!g || !chain_off || !chain_edges) { tg_set_error("NULL argument"); return TG_ERR_INVALID; }
+    if (!g->built) { tg_set_error("graph not built"); return TG_ERR_STATE; }
+    DeviceGuard dg(g->device);
+    const ChainGraph &c = mirrored ? g->mir : g->fwd;
+    const uint64_t m = g->m, nc = c.nchains;
+    std::vector<uint32_t> first(nc + 1);
+    std::vector<int4> slots(m);
+    TG_TRY_CUDA(cudaMemcpy(first.data(), c.chain_first, (nc + 1) * 4, cudaMemcpyDeviceToHost));
+    if (m) TG_TRY_CUDA(cudaMemcpy(slots.data(), c.slots, m * 16, cudaMemcpyDeviceToHost));
+    for (uint64_t i = 0; i <= nc; i++) chain_off[i] = first[i];
+    for (uint64_t s = 0; s < m; s++) chain_edges[s] = (uint32_t)slots[s].z;
+    if (sc_tail_v || sc_arr || sc_sum_w || sc_elapsed) {
+        std::vector<int4> sc(c.nlong);
+        std::vector<unsigned long long> sumw(c.nlong);
+        std::vector<uint32_t> el(c.nlong), w(m), slot_w(m), t(m);
+        if (c.nlong) {
+            TG_TRY_CUDA(cudaMemcpy(sc.data(), c.sc, c.nlong * 16, cudaMemcpyDeviceToHost));
+            TG_TRY_CUDA(cudaMemcpy(sumw.data(), c.sc_sumw, c.nlong * 8, cudaMemcpyDeviceToHost));
+            TG_TRY_CUDA(cudaMemcpy(el.data(), c.sc_elapsed, c.nlong * 4, cudaMemcpyDeviceToHost));
+        }
+        if (m) {
+            TG_TRY_CUDA(cudaMemcpy(slot_w.data(), c.slot_w, m * 4, cudaMemcpyDeviceToHost));
+            // departure time of a one-edge chain = arrival - duration of its edge
+            std::vector<uint32_t> dur(m);
+            TG_TRY_CUDA(cudaMemcpy(dur.data(), g->d_dur, m * 4, cudaMemcpyDeviceToHost));
+            for (uint64_t s = 0; s < m; s++) t[s] = (uint32_t)slots[s].y - dur[(uint32_t)slots[s].z];
+        }
+        for (uint64_t ch = 0; ch < nc; ch++) {
+            uint32_t b = first[ch], e = first[ch + 1];
+            int4 sl = slots[b];
+            if (e - b >= 2) {
+                uint32_t l = (uint32_t)sl.w;
+                if (sc_tail_v) sc_tail_v[ch] = (uint32_t)sc[l].x;
+                if (sc_arr) sc_arr[ch] = (uint32_t)sc[l].y;
+                if (sc_sum_w) sc_sum_w[ch] = sumw[l];
+                if (sc_elapsed) sc_elapsed[ch] = el[l];
+            } else {  // Alg. 2 line 8: a one-edge chain is its own shortcut
+                if (sc_tail_v) sc_tail_v[ch] = (uint32_t)sl.x;
+                if (sc_arr) sc_arr[ch] = (uint32_t)sl.y;
+                if (sc_sum_w) sc_sum_w[ch] = slot_w[b];
+                if (sc_elapsed) sc_elapsed[ch] = (uint32_t)sl.y - t[b];
+            }
+        }
+    }
+    return TG_OK;
+}
+
+tg_status tg_last_query_stats(const tg_graph *g, tg_query_stats *st, uint64_t *per_query_relax) {
+    if (!g || !st) { tg_set_error("NULL argument"); return TG_ERR_INVALID; }
+    *st = g->last;
+    if (per_query_relax && g->last_relax)
+        std::memcpy(per_query_relax, g->last_relax, (size_t)g->last_relax_len * 8);
+    return TG_OK;
+}
+
+tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
+    if (!g || !key) { tg_set_error("NULL argument"); return TG_ERR_INVALID; }
+    std::string k(key);
+    if (k == "sub_batch") g->opt_sub_batch = value;
+    else if (k == "stats") g->opt_stats = value;
+    else if (k == "shortcuts") g->opt_shortcuts = value;
+    else if (k == "round_group") g->opt_round_group = value;
+    else { tg_set_error("unknown option " + k); return TG_ERR_INVALID; }
+    return TG_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,395 @@
+// build.cu -- chain-based temporal graph transformation on the GPU (sm_100a).
+//
+// Paper: §4.1 "Chain-based Temporal Graph Transformation" (Alg. 1),
+// §4.2 "Skeleton-graph Generation" (Alg. 2), storage P:L273 (Fig. 8).
+// The paper runs Alg. 1 on CPU threads (DFS from each hub); here every step is a
+// data-parallel kernel:
+//   1. key = (u << tbits) | t, stable radix sort with edge-id payload  -> edges in (u, t, id) order
+//   2. segmentation into departure nodes (v, tau) = distinct (u, t)   (DAG vertices, reading A11)
+//   3. snap: tail node of each edge = first departure of v at or after t + duration (binary search)
+//   4. in-degree histogram, hub flags (Def. 2, P:L174 / P:L225)
+//   5. successor of each edge through non-hub nodes; chain heads = out-edges of hubs
+//   6. chain lengths (walk), scan -> slot offsets, scatter 16-byte slots chain-major
+//   7. shortcut per long chain (Alg. 2 fold) and the occurrence index (replaces the
+//      GPU hash table of: sorted-edge position -> slot)
+#include <algorithm>
+
+#include "tg_internal.cuh"
+
+namespace {
+
+constexpr int BT = 256;
+
+inline unsigned blocks_for(uint64_t n, int per_thread = 1) {
+    uint64_t b = (n + (uint64_t)BT * per_thread - 1) / ((uint64_t)BT * per_thread);
+    return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, 148ull * 64));
+}
+
+#define GRID_STRIDE(i, n) for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < (n); \
+                               i += (uint64_t)gridDim.x * blockDim.x)
+
+__global__ void k_make_keys(const uint32_t *__restrict__ u, const uint32_t *__restrict__ t, uint64_t m, int tbits,
+                            unsigned long long *__restrict__ keys, uint32_t *__restrict__ ids) {
+    GRID_STRIDE(i, m) {
+        keys[i] = ((unsigned long long)u[i] << tbits) | t[i];
+        ids[i] = (uint32_t)i;
+    }
+}
+
+// departure-node boundaries in (u, t)-sorted order
+__global__ void k_node_flags(const unsigned long long *__restrict__ keys, uint64_t m, uint32_t *__restrict__ flag) {
+    GRID_STRIDE(p, m) flag[p] = (p == 0 || keys[p] != keys[p - 1]) ? 1u : 0u;
+}
+
+// node_of[p] (exclusive-scanned flags, adjusted) and per-node arrays
+__global__ void k_nodes(const unsigned long long *__restrict__ keys, uint64_t m, int tbits,
+                        uint32_t *__restrict__ node_of /* in: excl scan of flags */,
+                        uint32_t *__restrict__ node_t, uint32_t *__restrict__ node_u,
+                        uint32_t *__restrict__ node_eoff) {
+    const unsigned long long tmask = (1ull << tbits) - 1ull;
+    GRID_STRIDE(p, m) {
+        unsigned long long k = keys[p];
+        bool head = (p == 0 || k != keys[p - 1]);
+        uint32_t j = node_of[p];
+        if (head) {
+            node_t[j] = (uint32_t)(k & tmask);
+            node_u[j] = (uint32_t)(k >> tbits);
+            node_eoff[j] = (uint32_t)p;
+            node_of[p] = j;
+        } else {
+            node_of[p] = j - 1;
+        }
+    }
+}
+
+// vnode_off[w] = first node of vertex w (CSR over vertices; empty vertices repeat)
+__global__ void k_vnode_off(const uint32_t *__restrict__ node_u, uint64_t nn, uint32_t n,
+                            uint32_t *__restrict__ vnode_off) {
+    GRID_STRIDE(j, nn + 1) {
+        int64_t prev = (j == 0) ? -1 : (int64_t)node_u[j - 1];
+        int64_t cur = (j == nn) ? (int64_t)n : (int64_t)node_u[j];
+        for (int64_t w = prev + 1; w <= cur; w++) vnode_off[w] = (uint32_t)j;
+    }
+}
+
+// snap each sorted edge to its tail departure node; count in-degrees
+__global__ void k_snap(const uint32_t *__restrict__ sid, uint64_t m, const uint32_t *__restrict__ V,
+                       const uint32_t *__restrict__ T, const uint32_t *__restrict__ DUR,
+                       const uint32_t *__restrict__ vnode_off, const uint32_t *__restrict__ node_t,
+                       uint32_t *__restrict__ tn, uint32_t *__restrict__ s_v, uint32_t *__restrict__ s_arr,
+                       uint32_t *__restrict__ indeg) {
+    GRID_STRIDE(p, m) {
+        uint32_t e = sid[p];
+        uint32_t v = V[e];
+        uint32_t arr = T[e] + DUR[e];
+        uint32_t lo = vnode_off[v], hi = vnode_off[v + 1];
+        uint32_t j = tg_lower_bound(node_t, lo, hi, arr);
+        uint32_t r = (j < hi) ? j : TG_NONE;
+        tn[p] = r;
+        s_v[p] = v;
+        s_arr[p] = arr;
+        if (r != TG_NONE) atomicAdd(&indeg[r], 1u);
+    }
+}
+
+// hub (Def. 2): in-degree 0, in-degree >= 2, or out-degree >= 2
+__global__ void k_hubs(const uint32_t *__restrict__ indeg, const uint32_t *__restrict__ node_eoff, uint64_t nn,
+                       unsigned char *__restrict__ hub) {
+    GRID_STRIDE(j, nn) {
+        uint32_t outdeg = node_eoff[j + 1] - node_eoff[j];
+        hub[j] = (indeg[j] != 1u || outdeg >= 2u) ? 1 : 0;
+    }
+}
+
+// chain heads = out-edges of hubs; successor through a non-hub tail node
+__global__ void k_succ(const uint32_t *__restrict__ node_of, const uint32_t *__restrict__ tn, uint64_t m,
+                       const unsigned char *__restrict__ hub, const uint32_t *__restrict__ node_eoff,
+                       uint32_t *__restrict__ head, uint32_t *__restrict__ succ) {
+    GRID_STRIDE(p, m) {
+        head[p] = hub[node_of[p]] ? 1u : 0u;
+        uint32_t r = tn[p];
+        succ[p] = (r != TG_NONE && !hub[r]) ? node_eoff[r] : TG_NONE;
+    }
+}
+
+// ChainPartitioning (Alg. 1 lines 8-19) as a walk from each head: chain length
+__global__ void k_chain_len(const uint32_t *__restrict__ head, const uint32_t *__restrict__ cidx,
+                            const uint32_t *__restrict__ succ, uint64_t m, uint32_t *__restrict__ chain_len,
+                            uint32_t *__restrict__ maxlen) {
+    uint32_t mx = 0;
+    GRID_STRIDE(p, m) {
+        if (!head[p]) continue;
+        uint32_t len = 1;
+        for (uint32_t q = succ[p]; q != TG_NONE; q = succ[q]) len++;
+        chain_len[cidx[p]] = len;
+        mx = max(mx, len);
+    }
+    for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if ((threadIdx.x & 31) == 0) atomicMax(maxlen, mx);
+}
+
+__global__ void k_long_flags(const uint32_t *__restrict__ chain_len, uint64_t nc, uint32_t *__restrict__ lflag) {
+    GRID_STRIDE(c, nc) lflag[c] = chain_len[c] >= 2 ? 1u : 0u;
+}
+
+// Scatter slots chain-major and generate shortcuts (Alg. 2): one thread per chain.
+__global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_t *__restrict__ cidx,
+                                const uint32_t *__restrict__ succ, uint64_t m,
+                                const uint32_t *__restrict__ chain_first, const uint32_t *__restrict__ chain_len,
+                                const uint32_t *__restrict__ lidx, const uint32_t *__restrict__ sid,
+                                const uint32_t *__restrict__ s_v, const uint32_t *__restrict__ s_arr,
+                                const uint32_t *__restrict__ tn, const uint32_t *__restrict__ node_of,
+                                const uint32_t *__restrict__ T, const uint32_t *__restrict__ Wt,
+                                int4 *__restrict__ slots, uint32_t *__restrict__ slot_w,
+                                uint32_t *__restrict__ slot_tn, uint32_t *__restrict__ occ_slot,
+                                uint2 *__restrict__ lc, int4 *__restrict__ sc,
+                                unsigned long long *__restrict__ sc_sumw, uint32_t *__restrict__ sc_elapsed) {
+    GRID_STRIDE(p, m) {
+        if (!head[p]) continue;
+        uint32_t c = cidx[p];
+        uint32_t first = chain_first[c];
+        uint32_t len = chain_len[c];
+        uint32_t l = (len >= 2) ? lidx[c] : TG_SINGLE;
+        uint32_t s = first;
+        uint32_t q = p, last = p;
+        unsigned long long sumw = 0;
+        while (q != TG_NONE) {
+            uint32_t e = sid[q];
+            uint32_t w = Wt[e];
+            slots[s] = make_int4((int)s_v[q], (int)s_arr[q], (int)e, (int)l);
+            slot_w[s] = w;
+            slot_tn[s] = tn[q];
+            occ_slot[q] = s;
+            sumw += w;  // GenerateShortcut: accumulate W_e (Alg. 2 line 5)
+            last = q;
+            s++;
+            q = succ[q];
+        }
+        if (len >= 2) {
+            lc[l] = make_uint2(first, len);
+            sc[l] = make_int4((int)s_v[last], (int)s_arr[last], (int)sid[last], (int)node_of[p]);
+            sc_sumw[l] = sumw;
+            sc_elapsed[l] = s_arr[last] - T[sid[p]];
+        }
+    }
+}
+
+__global__ void k_validate(const uint32_t *__restrict__ u, const uint32_t *__restrict__ v,
+                           const uint32_t *__restrict__ t, const uint32_t *__restrict__ dur,
+                           const uint32_t *__restrict__ w, uint64_t m, uint32_t n, uint32_t *__restrict__ res) {
+    // res: [0] flags (1 range id, 2 duration 0, 4 t+dur > TMAX), [1] max t, [2] max arr, [3] max w, [4] min t
+    uint32_t flags = 0, mt = 0, ma = 0, mw = 0, mn = 0xFFFFFFFFu;
+    GRID_STRIDE(i, m) {
+        uint32_t a = u[i], b = v[i], tt = t[i], d = dur[i];
+        if (a >= n || b >= n) flags |= 1u;
+        if (d == 0) flags |= 2u;
+        unsigned long long arr = (unsigned long long)tt + d;
+        if (arr > TG_TMAX) flags |= 4u;
+        mt = max(mt, tt);
+        mn = min(mn, tt);
+        ma = max(ma, (uint32_t)min(arr, 0xFFFFFFFFull));
+        mw = max(mw, w ? w[i] : d);
+    }
+    for (int o = 16; o; o >>= 1) {
+        flags |= __shfl_xor_sync(0xffffffffu, flags, o);
+        mt = max(mt, __shfl_xor_sync(0xffffffffu, mt, o));
+        mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+        ma = max(ma, __shfl_xor_sync(0xffffffffu, ma, o));
+        mw = max(mw, __shfl_xor_sync(0xffffffffu, mw, o));
+    }
+    if ((threadIdx.x & 31) == 0) {
+        if (flags) atomicOr(&res[0], flags);
+        atomicMax(&res[1], mt);
+        atomicMax(&res[2], ma);
+        atomicMax(&res[3], mw);
+        atomicMin(&res[4], mn);
+    }
+}
+
+__global__ void k_mirror(const uint32_t *__restrict__ t, const uint32_t *__restrict__ dur, uint64_t m, uint32_t C,
+                         uint32_t *__restrict__ mt) {
+    // reading A5: e = (u,v,t,lam) -> (v,u, C - (t + lam), lam)
+    GRID_STRIDE(i, m) mt[i] = C - (t[i] + dur[i]);
+}
+
+}  // namespace
+
+tg_status tg_validate_edges(tg_graph *g, cudaStream_t s) {
+    uint32_t *res = nullptr;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&res, 5 * 4, s));
+    uint32_t init[5] = {0, 0, 0, 0, 0xFFFFFFFFu};
+    TG_TRY_CUDA(cudaMemcpyAsync(res, init, sizeof(init), cudaMemcpyHostToDevice, s));
+    if (g->m) TG_LAUNCH(k_validate, blocks_for(g->m, 4), BT, 0, s, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, g->m, g->n, res);
+    uint32_t h[5];
+    TG_TRY_CUDA(cudaMemcpyAsync(h, res, sizeof(h), cudaMemcpyDeviceToHost, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    TG_TRY_CUDA(cudaFreeAsync(res, s));
+    if (h[0] & 1u) { tg_set_error("edge endpoint >= n_vertices"); return TG_ERR_RANGE; }
+    if (h[0] & 2u) { tg_set_error("edge duration 0 (durations must be >= 1, reading A2)"); return TG_ERR_INVALID; }
+    if (h[0] & 4u) { tg_set_error("t + duration > TG_TMAX"); return TG_ERR_RANGE; }
+    g->max_t = h[1];
+    g->max_arr = h[2];
+    g->max_w = h[3];
+    g->min_t = g->m ? h[4] : 0;
+    // SP distances: a legal path has strictly increasing departures (duration >= 1),
+    // so at most min(m, max_t - min_t + 1) edges; its distance fits in uint32 if
+    // that bound times max_w stays below 2^32 - 1.
+    unsigned long long maxlen = std::min<unsigned long long>(g->m, (unsigned long long)g->max_t - g->min_t + 1);
+    g->sp_ok = (unsigned __int128)maxlen * g->max_w < 0xFFFFFFFFull;
+    return TG_OK;
+}
+
+static int bits_for(uint64_t x) {  // bits to represent values in [0, x]
+    int b = 0;
+    while (b < 64 && (x >> b) != 0) b++;
+    return std::max(b, 1);
+}
+
+tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, const uint32_t *u, const uint32_t *v, const uint32_t *t,
+                             const uint32_t *dur, const uint32_t *w, cudaStream_t s) {
+    const uint64_t m = g->m;
+    const uint32_t n = g->n;
+    cg->n = n;
+    cg->m = m;
+    DevArena &A = g->arena;
+    TG_TRY(A.alloc((void **)&cg->vnode_off, ((size_t)n + 1) * 4));
+    if (m == 0) {
+        TG_TRY_CUDA(cudaMemsetAsync(cg->vnode_off, 0, ((size_t)n + 1) * 4, s));
+        TG_TRY(A.alloc((void **)&cg->chain_first, 4));
+        TG_TRY_CUDA(cudaMemsetAsync(cg->chain_first, 0, 4, s));
+        return TG_OK;
+    }
+    // ---- 1. sort by (u, t, id)
+    uint32_t maxt = 0;
+    {
+        // max over this direction's t (mirror times differ from forward ones)
+        uint32_t *res = nullptr;
+        TG_TRY_CUDA(cudaMallocAsync((void **)&res, 5 * 4, s));
+        uint32_t init[5] = {0, 0, 0, 0, 0xFFFFFFFFu};
+        TG_TRY_CUDA(cudaMemcpyAsync(res, init, sizeof(init), cudaMemcpyHostToDevice, s));
+        TG_LAUNCH(k_validate, blocks_for(m, 4), BT, 0, s, u, v, t, dur, w, m, n, res);
+        uint32_t h[5];
+        TG_TRY_CUDA(cudaMemcpyAsync(h, res, sizeof(h), cudaMemcpyDeviceToHost, s));
+        TG_TRY_CUDA(cudaStreamSynchronize(s));
+        TG_TRY_CUDA(cudaFreeAsync(res, s));
+        maxt = h[1];
+    }
+    const int tbits = bits_for(maxt);
+    const int ubits = bits_for(n - 1);
+    unsigned long long *keys = nullptr;
+    uint32_t *sid = nullptr;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&keys, m * 8, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&sid, m * 4, s));
+    TG_LAUNCH(k_make_keys, blocks_for(m, 4), BT, 0, s, u, t, m, tbits, keys, sid);
+    unsigned long long *sk;
+    uint32_t *sv;
+    TG_TRY(tg_radix_sort_pairs(keys, sid, m, tbits + ubits, &sk, &sv, s));
+
+    // ---- 2. departure nodes
+    uint32_t *node_of = nullptr, *d_cnt = nullptr;
+    TG_TRY(A.alloc((void **)&cg->occ_node, m * 4));
+    node_of = cg->occ_node;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&d_cnt, 16, s));
+    TG_LAUNCH(k_node_flags, blocks_for(m, 4), BT, 0, s, keys, m, node_of);
+    TG_TRY(tg_exclusive_scan_u32(node_of, node_of, m, d_cnt, s, nullptr));
+    uint32_t h_cnt = 0;
+    TG_TRY_CUDA(cudaMemcpyAsync(&h_cnt, d_cnt, 4, cudaMemcpyDeviceToHost, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    // the scan's total excludes the first flag (exclusive); nodes = total of flags
+    // k_nodes turns excl-scan values into node ids: head p -> j = excl[p], others excl[p]-1.
+    {
+        // number of nodes = excl[m-1] + flag[m-1]; recompute on host from the two values
+        uint32_t last_excl = 0;
+        unsigned long long k_last = 0, k_prev = 0;
+        TG_TRY_CUDA(cudaMemcpyAsync(&last_excl, node_of + (m - 1), 4, cudaMemcpyDeviceToHost, s));
+        TG_TRY_CUDA(cudaMemcpyAsync(&k_last, keys + (m - 1), 8, cudaMemcpyDeviceToHost, s));
+        if (m >= 2) TG_TRY_CUDA(cudaMemcpyAsync(&k_prev, keys + (m - 2), 8, cudaMemcpyDeviceToHost, s));
+        TG_TRY_CUDA(cudaStreamSynchronize(s));
+        bool last_head = (m == 1) || (k_last != k_prev);
+        cg->nnodes = (uint64_t)last_excl + (last_head ? 1 : 0);
+    }
+    const uint64_t nn = cg->nnodes;
+    TG_TRY(A.alloc((void **)&cg->node_t, nn * 4));
+    TG_TRY(A.alloc((void **)&cg->node_u, nn * 4));
+    TG_TRY(A.alloc((void **)&cg->node_eoff, (nn + 1) * 4));
+    // k_nodes: for heads excl == node id; for non-heads excl == node id + 1
+    TG_LAUNCH(k_nodes, blocks_for(m, 4), BT, 0, s, keys, m, tbits, node_of, cg->node_t, cg->node_u, cg->node_eoff);
+    {
+        uint32_t mm = (uint32_t)m;
+        TG_TRY_CUDA(cudaMemcpyAsync(cg->node_eoff + nn, &mm, 4, cudaMemcpyHostToDevice, s));
+    }
+    TG_LAUNCH(k_vnode_off, blocks_for(nn + 1, 4), BT, 0, s, cg->node_u, nn, n, cg->vnode_off);
+    TG_TRY_CUDA(cudaFreeAsync(keys, s));
+
+    // ---- 3./4. snap, in-degree, hubs
+    uint32_t *tn = nullptr, *s_v = nullptr, *s_arr = nullptr, *indeg = nullptr;
+    unsigned char *hub = nullptr;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&tn, m * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&s_v, m * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&s_arr, m * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&indeg, nn * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&hub, nn, s));
+    TG_TRY_CUDA(cudaMemsetAsync(indeg, 0, nn * 4, s));
+    TG_LAUNCH(k_snap, blocks_for(m, 4), BT, 0, s, sid, m, v, t, dur, cg->vnode_off, cg->node_t, tn, s_v, s_arr, indeg);
+    TG_LAUNCH(k_hubs, blocks_for(nn, 4), BT, 0, s, indeg, cg->node_eoff, nn, hub);
+    TG_TRY_CUDA(cudaFreeAsync(indeg, s));
+
+    // ---- 5. heads / successors; chain ids in (head u, head t, first id) order
+    uint32_t *head = nullptr, *succ = nullptr, *cidx = nullptr;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&head, m * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&succ, m * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&cidx, m * 4, s));
+    TG_LAUNCH(k_succ, blocks_for(m, 4), BT, 0, s, node_of, tn, m, hub, cg->node_eoff, head, succ);
+    TG_TRY(tg_exclusive_scan_u32(head, cidx, m, d_cnt, s, nullptr));
+    uint32_t nch = 0;
+    TG_TRY_CUDA(cudaMemcpyAsync(&nch, d_cnt, 4, cudaMemcpyDeviceToHost, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    cg->nchains = nch;
+
+    // ---- 6. chain lengths, slot offsets, long-chain numbering
+    uint32_t *chain_len = nullptr, *lidx = nullptr;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&chain_len, (uint64_t)nch * 4 + 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&lidx, (uint64_t)nch * 4 + 4, s));
+    TG_TRY_CUDA(cudaMemsetAsync(d_cnt + 2, 0, 4, s));
+    TG_LAUNCH(k_chain_len, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, chain_len, d_cnt + 2);
+    TG_TRY(A.alloc((void **)&cg->chain_first, ((uint64_t)nch + 1) * 4));
+    TG_TRY(tg_exclusive_scan_u32(chain_len, cg->chain_first, nch, cg->chain_first + nch, s, nullptr));
+    TG_LAUNCH(k_long_flags, blocks_for(nch, 4), BT, 0, s, chain_len, nch, lidx);
+    TG_TRY(tg_exclusive_scan_u32(lidx, lidx, nch, d_cnt + 1, s, nullptr));
+    uint32_t h2[3] = {0, 0, 0};
+    TG_TRY_CUDA(cudaMemcpyAsync(h2, d_cnt, 12, cudaMemcpyDeviceToHost, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    cg->nlong = h2[1];
+    cg->maxlen = h2[2];
+    const uint64_t L = cg->nlong;
+
+    TG_TRY(A.alloc((void **)&cg->slots, m * 16));
+    TG_TRY(A.alloc((void **)&cg->slot_w, m * 4));
+    TG_TRY(A.alloc((void **)&cg->slot_tn, m * 4));
+    TG_TRY(A.alloc((void **)&cg->occ_slot, m * 4));
+    TG_TRY(A.alloc((void **)&cg->lc, std::max<uint64_t>(L, 1) * 8));
+    TG_TRY(A.alloc((void **)&cg->sc, std::max<uint64_t>(L, 1) * 16));
+    TG_TRY(A.alloc((void **)&cg->sc_sumw, std::max<uint64_t>(L, 1) * 8));
+    TG_TRY(A.alloc((void **)&cg->sc_elapsed, std::max<uint64_t>(L, 1) * 4));
+    TG_LAUNCH(k_chain_scatter, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, cg->chain_first, chain_len, lidx, sid,
+              s_v, s_arr, tn, node_of, t, w, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
+              cg->sc_sumw, cg->sc_elapsed);
+
+    for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)s_v, (void *)s_arr, (void *)hub,
+                    (void *)head, (void *)succ, (void *)cidx, (void *)chain_len, (void *)lidx})
+        TG_TRY_CUDA(cudaFreeAsync(p, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    return TG_OK;
+}
+
+tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {
+    // reading A5: G^R maps (u, v, t, lam) to (v, u, C - (t + lam), lam), C = max(t + lam)
+    if (g->m == 0) return tg_build_direction(g, &g->mir, g->d_v, g->d_u, g->d_t, g->d_dur, g->d_w, s);
+    uint32_t *mt = nullptr;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&mt, g->m * 4, s));
+    TG_LAUNCH(k_mirror, blocks_for(g->m, 4), BT, 0, s, g->d_t, g->d_dur, g->m, g->max_arr, mt);
+    tg_status st = tg_build_direction(g, &g->mir, g->d_v, g->d_u, mt, g->d_dur, g->d_w, s);
+    cudaFreeAsync(mt, s);
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    return st;
+}

@@ -1,0 +1,321 @@
+// query_spfp.cu -- GAC execution for SHORTEST and FASTEST paths (sm_100a).
+//
+// Paper: §3.1 and Alg. 3 with the per-problem hooks of
+// Table 1: VInitial (root 0 / others +inf for SP),
+// GenerateShortcut (sum of W_e for SP, the chain's start-preserving hop for FP,
+// P:L185), Propagate (min(dst, src + w)).
+//
+// Unlike EAT, a chain vertex's state here depends on WHEN the path arrived, so
+// the state lives on departure nodes (v, tau) of the transformed DAG (reading
+// A11): dnode[q][j] = min distance (SP) or max latest start LS (FP, stored as
+// key = 0xFFFFFFFE - LS so both are atomicMin).  Waiting at a vertex is the
+// implicit wait edge (v, tau_i) -> (v, tau_{i+1}); it is propagated by a short
+// forward scan over the vertex's later departure nodes when a node improves.
+//
+// Round: frontier = improved nodes.  Activate: wait-propagate each improved node
+// over later nodes of its vertex (stop at the first node that is already as
+// good), then expand the out-edges of all improved nodes warp-cooperatively.
+// Compute: from each entered slot walk the chain ((min,+) for SP, max for FP),
+// atomicMin on tail node states and on the per-vertex output; stop where the
+// tail node does not improve (whoever improved it pushed it).
+#include <cooperative_groups.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "tg_internal.cuh"
+
+namespace cg = cooperative_groups;
+
+tg_status tg_ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state);
+uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state);
+
+namespace {
+
+constexpr int QT = 256;
+constexpr uint32_t BIG_T = 256;
+constexpr uint32_t CHUNK = 1024;
+constexpr uint32_t WAIT_MAX = 64;  // wait-propagation steps per item per round
+
+struct SpP {
+    const uint32_t *vnode_off, *node_t, *node_u, *node_eoff, *occ_slot, *occ_node;
+    const int4 *slots;
+    const uint32_t *slot_w, *slot_tn;
+    const uint2 *lc;
+    const int4 *sc;
+    const unsigned long long *sc_sumw;
+    uint32_t *dnode, *vout, *mark;
+    uint32_t n;
+    uint64_t nnodes;
+    uint32_t alpha, omega, stamp;
+    int use_sc;
+    const unsigned long long *fin;
+    const uint32_t *fin_cnt;
+    unsigned long long *fout;
+    uint32_t *fout_cnt;
+    uint4 *bigq;
+    uint32_t *big_cnt;
+    uint64_t bigcap;
+};
+
+__device__ __forceinline__ void push_node(const SpP &P, uint32_t q, uint32_t j) {
+    const size_t i = (size_t)q * P.nnodes + j;
+    if (atomicExch(P.mark + i, P.stamp) != P.stamp) {
+        cg::coalesced_group g = cg::coalesced_threads();
+        uint32_t base = 0;
+        if (g.thread_rank() == 0) base = atomicAdd(P.fout_cnt, g.size());
+        base = g.shfl(base, 0);
+        P.fout[base + g.thread_rank()] = ((unsigned long long)q << 32) | j;
+    }
+}
+
+// Walk the chain from slot s (entered with head-node value cur).
+template <bool FP>
+__device__ void spfp_walk(const SpP &P, uint32_t q, uint32_t s, uint32_t s_end, uint32_t cur) {
+    uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
+    uint32_t *vo = P.vout + (size_t)q * P.n;
+    for (; s < s_end; s++) {
+        const int4 sl = tg_ld_slot(P.slots + s);
+        const uint32_t arr = (uint32_t)sl.y;
+        if (arr > P.omega) return;
+        uint32_t cand;
+        if (FP) {
+            cand = cur;                                    // latest start is preserved along the path
+            atomicMin(vo + sl.x, arr - (0xFFFFFFFEu - cur));  // duration = end - start (reading A6)
+        } else {
+            cand = cur + __ldg(P.slot_w + s);              // Propagate: src + w
+            atomicMin(vo + sl.x, cand);
+        }
+        const uint32_t tn = __ldg(P.slot_tn + s);
+        if (tn == TG_NONE) return;  // sink
+        const uint32_t old = atomicMin(dn + tn, cand);
+        if (cand >= old) return;    // not improved: the improver pushed tn
+        push_node(P, q, tn);        // wait propagation + other out-edges next round
+        cur = cand;
+    }
+}
+
+template <bool FP>
+__device__ __forceinline__ void spfp_edge(const SpP &P, uint32_t q, uint32_t p) {
+    const uint32_t s = __ldg(P.occ_slot + p);
+    const uint32_t j = __ldg(P.occ_node + p);
+    const uint32_t cur = __ldcg(P.dnode + (size_t)q * P.nnodes + j);
+    if (cur == TG_NONE) return;
+    const int4 sl = tg_ld_slot(P.slots + s);
+    if ((uint32_t)sl.y > P.omega) return;
+    uint32_t s_end = s + 1;
+    if ((uint32_t)sl.w != TG_SINGLE) {
+        const uint32_t l = (uint32_t)sl.w;
+        const uint2 info = __ldg(P.lc + l);
+        s_end = info.x + info.y;
+        if (P.use_sc && s == info.x) {
+            // skeleton: Propagate(S_l) head -> tail with the shortcut weight (Alg. 2 / Alg. 3 line 6)
+            const int4 scv = __ldg(P.sc + l);
+            if ((uint32_t)scv.y <= P.omega) {
+                const uint32_t tn = __ldg(P.slot_tn + s_end - 1);
+                uint32_t cand;
+                if (FP) {
+                    cand = cur;
+                    atomicMin(P.vout + (size_t)q * P.n + scv.x, (uint32_t)scv.y - (0xFFFFFFFEu - cur));
+                } else {
+                    cand = cur + (uint32_t)__ldg(P.sc_sumw + l);
+                    atomicMin(P.vout + (size_t)q * P.n + scv.x, cand);
+                }
+                if (tn != TG_NONE) {
+                    const uint32_t old = atomicMin(P.dnode + (size_t)q * P.nnodes + tn, cand);
+                    if (cand < old) push_node(P, q, tn);
+                }
+            }
+        }
+    }
+    spfp_walk<FP>(P, q, s, s_end, cur);
+}
+
+template <bool FP>
+__global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
+    const uint32_t F = *P.fin_cnt;
+    const int lane = threadIdx.x & 31;
+    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t base = gw * 32; base < F; base += nw * 32) {
+        const uint32_t i = base + lane;
+        uint32_t q = 0, e0 = 0, cnt = 0;
+        if (i < F) {
+            const unsigned long long it = P.fin[i];
+            q = (uint32_t)(it >> 32);
+            const uint32_t j = (uint32_t)it;
+            uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
+            const uint32_t d = __ldcg(dn + j);
+            const uint32_t u = __ldg(P.node_u + j);
+            const uint32_t vend = __ldg(P.vnode_off + u + 1);
+            // wait edges: later departure nodes of u inherit d (reading A11)
+            uint32_t jend = j + 1;
+            for (uint32_t steps = 0; jend < vend; jend++, steps++) {
+                if (__ldg(P.node_t + jend) >= P.omega) break;  // no valid out-edge departs at >= omega
+                const uint32_t old = atomicMin(dn + jend, d);
+                if (old <= d) break;
+                if (steps == WAIT_MAX) { push_node(P, q, jend); break; }  // continue next round
+            }
+            e0 = __ldg(P.node_eoff + j);
+            cnt = __ldg(P.node_eoff + jend) - e0;
+        }
+        if (cnt > BIG_T) {
+            const uint32_t nch = (cnt + CHUNK - 1) / CHUNK;
+            const uint32_t k = atomicAdd(P.big_cnt, nch);
+            for (uint32_t c = 0; c < nch; c++) {
+                const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
+                if (k + c < P.bigcap) P.bigq[k + c] = make_uint4(q, b0, b1, 0);
+                else for (uint32_t p = b0; p < b1; p++) spfp_edge<FP>(P, q, p);
+            }
+            cnt = 0;
+        }
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+        const uint32_t excl = incl - cnt;
+        for (uint32_t gb = 0; gb < total; gb += 32) {
+            const uint32_t g = gb + lane;
+            uint32_t own = 0;
+#pragma unroll
+            for (int b = 16; b; b >>= 1) {
+                const uint32_t v = __shfl_sync(0xffffffffu, incl, own + b - 1);
+                if (v <= g) own += b;
+            }
+            own &= 31;
+            const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
+            const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
+            const uint32_t oq = __shfl_sync(0xffffffffu, q, own);
+            if (g < total) spfp_edge<FP>(P, oq, oe0 + (g - oex));
+        }
+    }
+}
+
+template <bool FP>
+__global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
+    const uint32_t B = (uint32_t)min((uint64_t)*P.big_cnt, P.bigcap);
+    const int lane = threadIdx.x & 31;
+    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t it = gw; it < B; it += nw) {
+        const uint4 c = P.bigq[it];
+        for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<FP>(P, c.x, p);
+    }
+}
+
+// VInitial: the source's departure nodes tau >= alpha get 0 (SP) / LS = tau (FP).
+template <bool FP>
+__global__ void k_spfp_init(SpP P, const uint32_t *srcs, uint32_t S) {
+    const uint32_t q = blockIdx.y;
+    if (q >= S) return;
+    const uint32_t x = srcs[q];
+    const uint32_t a = P.vnode_off[x], b = P.vnode_off[x + 1];
+    const uint32_t j0 = tg_lower_bound(P.node_t, a, b, P.alpha);
+    for (uint32_t j = j0 + blockIdx.x * blockDim.x + threadIdx.x; j < b; j += gridDim.x * blockDim.x) {
+        const uint32_t tau = P.node_t[j];
+        if (tau >= P.omega) break;
+        P.dnode[(size_t)q * P.nnodes + j] = FP ? (0xFFFFFFFEu - tau) : 0u;
+        push_node(P, q, j);
+    }
+}
+
+__global__ void k_spfp_extract(const uint32_t *__restrict__ vout, uint32_t n, const uint32_t *__restrict__ srcs,
+                               uint32_t *__restrict__ out) {
+    const uint32_t q = blockIdx.y;
+    const uint32_t src = srcs[q];
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        const size_t i = (size_t)q * n + v;
+        out[i] = (v == src) ? 0u : vout[i];
+    }
+}
+
+}  // namespace
+
+template <bool FP>
+static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t omega, cudaStream_t s,
+                             uint32_t *rounds_out) {
+    QueryScratch &Q = g->qs;
+    const ChainGraph &c = g->fwd;
+    const uint64_t n = g->n, nn = c.nnodes;
+    TG_TRY_CUDA(cudaMemsetAsync(Q.vout, 0xFF, Sb * n * 4, s));
+    if (nn) TG_TRY_CUDA(cudaMemsetAsync(Q.dnode, 0xFF, Sb * nn * 4, s));
+    uint32_t rounds = 0;
+    if (g->m == 0 || alpha >= omega) { *rounds_out = 0; return TG_OK; }
+    SpP P{};
+    P.vnode_off = c.vnode_off; P.node_t = c.node_t; P.node_u = c.node_u; P.node_eoff = c.node_eoff;
+    P.occ_slot = c.occ_slot; P.occ_node = c.occ_node; P.slots = c.slots; P.slot_w = c.slot_w; P.slot_tn = c.slot_tn;
+    P.lc = c.lc; P.sc = c.sc; P.sc_sumw = c.sc_sumw;
+    P.dnode = Q.dnode; P.vout = Q.vout; P.mark = Q.mark; P.n = g->n; P.nnodes = nn;
+    P.alpha = alpha; P.omega = omega; P.use_sc = (int)g->opt_shortcuts;
+    P.bigq = Q.bigq; P.bigcap = Q.bigcap;
+    // round 1 input = buffer 1
+    TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + 4, 0, 4, s));
+    if (++g->qs_epoch == 0) {
+        TG_TRY_CUDA(cudaMemsetAsync(Q.mark, 0, (uint64_t)Q.S * std::max<uint64_t>(n, nn) * 4, s));
+        g->qs_epoch = 1;
+    }
+    P.stamp = g->qs_epoch;
+    P.fout = Q.fr[1]; P.fout_cnt = Q.ctr + 4;
+    {
+        dim3 grid(4, Sb);
+        TG_LAUNCH(k_spfp_init<FP>, grid, 256, 0, s, P, Q.srcs, Sb);
+    }
+    const uint32_t grid = tg_grid_persistent(8);
+    const int group = (int)std::max<int64_t>(1, g->opt_round_group);
+    uint32_t r = 1;
+    for (;;) {
+        for (int k = 0; k < group; k++, r++) {
+            const int in = r & 1, outp = (r + 1) & 1;
+            TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + outp * 4, 0, 4, s));
+            TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + in * 4 + 1, 0, 8, s));
+            if (++g->qs_epoch == 0) {
+                TG_TRY_CUDA(cudaMemsetAsync(Q.mark, 0, (uint64_t)Q.S * std::max<uint64_t>(n, nn) * 4, s));
+                g->qs_epoch = 1;
+            }
+            P.stamp = g->qs_epoch;
+            P.fin = Q.fr[in]; P.fin_cnt = Q.ctr + in * 4;
+            P.fout = Q.fr[outp]; P.fout_cnt = Q.ctr + outp * 4;
+            P.big_cnt = Q.ctr + in * 4 + 1;
+            TG_LAUNCH(k_spfp_activate<FP>, grid, QT, 0, s, P);
+            TG_LAUNCH(k_spfp_big<FP>, grid, QT, 0, s, P);
+        }
+        TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctr, 32, cudaMemcpyDeviceToHost, s));
+        TG_TRY_CUDA(cudaStreamSynchronize(s));
+        if (Q.h_ctr[(r & 1) * 4] == 0) break;
+        if (r > 10000000) { tg_set_error("SP/FP rounds did not converge"); return TG_ERR_CUDA; }
+    }
+    rounds = r - 1;
+    *rounds_out = rounds;
+    return TG_OK;
+}
+
+tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
+                      bool out_dev, cudaStream_t s) {
+    const bool fp = (p == TG_FASTEST);
+    const uint32_t S = tg_pick_sub_batch(g, k, true);
+    TG_TRY(tg_ensure_scratch(g, S, true));
+    QueryScratch &Q = g->qs;
+    const uint64_t n = g->n;
+    if (!out_dev && !Q.out_stage) TG_TRY(Q.arena.alloc((void **)&Q.out_stage, (uint64_t)Q.S * n * 4));
+    g->last = tg_query_stats{};
+    const uint64_t launches0 = g_tg_launches;
+    for (uint32_t b0 = 0; b0 < k; b0 += S) {
+        const uint32_t Sb = std::min(S, k - b0);
+        TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources + b0, Sb * 4, cudaMemcpyHostToDevice, s));
+        uint32_t rounds = 0;
+        if (fp) TG_TRY((spfp_rounds<true>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
+        else TG_TRY((spfp_rounds<false>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
+        g->last.rounds = std::max(g->last.rounds, rounds);
+        g->last.sub_batches++;
+        uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
+        dim3 grid((unsigned)std::min<uint64_t>((n + 255) / 256, 1024), Sb);
+        TG_LAUNCH(k_spfp_extract, grid, 256, 0, s, Q.vout, g->n, Q.srcs, o);
+        if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
+    }
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    g->last.kernel_launches = g_tg_launches - launches0;
+    return TG_OK;
+}

@@ -1,0 +1,165 @@
+// tg_internal.cuh -- shared definitions of the CUDA path (product code).
+// Nothing here is shared with oracle/ (test infrastructure).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/tg.h"
+
+#define TG_NONE 0xFFFFFFFFu
+#define TG_SINGLE 0xFFFFFFFFu  // slot.w for a one-edge chain (no long-chain index)
+
+// ----------------------------------------------------------------------------- errors
+void tg_set_error(const std::string &msg);
+extern uint64_t g_tg_launches;  // kernels launched by this library (process-wide)
+
+#define TG_TRY_CUDA(expr)                                                                      \
+    do {                                                                                       \
+        cudaError_t _e = (expr);                                                               \
+        if (_e != cudaSuccess) {                                                               \
+            tg_set_error(std::string(#expr) + ": " + cudaGetErrorString(_e) + " @" __FILE__); \
+            return (_e == cudaErrorMemoryAllocation) ? TG_ERR_NOMEM : TG_ERR_CUDA;             \
+        }                                                                                      \
+    } while (0)
+
+#define TG_TRY(expr)                   \
+    do {                               \
+        tg_status _s = (expr);         \
+        if (_s != TG_OK) return _s;    \
+    } while (0)
+
+// Launch bookkeeping: every kernel launch goes through this macro so that the
+// bench can report how many of OUR kernels ran inside its timed region.
+#define TG_LAUNCH(kernel, grid, block, smem, stream, ...)                  \
+    do {                                                                   \
+        kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);        \
+        g_tg_launches++;                                                   \
+        TG_TRY_CUDA(cudaGetLastError());                                   \
+    } while (0)
+
+// ----------------------------------------------------------------------------- device memory
+// Simple owning device buffer list for a graph handle.
+struct DevArena {
+    struct Blk { void *p; size_t bytes; };
+    Blk blks[96];
+    int nb = 0;
+    size_t total = 0;
+    tg_status alloc(void **p, size_t bytes);
+    void free_all();
+};
+
+// One direction of the transformed graph (forward, or the LD mirror).
+// Layout in HBM:
+//   departure nodes (v, tau) in (v, tau) order:   vnode_off[n+1], node_t[N], node_u[N], node_eoff[N+1]
+//   sorted edges (by (u, t, id)), "occurrences": occ_slot[m] -> slot index, occ_node[m] -> node
+//   slots in chain-major order (chains ordered by head (u, t, first id)):
+//       slots int4[m] = {v, arr = t + duration, edge id, long-chain index | TG_SINGLE}
+//       slot_w[m], slot_tn[m] (tail departure node or TG_NONE)   -- SP/FP only
+//   long chains (>= 2 edges): lc uint2[L] = {first slot, length}
+//                             sc int4[L]  = {tail v, tail arrival, tail edge id, head node}
+//                             sc_sumw uint64[L], sc_elapsed uint32[L]  (Alg. 2 shortcut weights)
+//   chain_first[nchains+1]: first slot of every chain (export / parity)
+struct ChainGraph {
+    uint32_t n = 0;
+    uint64_t m = 0;
+    uint64_t nnodes = 0, nchains = 0, nlong = 0;
+    uint32_t maxlen = 0;
+    uint32_t *vnode_off = nullptr, *node_t = nullptr, *node_u = nullptr, *node_eoff = nullptr;
+    uint32_t *occ_slot = nullptr;
+    uint32_t *occ_node = nullptr;  // sorted-edge position -> departure node (SP/FP entry state)
+    int4 *slots = nullptr;
+    uint32_t *slot_w = nullptr, *slot_tn = nullptr;
+    uint2 *lc = nullptr;
+    int4 *sc = nullptr;
+    unsigned long long *sc_sumw = nullptr;
+    uint32_t *sc_elapsed = nullptr;
+    uint32_t *chain_first = nullptr;
+};
+
+struct QueryScratch {
+    uint32_t S = 0;          // sources per sub-batch this scratch was sized for
+    uint32_t n = 0;
+    uint64_t nlong = 0;
+    uint64_t nnodes = 0;
+    bool nodes_state = false;  // SP/FP node-state arrays present
+    unsigned long long *st = nullptr;  // [S][n] packed (time << 32 | pred)
+    uint32_t *act = nullptr;           // [S][n] last activated time
+    uint32_t *mark = nullptr;          // [S][n] (EAT) or [S][nnodes] (SP/FP) frontier dedupe stamp
+    uint32_t *entry = nullptr;         // [S][nlong] first entered position per long chain
+    uint32_t *dnode = nullptr;         // [S][nnodes] SP/FP node state
+    uint32_t *vout = nullptr;          // [S][n] SP/FP per-vertex output
+    unsigned long long *fr[2] = {nullptr, nullptr};  // frontier items (q << 32 | vertex-or-node)
+    uint64_t fcap = 0;
+    uint4 *bigq = nullptr;   // big activation chunks {q, e_begin, e_end, -}
+    uint64_t bigcap = 0;
+    uint4 *chq = nullptr;    // long chain walks {q, s_begin, s_end, -}
+    uint64_t chcap = 0;
+    uint32_t *ctr = nullptr;   // counters [2][4]
+    uint32_t *h_ctr = nullptr; // pinned host mirror
+    uint32_t *srcs = nullptr;  // [S] sources of the sub-batch
+    unsigned long long *relax_cnt = nullptr;  // [S]
+    uint32_t *out_stage = nullptr, *pred_stage = nullptr;  // [S][n] when out is host memory
+    DevArena arena;
+};
+
+struct tg_graph {
+    int device = 0;
+    uint32_t n = 0;
+    uint64_t m = 0;
+    uint32_t *d_u = nullptr, *d_v = nullptr, *d_t = nullptr, *d_dur = nullptr, *d_w = nullptr;
+    uint32_t max_t = 0, max_arr = 0, min_t = 0, max_w = 0;
+    bool sp_ok = true;
+    bool built = false;
+    double build_ms = 0;
+    ChainGraph fwd, mir;
+    DevArena arena;        // input copies + chain structures
+    QueryScratch qs;
+    uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
+    // options
+    int64_t opt_sub_batch = 0;
+    int64_t opt_stats = 0;
+    int64_t opt_shortcuts = 1;
+    int64_t opt_round_group = 4;
+    // last query statistics
+    tg_query_stats last{};
+    uint64_t *last_relax = nullptr;  // host, per query
+    uint32_t last_relax_len = 0;
+};
+
+// ----------------------------------------------------------------------------- primitives
+// Exclusive prefix sum of in[0..count) into out (may alias), total -> *d_total (device, may be null).
+tg_status tg_exclusive_scan_u32(const uint32_t *in, uint32_t *out, uint64_t count, uint32_t *d_total,
+                                cudaStream_t s, DevArena *tmp_owner);
+// Stable LSD radix sort of (key, val) pairs on the low `key_bits` bits.
+tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
+                              unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s);
+
+tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, const uint32_t *u, const uint32_t *v,
+                             const uint32_t *t, const uint32_t *dur, const uint32_t *w, cudaStream_t s);
+
+tg_status tg_run_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
+                       uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
+
+// ----------------------------------------------------------------------------- device helpers
+__device__ __forceinline__ uint32_t tg_lower_bound(const uint32_t *__restrict__ a, uint32_t lo, uint32_t hi,
+                                                   uint32_t key) {
+    while (lo < hi) {
+        uint32_t mid = lo + ((hi - lo) >> 1);
+        if (__ldg(a + mid) < key) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+__device__ __forceinline__ int4 tg_ld_slot(const int4 *p) {
+    int4 r;
+    asm volatile("ld.global.nc.v4.s32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    return r;
+}
+
+static inline uint32_t tg_grid_persistent(int blocks_per_sm = 8) {
+    return 148u * (uint32_t)blocks_per_sm;
+}

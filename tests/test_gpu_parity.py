@@ -1,0 +1,256 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the oracle, element by
+element, bit-exact (all quantities are integers).
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import tgsynth
+
+pytestmark = pytest.mark.gpu
+
+NONE = 0xFFFFFFFF
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "figure1.json")
+
+
+@pytest.fixture(scope="module")
+def tg(cuda_ok):
+    import paper_conf_asplos_0003wh0dhwy0lyl25_b200 as m
+    from paper_conf_asplos_0003wh0dhwy0lyl25_b200 import _build
+    _build.build()
+    return m
+
+
+def _gpu_graph(tg, n, u, v, t, lam, w=None, **opts):
+    import torch
+    f = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.uint32).view(np.int32)).cuda()
+    g = tg.Graph(n, f(u), f(v), f(t), f(lam), None if w is None else f(w), device=0)
+    for k, val in opts.items():
+        g.set_option(k, val)
+    return g.build()
+
+
+def _check_rows(tg, g, og, problem, sources, win, with_pred=True, stats=False):
+    u32 = tg.as_u32
+    if problem in ("eat", "ld", "reach"):
+        out, pred = g.query(problem, sources, win, with_pred=True)
+    else:
+        out, pred = g.query(problem, sources, win), None
+    out = u32(out)
+    pred = u32(pred) if pred is not None else None
+    per = g.last_stats(len(sources)).get("per_query_relax") if stats else None
+    for r, x in enumerate(sources):
+        if problem == "eat":
+            A, P, W = oracle.eat(og, x, *win)
+            np.testing.assert_array_equal(out[r], A, err_msg=f"EAT x={x} win={win}")
+            np.testing.assert_array_equal(pred[r], P, err_msg=f"EAT pred x={x} win={win}")
+            if per is not None:
+                assert int(per[r]) == W, f"first-touch: relaxations {per[r]} != W {W}"
+        elif problem == "ld":
+            L, S, _ = oracle.ld(og, x, *win)
+            np.testing.assert_array_equal(out[r], L, err_msg=f"LD x={x} win={win}")
+            np.testing.assert_array_equal(pred[r], S, err_msg=f"LD succ x={x} win={win}")
+        elif problem == "reach":
+            np.testing.assert_array_equal(out[r], oracle.reach(og, x, *win))
+        elif problem == "sp":
+            np.testing.assert_array_equal(out[r], oracle.sp(og, x, *win), err_msg=f"SP x={x} win={win}")
+        elif problem == "fp":
+            np.testing.assert_array_equal(out[r], oracle.fp(og, x, *win), err_msg=f"FP x={x} win={win}")
+
+
+# --------------------------------------------------------------------------- Figure 1
+def test_figure1(tg):
+    d = json.load(open(GOLDEN))
+    ix = {s: i for i, s in enumerate(d["vertices"])}
+    E = d["edges"]
+    arr = lambda k: np.array([e[k] if k >= 2 else ix[e[k]] for e in E], np.uint32)
+    n = len(ix)
+    g = _gpu_graph(tg, n, arr(0), arr(1), arr(2), arr(3))
+    og = oracle.Graph(n, arr(0), arr(1), arr(2), arr(3))
+    for q in d["queries"]:
+        _check_rows(tg, g, og, q["problem"], [ix[q["source"]]], tuple(q["window"]))
+    ch = g.export_chains()
+    got = [ch["chain_edges"][ch["chain_off"][i]:ch["chain_off"][i + 1]].tolist() for i in range(len(ch["chain_off"]) - 1)]
+    assert got == d["chains"]["edge_sequences"]
+
+
+# --------------------------------------------------------------------------- random graphs
+@pytest.mark.parametrize("seed", range(40))
+def test_tiny_random_all_problems(tg, seed):
+    n, u, v, t, lam, w = tgsynth.tiny_random(seed, n_max=9, m_max=30, t_max=12)
+    g = _gpu_graph(tg, n, u, v, t, lam, w, stats=1)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    srcs = list(range(n))
+    for win in [(0, 100), (2, 9), (3, 3)]:
+        for p in ("eat", "ld", "reach", "sp", "fp"):
+            _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_medium_random(tg, seed):
+    rng = np.random.default_rng(seed)
+    n, m = 3000, 40000
+    u = rng.integers(0, n, m).astype(np.uint32)
+    v = rng.integers(0, n, m).astype(np.uint32)
+    t = rng.integers(0, 500, m).astype(np.uint32)
+    lam = rng.integers(1, 8, m).astype(np.uint32)
+    w = rng.integers(0, 20, m).astype(np.uint32)
+    g = _gpu_graph(tg, n, u, v, t, lam, w, stats=1, sub_batch=7)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    srcs = [int(x) for x in rng.choice(n, 24, replace=False)]
+    for win in [(0, 10**6), (100, 300)]:
+        for p in ("eat", "ld", "sp", "fp"):
+            _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
+
+
+def test_chains_match_alg1_random(tg):
+    for seed in range(20):
+        n, u, v, t, lam, w = tgsynth.tiny_random(seed + 500, n_max=40, m_max=400, t_max=30, lam_max=5)
+        g = _gpu_graph(tg, n, u, v, t, lam, w)
+        og = oracle.Graph(n, u, v, t, lam, w)
+        off, ce = oracle.chains(og)
+        sc = oracle.shortcuts(og, off, ce)
+        ch = g.export_chains()
+        np.testing.assert_array_equal(ch["chain_off"], off)
+        np.testing.assert_array_equal(ch["chain_edges"], ce)
+        for k in ("tail_v", "arr", "elapsed", "sum_w"):
+            np.testing.assert_array_equal(ch[k], sc[k], err_msg=k)
+
+
+# --------------------------------------------------------------------------- configs
+def test_c1_full(tg):
+    """configs[0]: R-MAT 2^14 V / 2^18 E, t in [0,1000), EAT from 0 (+ all problems)."""
+    ge = tgsynth.make_graph("C1")
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, w, stats=1)
+    og = oracle.Graph(n, u, v, t, d, w)
+    off, ce = oracle.chains(og)
+    ch = g.export_chains()
+    np.testing.assert_array_equal(ch["chain_off"], off)
+    np.testing.assert_array_equal(ch["chain_edges"], ce)
+    for win in tgsynth.CONFIGS["C1"]["windows"]:
+        for p in ("eat", "ld", "sp", "fp", "reach"):
+            _check_rows(tg, g, og, p, [0, 1, 17, 4000], win, stats=(p == "eat"))
+
+
+def test_c2_small_batch(tg):
+    """configs[1] shape at 1/16 scale: EAT + LD, 64-source batch, several tiles + ragged sub-batch."""
+    ge = tgsynth.make_graph("C2", scale_shift=-4)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, w, stats=1, sub_batch=24)
+    og = oracle.Graph(n, u, v, t, d, w)
+    srcs = tgsynth.config_sources("C2", ge)
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        _check_rows(tg, g, og, "eat", srcs, win, stats=True)
+        _check_rows(tg, g, og, "ld", srcs[:16], win)
+
+
+def test_c3_small_all_problems(tg):
+    """configs[2] shape at 1/16 scale: wiki-talk-shaped, all four problems."""
+    ge = tgsynth.make_graph("C3", scale_shift=-4)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, w, stats=1)
+    og = oracle.Graph(n, u, v, t, d, w)
+    srcs = tgsynth.config_sources("C3", ge)
+    for win in tgsynth.CONFIGS["C3"]["windows"]:
+        for p in ("eat", "ld", "sp", "fp"):
+            _check_rows(tg, g, og, p, srcs[:8], win, stats=(p == "eat"))
+
+
+@pytest.mark.slow
+def test_c2_full_sampled_rows(tg):
+    """configs[1] at full size in the bench's launch configuration: 64-source EAT and
+    LD batches; a seeded sample of rows is compared with the oracle row by row."""
+    import torch
+    ge = tgsynth.make_graph("C2", device="cuda")
+    g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, None, device=0).build()
+    srcs = tgsynth.config_sources("C2", ge)
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d)
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        out, pred = g.query("eat", srcs, win, with_pred=True)
+        lout, lpred = g.query("ld", srcs, win, with_pred=True)
+        torch.cuda.synchronize()
+        for r in (0, 13, 63):
+            A, P, _ = oracle.eat(og, srcs[r], *win)
+            np.testing.assert_array_equal(tg.as_u32(out[r]), A)
+            np.testing.assert_array_equal(tg.as_u32(pred[r]), P)
+            L, S, _ = oracle.ld(og, srcs[r], *win)
+            np.testing.assert_array_equal(tg.as_u32(lout[r]), L)
+            np.testing.assert_array_equal(tg.as_u32(lpred[r]), S)
+
+
+# --------------------------------------------------------------------------- edge cases
+def test_edge_cases(tg):
+    # no edges
+    g = _gpu_graph(tg, 5, np.zeros(0, np.uint32), np.zeros(0, np.uint32), np.zeros(0, np.uint32), np.zeros(0, np.uint32))
+    og = oracle.Graph(5, [], [], [], [])
+    for p in ("eat", "ld", "sp", "fp", "reach"):
+        _check_rows(tg, g, og, p, [0, 4], (0, 10))
+    # one vertex, self-loops and duplicates
+    u = np.array([0, 0, 0], np.uint32); t = np.array([1, 1, 3], np.uint32); lam = np.array([1, 1, 2], np.uint32)
+    g = _gpu_graph(tg, 1, u, u, t, lam)
+    og = oracle.Graph(1, u, u, t, lam)
+    for p in ("eat", "ld", "sp", "fp", "reach"):
+        _check_rows(tg, g, og, p, [0], (0, 10))
+
+
+def test_long_chain_and_hub(tg):
+    # a path 0 -> 1 -> ... -> L (one long chain) plus a hub with many out-edges at one time
+    L = 5000
+    u = list(range(L)); v = list(range(1, L + 1)); t = list(range(L)); lam = [1] * L
+    H = 20000
+    u += [0] * H; v += list(np.random.default_rng(0).integers(1, L + 1, H)); t += [0] * H; lam += [3] * H
+    u, v, t, lam = (np.array(a, np.uint32) for a in (u, v, t, lam))
+    g = _gpu_graph(tg, L + 1, u, v, t, lam, stats=1)
+    og = oracle.Graph(L + 1, u, v, t, lam)
+    for win in [(0, 10**6), (0, 2500), (7, 4000)]:
+        for p in ("eat", "ld", "sp", "fp"):
+            _check_rows(tg, g, og, p, [0, 1, 2500], win, stats=(p == "eat"))
+    assert g.info()["max_chain_len"] >= 2
+
+
+def test_host_and_device_buffers_agree(tg):
+    import torch
+    n, u, v, t, lam, w = tgsynth.tiny_random(7, n_max=30, m_max=300, t_max=20)
+    g = _gpu_graph(tg, n, u, v, t, lam, w)
+    srcs = list(range(min(n, 5)))
+    dev = g.query("eat", srcs, (0, 100))
+    host = torch.empty((len(srcs), n), dtype=torch.int32)
+    tg.tg_query(g.h, tg.TG_EAT, srcs, (0, 100), host)
+    assert torch.equal(dev.cpu(), host)
+
+
+def test_abi_errors_on_gpu(tg):
+    n, u, v, t, lam, w = tgsynth.tiny_random(3, n_max=5, m_max=10)
+    import torch
+    f = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.uint32).view(np.int32)).cuda()
+    with pytest.raises(tg.TGError) as e:
+        tg.Graph(n, f(u), f(np.full_like(v, n)), f(t), f(lam))
+    assert e.value.status == 2
+    with pytest.raises(tg.TGError) as e:
+        tg.Graph(n, f(u), f(v), f(t), f(np.zeros_like(lam)))
+    assert e.value.status == 1
+    big = np.full_like(t, 0x7FFFFFFE)
+    if len(t):
+        with pytest.raises(tg.TGError) as e:
+            tg.Graph(n, f(u), f(v), f(big), f(lam))
+        assert e.value.status == 2
+    g = tg.Graph(n, f(u), f(v), f(t), f(lam))
+    out = torch.empty((1, n), dtype=torch.int32, device="cuda")
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_query(g.h, tg.TG_EAT, [0], (0, 10), out)  # before build
+    assert e.value.status == 5
+    g.build()
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_query(g.h, tg.TG_EAT, [0], (10, 0), out)
+    assert e.value.status == 1
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_query(g.h, tg.TG_EAT, [n], (0, 10), out)
+    assert e.value.status == 2
+    with pytest.raises(tg.TGError) as e:
+        tg.tg_query(g.h, tg.TG_SHORTEST, [0], (0, 10), out, pred=out)
+    assert e.value.status == 1
