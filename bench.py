@@ -1,0 +1,446 @@
+#!/usr/bin/env python
+"""TempGraph on B200 -- benchmark harness (one JSON line on rank 0).
+
+Metric (BASELINE.json): EAT queries/s & temporal-edges/s at 1/2/4/8 B200, HBM
+GB/s against the peak.  Default workload = configs[1] ("C2"): R-MAT 2^20
+vertices / 16,777,216 temporal edges, t ~ U[0, 2^16), duration ~ U[1, 16],
+earliest-arrival + latest-departure batches of 64 sources, full window.
+
+A step is one pass of the whole hot path over the
+step's input: tg_graph_create from the device-resident edge arrays (validate),
+tg_build_chains (sort, departure nodes, hubs, chains, shortcuts, occurrence
+index; forward + LD mirror), then tg_query for the EAT batch and for the LD
+batch (activation, chain relaxation, rounds, extraction), then destroy.
+`value` = (queries answered by all ranks per step) / (max-over-ranks ms/step).
+
+--gpus N (under torchrun): every rank holds its own replica of the graph and
+answers its own block of 64 sources per problem (weak scaling, no data-path
+collective).  --impl reference: the oracle on host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+HBM_FALLBACK_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--k", type=int, default=None, help="sources per problem per rank (default: config)")
+    ap.add_argument("--sub-batch", type=int, default=0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-profile", action="store_true", help="do not bracket kernels with CUDA events")
+    ap.add_argument("--query-only", action="store_true", help="time only tg_query (graph built once)")
+    return ap.parse_args()
+
+
+# --------------------------------------------------------------------------- helpers
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, STREAM-style copy)"
+    return HBM_FALLBACK_GBS, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """NVML sampling of SM clock and throttle reasons during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, device_index):
+        self.samples = []
+        self.reasons = set()
+        self.max_mhz = None
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover - no NVML on CPU boxes
+            self.err = str(e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                mhz = self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM)
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.samples.append(mhz)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name not in ("gpu_idle",):
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.01)
+
+    def start(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+
+    def stop(self):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+        return {"sm_mhz": (statistics.median(self.samples) if self.samples else None),
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# --------------------------------------------------------------------------- workload
+def workload(cfg_name, k_per_rank, rank, world, device):
+    import tgsynth
+    cfg = tgsynth.CONFIGS[cfg_name]
+    ge = tgsynth.make_graph(cfg_name, device=device)
+    k = k_per_rank if k_per_rank else cfg["k"]
+    all_src = tgsynth.config_sources(cfg_name, ge, k=k * world)
+    if len(all_src) < k * world:  # small graphs: cycle
+        all_src = (all_src * (k * world // max(1, len(all_src)) + 1))[: k * world]
+    mine = all_src[rank * k:(rank + 1) * k]
+    problems = [p for p in cfg["problems"] if p in ("eat", "ld")] or ["eat"]
+    win = cfg["windows"][0]
+    weighted = cfg["kind"] == "wikitalk"
+    return ge, mine, problems, win, weighted, cfg
+
+
+def describe(cfg_name, ge, k, problems, win):
+    return (f"{cfg_name}: {ge.meta.get('config')} n={ge.n} m={ge.m}; {'+'.join(problems)} batches of {k} "
+            f"sources per rank, window [{win[0]}, {win[1]}]")
+
+
+def algorithmic_bytes(kernel, m, n, k, W):
+    """Algorithmic bytes per launch-group of a kernel."""
+    if kernel == "relax":  # activation + chain relax: slot 16 B + occ 4 B + packed atomic 8 B per relaxed slot
+        return 28 * W
+    if kernel.startswith("k_radix_scatter"):
+        return 24 * m  # read + write 12-byte (key, id) pairs
+    if kernel.startswith("k_radix_hist"):
+        return 8 * m
+    return None
+
+
+# --------------------------------------------------------------------------- our arm
+def run_ours(a, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_asplos_0003wh0dhwy0lyl25_b200 as tg
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    ge, mine, problems, win, weighted, cfg = workload(a.config, a.k, rank, world, dev)
+    k = len(mine)
+    n, m = ge.n, ge.m
+    w_arg = ge.w if weighted else None
+    outs = {p: torch.empty((k, n), dtype=torch.int32, device=dev) for p in problems}
+    torch.cuda.synchronize()
+
+    def make_graph():
+        g = tg.Graph(n, ge.u, ge.v, ge.t, ge.dur, w_arg, device=local_rank)
+        if a.sub_batch:
+            g.set_option("sub_batch", a.sub_batch)
+        return g.build()
+
+    persistent = make_graph() if a.query_only else None
+
+    def step():
+        g = persistent or make_graph()
+        for p in problems:
+            g.query(p, mine, win, out=outs[p])
+        if persistent is None:
+            g.close()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    # warm-up
+    for _ in range(max(a.warmup, 0)):
+        step()
+    torch.cuda.synchronize()
+
+    # work counts (untimed): W per query from the engine's first-touch counter (== oracle W, tested)
+    gstat = persistent or make_graph()
+    gstat.set_option("stats", 1)
+    W_by_problem = {}
+    for p in problems:
+        gstat.query(p, mine, win, out=outs[p])
+        W_by_problem[p] = int(gstat.last_stats(k)["per_query_relax"].sum())
+    rounds = {p: None for p in problems}
+    gstat.set_option("stats", 0)
+    for p in problems:
+        gstat.query(p, mine, win, out=outs[p])
+        rounds[p] = gstat.last_stats()["rounds"]
+    info = gstat.info()
+    if persistent is None:
+        gstat.close()
+    torch.cuda.synchronize()
+
+    # timed region (CUDA events on the stream all our kernels run on: the legacy default stream)
+    prof = not a.no_profile
+    sampler = ClockSampler(local_rank)
+    if prof:
+        tg.tg_profile_report()  # clear
+        tg.tg_profile_enable(True)
+    launches0 = tg.tg_kernel_launch_count()
+    barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(a.steps):
+        step()
+    e1.record()
+    torch.cuda.synchronize()
+    barrier()
+    clocks = sampler.stop()
+    launches = tg.tg_kernel_launch_count() - launches0
+    kprof = tg.tg_profile_report() if prof else {}
+    tg.tg_profile_enable(False)
+    ms = e0.elapsed_time(e1) / a.steps
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+
+    queries_per_step = k * len(problems) * world
+    value = queries_per_step / (ms / 1e3)
+
+    # roofline of the dominant kernel group
+    peak, peak_src = peaks()
+    roof = None
+    if kprof:
+        relax_names = [x for x in kprof if x.startswith(("k_eat_activate", "k_eat_big", "k_eat_chain"))]
+        relax_ms = sum(kprof[x][1] for x in relax_names)
+        relax_launches = sum(kprof[x][0] for x in relax_names)
+        dom = max(kprof.items(), key=lambda kv: kv[1][1])
+        total_kernel_ms = sum(v[1] for v in kprof.values())
+        W_total = sum(W_by_problem.values()) * a.steps
+        relax_bytes = 28 * W_total
+        roof = {
+            "bound": "hbm",
+            "kernel": "relax phase (k_eat_activate + k_eat_big + k_eat_chain: activation with inline "
+                      "one-edge-chain relax, chunked big ranges, chain engine)",
+            "achieved": relax_bytes / (relax_ms / 1e3) / 1e9 if relax_ms else None,
+            "peak": peak,
+            "unit": "GB/s",
+            "frac": (relax_bytes / (relax_ms / 1e3) / 1e9 / peak) if relax_ms else None,
+            "traffic": None,
+            "peak_source": peak_src,
+            "algorithmic_bytes_per_step": relax_bytes / a.steps,
+            "relax_ms_per_step": relax_ms / a.steps,
+            "relax_launches_per_step": relax_launches / a.steps,
+            "relax_share_of_kernel_time": relax_ms / total_kernel_ms if total_kernel_ms else None,
+            "dominant_single_kernel": dom[0],
+            "dominant_single_kernel_share": dom[1][1] / total_kernel_ms if total_kernel_ms else None,
+            "kernels_ms_per_step": {x: round(v[1] / a.steps, 4) for x, v in
+                                    sorted(kprof.items(), key=lambda kv: -kv[1][1])[:12]},
+        }
+
+    e2e = None
+    if not a.no_e2e:
+        e2e = run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev)
+
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        cpu = cpu_baseline(ge, mine, problems, win, weighted)
+
+    res = {
+        "metric": "EAT (+LD) temporal-path queries/s; temporal-edges/s and relax-phase HBM GB/s in extras",
+        "value": value,
+        "unit": "queries/s",
+        "n_gpus": world,
+        "steps": a.steps,
+        "warmup": a.warmup,
+        "ms_per_step": ms,
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "u32",
+        "data": "synthetic",
+        "config": {
+            "workload": describe(a.config, ge, k, problems, win),
+            "parallelism": f"source-sharded x{world} (replicated graph, no data-path collective)",
+            "step": "create+validate, build_chains (fwd+mirror), " + " + ".join(f"{p} x{k}" for p in problems),
+            "query_only": a.query_only,
+            "l2": "inputs larger than L2 (edge list %.0f MB, chain structure %.0f MB > 126 MB)" % (
+                m * (20 if weighted else 16) / 1e6, info["device_bytes"] / 1e6),
+            "sub_batch": a.sub_batch or "auto",
+        },
+        "teps_graph": value * m / 1.0,  # queries/s x |E|: the paper-comparable |E|-normalised rate
+        "teps_work": (sum(W_by_problem.values()) * world) / (ms / 1e3),
+        "W_per_query": {p: W_by_problem[p] / k for p in problems},
+        "rounds": rounds,
+        "graph": {"n": n, "m": m, "nodes": info["n_nodes"], "chains": info["n_chains"],
+                  "long_chains": info["n_long_chains"], "max_chain_len": info["max_chain_len"],
+                  "device_bytes": info["device_bytes"], "build_ms": info["build_ms"]},
+        "roofline": roof,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": launches,
+        "clocks": clocks,
+    }
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev):
+    """Same metric through the public C-ABI with HOST buffers: pinned host edge arrays
+    -> tg_graph_create (H2D inside) -> build -> tg_query into pinned host outputs (D2H inside)."""
+    import torch
+    n, m = ge.n, ge.m
+    k = len(mine)
+    hu, hv, ht, hd = (x.cpu().pin_memory() for x in (ge.u, ge.v, ge.t, ge.dur))
+    hw = ge.w.cpu().pin_memory() if weighted else None
+    houts = {p: torch.empty((k, n), dtype=torch.int32).pin_memory() for p in problems}
+
+    def step():
+        g = tg.Graph(n, hu, hv, ht, hd, hw, device=dev.index)
+        if a.sub_batch:
+            g.set_option("sub_batch", a.sub_batch)
+        g.build()
+        for p in problems:
+            tg.tg_query(g.h, tg.PROBLEMS[p], mine, win, houts[p])
+        g.close()
+
+    step()
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    steps = max(1, min(a.steps, 3))
+    e0.record()
+    for _ in range(steps):
+        step()
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+    h2d = m * (20 if weighted else 16) + k * 4 * len(problems)
+    d2h = len(problems) * k * n * 4
+    return {"value": k * len(problems) * world / (ms / 1e3), "unit": "queries/s", "ms_per_step": ms,
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": steps}
+
+
+# --------------------------------------------------------------------------- oracle (CPU) legs
+def _oracle_graph(ge, weighted):
+    import oracle
+    n, u, v, t, d, w = ge.numpy()
+    return oracle.Graph(n, u, v, t, d, w if weighted else None)
+
+
+def _oracle_build_seconds(og):
+    """The oracle's own preprocessing: the stable time sort its one-pass scans need
+    (EAT ascending, LD descending over the same order)."""
+    t0 = time.perf_counter()
+    _ = og.order
+    return time.perf_counter() - t0
+
+
+def cpu_baseline(ge, mine, problems, win, weighted, n_sample=2):
+    import oracle
+    og = _oracle_graph(ge, weighted)
+    t_build = _oracle_build_seconds(og)
+    per = {}
+    for p in problems:
+        ts = []
+        for x in mine[:n_sample]:
+            t0 = time.perf_counter()
+            (oracle.eat if p == "eat" else oracle.ld)(og, x, *win)
+            ts.append(time.perf_counter() - t0)
+        per[p] = statistics.mean(ts)
+    k = len(mine)
+    t_step = t_build + sum(k * per[p] for p in problems)
+    return {"value": k * len(problems) / t_step, "unit": "queries/s", "cores": 1, "kind": "oracle",
+            "sample": f"oracle preprocessing (stable numpy time sort) timed once "
+                      f"({t_build:.2f} s) + {n_sample} single-thread queries per problem "
+                      f"({', '.join(f'{p} {per[p]*1e3:.1f} ms' for p in problems)}), extrapolated to "
+                      f"the step's {k} sources per problem",
+            "host_cores_available": os.cpu_count()}
+
+
+def run_reference(a, rank, world):
+    if rank != 0:
+        return
+    import torch
+    ge, mine, problems, win, weighted, cfg = workload(a.config, a.k, 0, 1, "cpu" if not torch.cuda.is_available() else "cuda")
+    import oracle
+    og = _oracle_graph(ge, weighted)
+    t_build = _oracle_build_seconds(og)
+    k = len(mine)
+    samples = []
+    it = 0
+    for s in range(a.warmup + a.steps):
+        x = mine[it % k]
+        it += 1
+        t0 = time.perf_counter()
+        for p in problems:
+            (oracle.eat if p == "eat" else oracle.ld)(og, x, *win)
+        dt = time.perf_counter() - t0
+        if s >= a.warmup:
+            samples.append(dt)
+    per_source = statistics.mean(samples)  # one query of every problem
+    t_step = t_build + k * per_source
+    value = k * len(problems) / t_step
+    sample = (f"each step = 1 source x ({'+'.join(problems)}) single-thread oracle scans "
+              f"(mean {per_source*1e3:.1f} ms); time sort timed once ({t_build:.2f} s); value "
+              f"extrapolated to the full step of {k} sources per problem")
+    res = {"impl": "reference", "metric": "EAT (+LD) temporal-path queries/s", "value": value, "unit": "queries/s",
+           "n_gpus": world, "steps": a.steps, "warmup": a.warmup, "ms_per_step": per_source * 1e3,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+           "config": {"workload": describe(a.config, ge, k, problems, win)},
+           "cpu_baseline": {"value": value, "unit": "queries/s", "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(res), flush=True)
+
+
+def main():
+    a = parse_args()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world == 1 and a.gpus > 1:
+        print(json.dumps({"error": "use torchrun --nproc-per-node N for --gpus N > 1"}))
+        return 2
+    if a.impl == "reference":
+        run_reference(a, rank, world)
+    else:
+        run_ours(a, rank, world, local_rank)
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -186,6 +186,16 @@ TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
 /* Total kernels this library has launched in this process (all handles). */
 TG_API uint64_t tg_kernel_launch_count(void);
 
+/* Per-kernel timing for measurement: when enabled, every launch is bracketed by
+ * a CUDA event pair recorded on the launching stream.  tg_profile_report
+ * synchronises on the recorded events and folds them into a per-kernel table;
+ * with buf != NULL it writes the table as a JSON object
+ * {"kernel_name": [launches, total_ms], ...} (NUL-terminated, truncated to
+ * buf_len) and clears it; with buf == NULL it only returns the size.  Returns
+ * the length needed (incl. NUL). */
+TG_API void tg_profile_enable(int on);
+TG_API int tg_profile_report(char *buf, uint64_t buf_len);
+
 #ifdef __cplusplus
 }
 #endif

@@ -1,5 +1,7 @@
 // api.cu -- the C-ABI entry points of include/tg.h.
+#include <algorithm>
 #include <chrono>
+#include <cstdio>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -8,6 +10,32 @@
 
 uint64_t g_tg_launches = 0;
 static thread_local std::string t_err;
+
+// ----------------------------------------------------------------------------- profiling
+int g_tg_profile = 0;
+namespace {
+struct ProfRec { const char *name; cudaEvent_t e0, e1; };
+std::vector<ProfRec> g_prof;
+std::vector<cudaEvent_t> g_ev_pool;
+cudaEvent_t ev_get() {
+    if (!g_ev_pool.empty()) { cudaEvent_t e = g_ev_pool.back(); g_ev_pool.pop_back(); return e; }
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    return e;
+}
+}  // namespace
+
+cudaEvent_t tg_prof_begin(cudaStream_t s) {
+    cudaEvent_t e = ev_get();
+    cudaEventRecord(e, s);
+    return e;
+}
+
+void tg_prof_end(const char *name, cudaStream_t s, cudaEvent_t ev0) {
+    cudaEvent_t e = ev_get();
+    cudaEventRecord(e, s);
+    g_prof.push_back({name, ev0, e});
+}
 
 void tg_set_error(const std::string &msg) { t_err = msg; }
 
@@ -86,6 +114,40 @@ const char *tg_status_string(tg_status s) {
 const char *tg_last_error(void) { return t_err.c_str(); }
 
 uint64_t tg_kernel_launch_count(void) { return g_tg_launches; }
+
+void tg_profile_enable(int on) { g_tg_profile = on ? 1 : 0; }
+
+int tg_profile_report(char *buf, uint64_t buf_len) {
+    // {"kernel": [launches, total_ms], ...}.  Recorded launches are folded into a
+    // running table; a call with a buffer writes the table and clears it, a call
+    // with buf == NULL only returns the size needed.
+    struct Acc { std::string name; uint64_t n = 0; double ms = 0; };
+    static std::vector<Acc> acc;
+    for (auto &r : g_prof) {
+        cudaEventSynchronize(r.e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, r.e0, r.e1);
+        auto it = std::find_if(acc.begin(), acc.end(), [&](const Acc &p) { return p.name == r.name; });
+        if (it == acc.end()) { acc.push_back(Acc{r.name}); it = acc.end() - 1; }
+        it->n++;
+        it->ms += ms;
+        g_ev_pool.push_back(r.e0);
+        g_ev_pool.push_back(r.e1);
+    }
+    g_prof.clear();
+    std::string js = "{";
+    for (size_t i = 0; i < acc.size(); i++) {
+        char tmp[320];
+        snprintf(tmp, sizeof(tmp), "%s\"%s\": [%llu, %.6f]", i ? ", " : "", acc[i].name.c_str(),
+                 (unsigned long long)acc[i].n, acc[i].ms);
+        js += tmp;
+    }
+    js += "}";
+    if (!buf || buf_len == 0) return (int)js.size() + 1;
+    snprintf(buf, buf_len, "%s", js.c_str());
+    acc.clear();
+    return (int)js.size() + 1;
+}
 
 tg_status tg_graph_create(uint32_t n_vertices, uint64_t n_edges, const uint32_t *u, const uint32_t *v,
                           const uint32_t *t_start, const uint32_t *duration, const uint32_t *weight, int device,

@@ -33,10 +33,17 @@ extern uint64_t g_tg_launches;  // kernels launched by this library (process-wid
 
 // Launch bookkeeping: every kernel launch goes through this macro so that the
 // bench can report how many of OUR kernels ran inside its timed region.
+// With profiling enabled (tg_profile_enable) a CUDA event pair is recorded around
+// every launch on the launching stream; tg_profile_report sums them per kernel.
+extern int g_tg_profile;
+cudaEvent_t tg_prof_begin(cudaStream_t s);
+void tg_prof_end(const char *name, cudaStream_t s, cudaEvent_t ev0);
 #define TG_LAUNCH(kernel, grid, block, smem, stream, ...)                  \
     do {                                                                   \
+        cudaEvent_t _ev0 = g_tg_profile ? tg_prof_begin(stream) : nullptr; \
         kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);        \
         g_tg_launches++;                                                   \
+        if (_ev0) tg_prof_end(#kernel, stream, _ev0);                      \
         TG_TRY_CUDA(cudaGetLastError());                                   \
     } while (0)
 

@@ -26,7 +26,7 @@ TG_TMAX = 0x7FFFFFFE
 
 EXPORTED = ["tg_graph_create", "tg_build_chains", "tg_query", "tg_graph_destroy", "tg_status_string",
             "tg_last_error", "tg_graph_info", "tg_export_chains", "tg_last_query_stats", "tg_set_option",
-            "tg_kernel_launch_count"]
+            "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report"]
 
 
 class TGError(RuntimeError):
@@ -87,6 +87,10 @@ def load_library(path: str = LIB_PATH):
     lib.tg_set_option.argtypes = [P, ctypes.c_char_p, i64]
     lib.tg_kernel_launch_count.restype = u64
     lib.tg_kernel_launch_count.argtypes = []
+    lib.tg_profile_enable.restype = None
+    lib.tg_profile_enable.argtypes = [ctypes.c_int]
+    lib.tg_profile_report.restype = ctypes.c_int
+    lib.tg_profile_report.argtypes = [ctypes.c_char_p, u64]
     _lib = lib
     return lib
 
@@ -180,6 +184,20 @@ def tg_set_option(g, key: str, value: int):
 
 def tg_kernel_launch_count() -> int:
     return int(load_library().tg_kernel_launch_count())
+
+
+def tg_profile_enable(on: bool = True):
+    load_library().tg_profile_enable(1 if on else 0)
+
+
+def tg_profile_report() -> dict:
+    """{kernel: (launches, total_ms)} of the launches recorded since the last report."""
+    import json
+    lib = load_library()
+    need = lib.tg_profile_report(None, 0)
+    buf = ctypes.create_string_buffer(max(need, 2) + 4096)
+    lib.tg_profile_report(buf, len(buf))
+    return {k: (int(v[0]), float(v[1])) for k, v in json.loads(buf.value.decode()).items()}
 
 
 # --------------------------------------------------------------------------- convenience

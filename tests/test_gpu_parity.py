@@ -225,7 +225,9 @@ def test_host_and_device_buffers_agree(tg):
 
 
 def test_abi_errors_on_gpu(tg):
-    n, u, v, t, lam, w = tgsynth.tiny_random(3, n_max=5, m_max=10)
+    n = 5
+    u = np.array([0, 1, 2, 3], np.uint32); v = np.array([1, 2, 3, 4], np.uint32)
+    t = np.array([1, 2, 3, 4], np.uint32); lam = np.array([1, 1, 1, 1], np.uint32)
     import torch
     f = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.uint32).view(np.int32)).cuda()
     with pytest.raises(tg.TGError) as e:
