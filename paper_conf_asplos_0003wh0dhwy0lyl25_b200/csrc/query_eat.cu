@@ -6,25 +6,30 @@
 //
 // state    st[q][v] = (arrival << 32 | pred edge id), relaxed with 64-bit atomicMin,
 //          so the min word carries EAT and the smallest optimal edge id (reading A9).
+//          A plain (possibly stale, hence conservative) read filters relaxations
+//          that cannot improve before any atomic is issued.
 // frontier (q, u) items whose arrival improved in the previous round.
-// Activate (k_eat_activate, the "skeleton engine"): for an improved vertex u
-//          (old -> new arrival), the out-edges of u departing in [max(new, alpha),
-//          old) become usable for the first time.  They are found by binary search
-//          in u's departure nodes and expanded warp-cooperatively (warp scan +
-//          shuffle binary search); large ranges are split into chunks
-//          (k_eat_big).  For each newly usable occurrence:
-//            one-edge chain  -> relaxed at once (RemoveChain: 2-vertex
-//                               chains are done by the skeleton engine);
-//            longer chain    -> atomicMin on the chain's entry position per query;
-//                               on the first entry the tail is relaxed through
-//                               the shortcut (Alg. 2; Propagate(S_l), Alg. 3
-//                               line 6); the newly entered slots [pos, old) are
-//                               walked inline when short, else queued.
-// Compute  (k_eat_chain, the "chain engine"): one warp per queued chain segment,
-//          lanes over consecutive 16-byte slots (coalesced 512 B per step).
-// Every usable valid slot is relaxed exactly once per query ("first touch"):
-// activation ranges of a vertex are disjoint over rounds and chain entries only
-// move backwards, so slot visits == the one-pass work count W.
+// Activate (k_eat_activate, the "skeleton engine"): for an improved vertex u the
+//          out-edges of u departing in [max(new, alpha), previous boundary) become
+//          usable for the first time.  The boundary is kept as an edge index
+//          act[q][u] (one binary search per activation).  Ranges are expanded
+//          warp-cooperatively (warp scan + shuffle binary search); large ranges
+//          are split into chunks (k_eat_big).  For each newly usable occurrence:
+//            one-edge chain -> relaxed at once (RemoveChain: 2-vertex
+//                              chains are done by the skeleton engine);
+//            longer chain   -> the slot is claimed (test-and-set of its bit in
+//                              claimed[q][slot]; position 0 needs no bit: it is
+//                              only ever reached through its own occurrence),
+//                              the tail is relaxed through the shortcut
+//                              (Propagate(S_l), Alg. 3 line 6) and the chain is
+//                              walked forward claiming slot after slot.  A walker
+//                              stops at the first slot somebody else claimed --
+//                              that claimer continues -- or past omega.
+// Compute  (k_eat_chain, the "chain engine"): one warp per long walk, lanes over
+//          consecutive 16-byte slots (coalesced 512 B per step); it continues
+//          iff its last lane claimed its slot.
+// First touch: every usable valid slot is relaxed exactly once per query, so the
+// relaxation count equals the one-pass work count W (tested).
 #include <cooperative_groups.h>
 
 #include <algorithm>
@@ -39,7 +44,7 @@ namespace {
 constexpr int QT = 256;                 // threads per block
 constexpr uint32_t BIG_T = 256;         // ranges above this are split into chunks
 constexpr uint32_t CHUNK = 1024;        // edges per chunk (one warp)
-constexpr uint32_t INLINE_WALK = 16;    // chain segments up to this length are walked inline
+constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in the activating thread
 
 struct EatP {
     const uint32_t *vnode_off, *node_t, *node_eoff, *occ_slot;
@@ -47,88 +52,135 @@ struct EatP {
     const uint2 *lc;
     const int4 *sc;
     unsigned long long *st;
-    uint32_t *act, *mark, *entry;
+    uint32_t *act, *mark, *bits;
+    uint64_t bit_words;
     uint32_t n;
-    uint64_t nlong;
-    uint32_t alpha, omega, stamp;
+    uint32_t alpha, omega;
     int use_sc, stats;
-    const unsigned long long *fin;
-    const uint32_t *fin_cnt;
-    unsigned long long *fout;
-    uint32_t *fout_cnt;
+    RoundCtl *ctl;
+    unsigned long long *fr0, *fr1;
     uint4 *bigq;
-    uint32_t *big_cnt;
     uint64_t bigcap;
     uint4 *chq;
-    uint32_t *ch_cnt;
     uint64_t chcap;
     unsigned long long *relax_cnt;
 };
 
-__device__ __forceinline__ void eat_relax(const EatP &P, uint32_t q, uint32_t v, uint32_t arr, uint32_t id) {
-    const size_t i = (size_t)q * P.n + v;
-    const unsigned long long pk = ((unsigned long long)arr << 32) | id;
-    const unsigned long long old = atomicMin(P.st + i, pk);
-    if (P.stats) atomicAdd(P.relax_cnt + q, 1ull);
-    if (arr < (uint32_t)(old >> 32)) {
-        if (atomicExch(P.mark + i, P.stamp) != P.stamp) {
-            cg::coalesced_group g = cg::coalesced_threads();
-            uint32_t base = 0;
-            if (g.thread_rank() == 0) base = atomicAdd(P.fout_cnt, g.size());
-            base = g.shfl(base, 0);
-            P.fout[base + g.thread_rank()] = ((unsigned long long)q << 32) | v;
+// per-round view derived from the device-side round control
+struct RoundV {
+    uint32_t stamp;
+    const unsigned long long *fin;
+    uint32_t fin_n;
+    unsigned long long *fout;
+    uint32_t *fout_cnt, *big_cnt, *ch_cnt;
+};
+
+__device__ __forceinline__ RoundV round_view(const EatP &P) {
+    RoundV R;
+    const uint32_t r = *(volatile uint32_t *)&P.ctl->round;
+    R.stamp = *(volatile uint32_t *)&P.ctl->stamp;
+    R.fin = (r & 1) ? P.fr1 : P.fr0;
+    R.fout = (r & 1) ? P.fr0 : P.fr1;
+    R.fin_n = *(volatile uint32_t *)&P.ctl->cnt[r & 3][0];
+    R.fout_cnt = &P.ctl->cnt[(r + 1) & 3][0];
+    R.big_cnt = &P.ctl->cnt[r & 3][1];
+    R.ch_cnt = &P.ctl->cnt[r & 3][2];
+    return R;
+}
+
+// The last block to finish the round's last kernel advances the round.
+__device__ __forceinline__ void round_advance(RoundCtl *ctl) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const uint32_t d = atomicAdd(&ctl->done_blocks, 1u);
+        if (d == gridDim.x - 1) {
+            const uint32_t r = ctl->round;
+            for (int i = 0; i < 4; i++) ctl->cnt[(r + 2) & 3][i] = 0;
+            ctl->cnt[(r + 1) & 3][1] = 0;
+            ctl->cnt[(r + 1) & 3][2] = 0;
+            ctl->done_blocks = 0;
+            ctl->stamp = ctl->stamp + 1;
+            ctl->round = r + 1;
+            __threadfence();
         }
     }
 }
 
-// relax chain slots [s_begin, s_end) sequentially (stop at the window end)
-__device__ __forceinline__ void eat_walk(const EatP &P, uint32_t q, uint32_t s_begin, uint32_t s_end) {
-    for (uint32_t s = s_begin; s < s_end; s++) {
-        int4 sl = tg_ld_slot(P.slots + s);
-        if ((uint32_t)sl.y > P.omega) break;  // arrivals increase strictly along a chain
-        eat_relax(P, q, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+__device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t v, uint32_t arr,
+                                          uint32_t id) {
+    const size_t i = (size_t)q * P.n + v;
+    const unsigned long long pk = ((unsigned long long)arr << 32) | id;
+    if (P.stats) atomicAdd(P.relax_cnt + q, 1ull);
+    // States only decrease: a stale cached read is an upper bound, so when it is
+    // already <= pk the atomic cannot change anything (most relaxations, W >> n).
+    if (P.st[i] <= pk) return;
+    const unsigned long long old = atomicMin(P.st + i, pk);
+    if (arr < (uint32_t)(old >> 32)) {
+        if (atomicExch(P.mark + i, R.stamp) != R.stamp) {
+            cg::coalesced_group g = cg::coalesced_threads();
+            uint32_t base = 0;
+            if (g.thread_rank() == 0) base = atomicAdd(R.fout_cnt, g.size());
+            base = g.shfl(base, 0);
+            R.fout[base + g.thread_rank()] = ((unsigned long long)q << 32) | v;
+        }
+    }
+}
+
+// test-and-set of slot s's claim bit for query q; true if this caller claimed it
+__device__ __forceinline__ bool claim(const EatP &P, uint32_t q, uint32_t s) {
+    const uint32_t bit = 1u << (s & 31);
+    return (atomicOr(P.bits + (size_t)q * P.bit_words + (s >> 5), bit) & bit) == 0;
+}
+
+// sequential walk over slots [s, s_end): claim, relax, continue; stop at a slot
+// somebody else claimed (they continue) or past omega.
+__device__ __forceinline__ void eat_walk(const EatP &P, const RoundV &R, uint32_t q, uint32_t s, uint32_t s_end) {
+    for (; s < s_end; s++) {
+        const int4 sl = tg_ld_slot(P.slots + s);
+        if ((uint32_t)sl.y > P.omega) return;  // arrivals increase strictly along a chain
+        if (!claim(P, q, s)) return;
+        eat_relax(P, R, q, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     }
 }
 
 // A newly usable occurrence p (sorted-edge position) for query q.
-__device__ __forceinline__ void eat_edge(const EatP &P, uint32_t q, uint32_t p) {
+__device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_t q, uint32_t p) {
     const uint32_t s = __ldg(P.occ_slot + p);
     const int4 sl = tg_ld_slot(P.slots + s);
     const uint32_t arr = (uint32_t)sl.y;
     if (arr > P.omega) return;
     if ((uint32_t)sl.w == TG_SINGLE) {
-        eat_relax(P, q, (uint32_t)sl.x, arr, (uint32_t)sl.z);
+        eat_relax(P, R, q, (uint32_t)sl.x, arr, (uint32_t)sl.z);
         return;
     }
     const uint32_t l = (uint32_t)sl.w;
     const uint2 info = __ldg(P.lc + l);  // {first slot, length}
-    const uint32_t pos = s - info.x;
-    const uint32_t old = atomicMin(P.entry + (size_t)q * P.nlong + l, pos);
-    if (pos >= old) return;  // already entered at or before pos
-    uint32_t end = min(old, info.y);
-    if (old == TG_NONE && P.use_sc) {
-        // first entry: Propagate along the shortcut head -> tail (Alg. 3 line 6)
+    if (s != info.x && !claim(P, q, s)) return;  // a walker from an earlier entry got here first
+    eat_relax(P, R, q, (uint32_t)sl.x, arr, (uint32_t)sl.z);
+    uint32_t s_end = info.x + info.y;
+    if (s + 1 >= s_end) return;
+    if (P.use_sc) {
+        // skeleton: Propagate along the shortcut head -> tail (Alg. 2 / Alg. 3 line 6)
         const int4 scv = __ldg(P.sc + l);
-        if ((uint32_t)scv.y <= P.omega) {
-            eat_relax(P, q, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
-            end = info.y - 1;
+        if ((uint32_t)scv.y <= P.omega && claim(P, q, s_end - 1)) {
+            eat_relax(P, R, q, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
+            s_end -= 1;
         }
     }
-    if (pos >= end) return;
-    eat_relax(P, q, (uint32_t)sl.x, arr, (uint32_t)sl.z);
-    const uint32_t s1 = info.x + end;
-    if (s1 - (s + 1) > INLINE_WALK) {
-        uint32_t k = atomicAdd(P.ch_cnt, 1u);
+    if (s_end - (s + 1) > INLINE_WALK) {
+        const uint32_t k = atomicAdd(R.ch_cnt, 1u);
         if (k < P.chcap) {
-            P.chq[k] = make_uint4(q, s + 1, s1, 0);
+            P.chq[k] = make_uint4(q, s + 1, s_end, 0);
             return;
         }
     }
-    eat_walk(P, q, s + 1, s1);
+    eat_walk(P, R, q, s + 1, s_end);
 }
 
 __global__ void __launch_bounds__(QT) k_eat_activate(EatP P) {
-    const uint32_t F = *P.fin_cnt;
+    const RoundV R = round_view(P);
+    const uint32_t F = R.fin_n;
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
@@ -136,31 +188,31 @@ __global__ void __launch_bounds__(QT) k_eat_activate(EatP P) {
         const uint32_t i = base + lane;
         uint32_t q = 0, e0 = 0, cnt = 0;
         if (i < F) {
-            const unsigned long long it = P.fin[i];
+            const unsigned long long it = R.fin[i];
             q = (uint32_t)(it >> 32);
             const uint32_t u = (uint32_t)it;
             const size_t si = (size_t)q * P.n + u;
             const uint32_t now = (uint32_t)(__ldcg(P.st + si) >> 32);
-            const uint32_t old = atomicMin(P.act + si, now);
-            if (now < old) {
-                const uint32_t lo_t = max(now, P.alpha);
-                const uint32_t hi_t = min(old, P.omega);  // t + duration <= omega needs t < omega
-                if (lo_t < hi_t) {
-                    const uint32_t a = __ldg(P.vnode_off + u), b = __ldg(P.vnode_off + u + 1);
-                    const uint32_t j0 = tg_lower_bound(P.node_t, a, b, lo_t);
-                    const uint32_t j1 = tg_lower_bound(P.node_t, j0, b, hi_t);
-                    e0 = __ldg(P.node_eoff + j0);
-                    cnt = __ldg(P.node_eoff + j1) - e0;
-                }
+            const uint32_t a = __ldg(P.vnode_off + u), b = __ldg(P.vnode_off + u + 1);
+            const uint32_t lo_t = max(now, P.alpha);
+            const uint32_t j0 = tg_lower_bound(P.node_t, a, b, lo_t);
+            const uint32_t elo = __ldg(P.node_eoff + j0);
+            // previous boundary: edges at index >= act were activated before; the first
+            // activation starts from the window end (t + duration <= omega needs t < omega)
+            const uint32_t prev = atomicMin(P.act + si, elo);
+            if (elo < prev) {
+                uint32_t ehi = prev;
+                if (prev == TG_NONE) ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, j0, b, P.omega));
+                if (elo < ehi) { e0 = elo; cnt = ehi - elo; }
             }
         }
         if (cnt > BIG_T) {
             const uint32_t nch = (cnt + CHUNK - 1) / CHUNK;
-            const uint32_t k = atomicAdd(P.big_cnt, nch);
+            const uint32_t k = atomicAdd(R.big_cnt, nch);
             for (uint32_t c = 0; c < nch; c++) {
                 const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
                 if (k + c < P.bigcap) P.bigq[k + c] = make_uint4(q, b0, b1, 0);
-                else for (uint32_t p = b0; p < b1; p++) eat_edge(P, q, p);  // never expected: bigcap is a bound
+                else for (uint32_t p = b0; p < b1; p++) eat_edge(P, R, q, p);  // bigcap is a bound
             }
             cnt = 0;
         }
@@ -176,33 +228,37 @@ __global__ void __launch_bounds__(QT) k_eat_activate(EatP P) {
             const uint32_t g = gb + lane;
             uint32_t own = 0;  // number of lanes whose inclusive prefix <= g == owner lane
 #pragma unroll
-            for (int b = 16; b; b >>= 1) {
-                const uint32_t v = __shfl_sync(0xffffffffu, incl, own + b - 1);
-                if (v <= g) own += b;
+            for (int bb = 16; bb; bb >>= 1) {
+                const uint32_t v = __shfl_sync(0xffffffffu, incl, own + bb - 1);
+                if (v <= g) own += bb;
             }
             own &= 31;
             const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
             const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
             const uint32_t oq = __shfl_sync(0xffffffffu, q, own);
-            if (g < total) eat_edge(P, oq, oe0 + (g - oex));
+            if (g < total) eat_edge(P, R, oq, oe0 + (g - oex));
         }
     }
 }
 
 __global__ void __launch_bounds__(QT) k_eat_big(EatP P) {
-    const uint32_t B = (uint32_t)min((uint64_t)*P.big_cnt, P.bigcap);
+    const RoundV R = round_view(P);
+    const uint32_t B = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.big_cnt, P.bigcap);
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
-        for (uint32_t p = c.y + lane; p < c.z; p += 32) eat_edge(P, c.x, p);
+        for (uint32_t p = c.y + lane; p < c.z; p += 32) eat_edge(P, R, c.x, p);
     }
 }
 
-// ChainEngine: warp per queued chain segment, lanes over consecutive slots.
+// ChainEngine: warp per queued walk, lanes over consecutive slots; the warp
+// continues iff its last lane claimed its slot (otherwise that slot's claimer
+// continues the chain).  Advances the round when the last block finishes.
 __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
-    const uint32_t C = (uint32_t)min((uint64_t)*P.ch_cnt, P.chcap);
+    const RoundV R = round_view(P);
+    const uint32_t C = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.ch_cnt, P.chcap);
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
@@ -210,25 +266,40 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
         const uint4 c = P.chq[it];
         for (uint32_t b = c.y; b < c.z; b += 32) {
             const uint32_t s = b + lane;
-            bool stop = false;
+            bool cont = false, past = false;
             if (s < c.z) {
                 const int4 sl = tg_ld_slot(P.slots + s);
-                if ((uint32_t)sl.y > P.omega) stop = true;
-                else eat_relax(P, c.x, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+                if ((uint32_t)sl.y > P.omega) {
+                    past = true;
+                } else if (claim(P, c.x, s)) {
+                    eat_relax(P, R, c.x, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+                    cont = true;
+                }
             }
-            if (__any_sync(0xffffffffu, stop)) break;
+            const uint32_t last = min(31u, c.z - 1 - b);
+            const bool go_on = __shfl_sync(0xffffffffu, cont, last);
+            if (__any_sync(0xffffffffu, past) || !go_on) break;
         }
     }
+    round_advance(P.ctl);
 }
 
+// VInitial (Table 1): every state INF (memset), the source = (alpha, no pred),
+// frontier = the sources; round control reset for a new loop.
 __global__ void k_eat_init(unsigned long long *st, uint32_t n, const uint32_t *srcs, uint32_t S, uint32_t alpha,
-                           unsigned long long *fr, uint32_t *fr_cnt, int push) {
-    // VInitial (Table 1): every state INF (memset), the source = (alpha, no pred)
+                           unsigned long long *fr1, RoundCtl *ctl, int push) {
     for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < S; q += gridDim.x * blockDim.x) {
         st[(size_t)q * n + srcs[q]] = ((unsigned long long)alpha << 32) | TG_NONE;
-        if (push) fr[q] = ((unsigned long long)q << 32) | srcs[q];
+        if (push) fr1[q] = ((unsigned long long)q << 32) | srcs[q];
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) *fr_cnt = push ? S : 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        for (int i = 0; i < 4; i++)
+            for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
+        ctl->cnt[1][0] = push ? S : 0;
+        ctl->round = 1;
+        ctl->done_blocks = 0;
+        ctl->stamp = ctl->stamp + 1;  // stamps only grow: marks from earlier loops never match
+    }
 }
 
 // mode 0 = EAT, 1 = LD (mirror: value = C - time; target = omega), 2 = REACH
@@ -260,16 +331,14 @@ __global__ void k_eat_extract(const unsigned long long *__restrict__ st, uint32_
 
 static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     QueryScratch &Q = g->qs;
-    const uint64_t nlong = std::max(g->fwd.nlong, g->mir.nlong);
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
-    if (Q.S >= S && Q.n == g->n && Q.nlong >= nlong && (!nodes_state || Q.nodes_state)) return TG_OK;
+    if (Q.S >= S && Q.n == g->n && (!nodes_state || Q.nodes_state)) return TG_OK;
     Q.arena.free_all();
     if (Q.h_ctr) { cudaFreeHost(Q.h_ctr); Q.h_ctr = nullptr; }
     Q = QueryScratch{};
     const uint64_t n = g->n, m = g->m;
     Q.S = S;
     Q.n = g->n;
-    Q.nlong = nlong;
     Q.nnodes = nnodes;
     Q.nodes_state = nodes_state;
     DevArena &A = Q.arena;
@@ -278,17 +347,20 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     const uint64_t mark_len = S * std::max<uint64_t>(n, nodes_state ? nnodes : 0);
     TG_TRY(A.alloc((void **)&Q.mark, mark_len * 4));
     TG_TRY_CUDA(cudaMemset(Q.mark, 0, mark_len * 4));
-    TG_TRY(A.alloc((void **)&Q.entry, std::max<uint64_t>(S * nlong, 1) * 4));
+    Q.bit_words = (m + 31) / 32 + 1;
+    TG_TRY(A.alloc((void **)&Q.bits, S * Q.bit_words * 4));
     Q.fcap = S * std::max<uint64_t>(n, nodes_state ? nnodes : 0) + 64;
     TG_TRY(A.alloc((void **)&Q.fr[0], Q.fcap * 8));
     TG_TRY(A.alloc((void **)&Q.fr[1], Q.fcap * 8));
     Q.bigcap = S * (m / CHUNK + std::max<uint64_t>(n, nnodes) / BIG_T + 2) + 1024;
     TG_TRY(A.alloc((void **)&Q.bigq, Q.bigcap * 16));
-    Q.chcap = S * nlong + (1u << 20);
+    Q.chcap = S * (m / (INLINE_WALK + 1)) + (1u << 16);
     TG_TRY(A.alloc((void **)&Q.chq, Q.chcap * 16));
     TG_TRY(A.alloc((void **)&Q.ctr, 64));
     TG_TRY_CUDA(cudaMemset(Q.ctr, 0, 64));
-    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 64));
+    TG_TRY(A.alloc((void **)&Q.ctl, sizeof(RoundCtl)));
+    TG_TRY_CUDA(cudaMemset(Q.ctl, 0, sizeof(RoundCtl)));
+    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
     TG_TRY(A.alloc((void **)&Q.srcs, S * 4));
     TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8));
     if (nodes_state) {
@@ -298,16 +370,17 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     return TG_OK;
 }
 
+// Sub-batch size: the hot per-query state (packed states, activation boundary,
+// frontier stamps, claim bits) of a sub-batch should stay resident in the 126 MB L2.
 uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
     if (g->opt_sub_batch > 0) return (uint32_t)std::min<int64_t>(g->opt_sub_batch, k);
     const uint64_t n = g->n;
-    const uint64_t nlong = std::max(g->fwd.nlong, g->mir.nlong);
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
-    uint64_t per = n * (8 + 4 + 4 + 16) + nlong * (4 + 16) + g->m / CHUNK * 16 + 64;
-    if (nodes_state) per += nnodes * (4 + 4 + 16) + n * 4;
-    const uint64_t budget = 6ull << 30;  // device bytes for per-query state
-    uint64_t S = std::max<uint64_t>(1, budget / per);
-    S = std::min<uint64_t>(S, 256);
+    uint64_t hot = n * (8 + 4 + 4) + g->m / 8 + 64;
+    if (nodes_state) hot = nnodes * (4 + 4) + n * 4 + 64;
+    const uint64_t budget = 64ull << 20;
+    uint64_t S = std::max<uint64_t>(1, budget / hot);
+    S = std::min<uint64_t>(S, 64);
     return (uint32_t)std::min<uint64_t>(S, k);
 }
 
@@ -320,47 +393,34 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     const uint64_t n = g->n;
     TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, S * n * 8, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, S * n * 4, s));
-    if (cgr.nlong) TG_TRY_CUDA(cudaMemsetAsync(Q.entry, 0xFF, S * cgr.nlong * 4, s));
+    TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, S * Q.bit_words * 4, s));
     if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8, s));
     const bool work = any_work && g->m > 0 && alpha < omega;
-    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, Q.srcs, S, alpha, Q.fr[1], Q.ctr + 4, work ? 1 : 0);
+    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, Q.srcs, S, alpha, Q.fr[1], Q.ctl, work ? 1 : 0);
     uint32_t rounds = 0;
     if (work) {
         EatP P{};
         P.vnode_off = cgr.vnode_off; P.node_t = cgr.node_t; P.node_eoff = cgr.node_eoff; P.occ_slot = cgr.occ_slot;
         P.slots = cgr.slots; P.lc = cgr.lc; P.sc = cgr.sc;
-        P.st = Q.st; P.act = Q.act; P.mark = Q.mark; P.entry = Q.entry;
-        P.n = g->n; P.nlong = cgr.nlong; P.alpha = alpha; P.omega = omega;
+        P.st = Q.st; P.act = Q.act; P.mark = Q.mark; P.bits = Q.bits; P.bit_words = Q.bit_words;
+        P.n = g->n; P.alpha = alpha; P.omega = omega;
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
+        P.ctl = Q.ctl; P.fr0 = Q.fr[0]; P.fr1 = Q.fr[1];
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         const uint32_t grid = tg_grid_persistent(8);
         const int group = (int)std::max<int64_t>(1, g->opt_round_group);
-        uint32_t r = 1;
         for (;;) {
-            for (int k = 0; k < group; k++, r++) {
-                const int in = r & 1, outp = (r + 1) & 1;
-                // counters: ctr[par*4 + 0] = frontier count of buffer par; [1] big; [2] chain
-                TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + outp * 4, 0, 4, s));
-                TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + in * 4 + 1, 0, 8, s));
-                if (++g->qs_epoch == 0) {  // stamp wrapped: clear marks
-                    TG_TRY_CUDA(cudaMemsetAsync(Q.mark, 0, (uint64_t)Q.S * n * 4, s));
-                    g->qs_epoch = 1;
-                }
-                P.stamp = g->qs_epoch;
-                P.fin = Q.fr[in]; P.fin_cnt = Q.ctr + in * 4;
-                P.fout = Q.fr[outp]; P.fout_cnt = Q.ctr + outp * 4;
-                P.big_cnt = Q.ctr + in * 4 + 1; P.ch_cnt = Q.ctr + in * 4 + 2;
+            for (int k = 0; k < group; k++) {
                 TG_LAUNCH(k_eat_activate, grid, QT, 0, s, P);
                 TG_LAUNCH(k_eat_big, grid, QT, 0, s, P);
                 TG_LAUNCH(k_eat_chain, grid, QT, 0, s, P);
             }
-            // r is the next round; its input count is ctr[(r & 1) * 4]
-            TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctr, 32, cudaMemcpyDeviceToHost, s));
+            TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
-            if (Q.h_ctr[(r & 1) * 4] == 0) break;
-            if (r > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
+            const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
+            if (h->cnt[h->round & 3][0] == 0) { rounds = h->round - 1; break; }
+            if (h->round > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
         }
-        rounds = r - 1;
     }
     *rounds_out = rounds;
     return TG_OK;

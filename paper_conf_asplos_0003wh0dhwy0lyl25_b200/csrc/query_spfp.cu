@@ -79,15 +79,18 @@ __device__ void spfp_walk(const SpP &P, uint32_t q, uint32_t s, uint32_t s_end, 
         const uint32_t arr = (uint32_t)sl.y;
         if (arr > P.omega) return;
         uint32_t cand;
+        uint32_t val;
         if (FP) {
-            cand = cur;                                    // latest start is preserved along the path
-            atomicMin(vo + sl.x, arr - (0xFFFFFFFEu - cur));  // duration = end - start (reading A6)
+            cand = cur;                          // latest start is preserved along the path
+            val = arr - (0xFFFFFFFEu - cur);     // duration = end - start (reading A6)
         } else {
-            cand = cur + __ldg(P.slot_w + s);              // Propagate: src + w
-            atomicMin(vo + sl.x, cand);
+            cand = cur + __ldg(P.slot_w + s);    // Propagate: src + w
+            val = cand;
         }
+        if (vo[sl.x] > val) atomicMin(vo + sl.x, val);  // stale read is an upper bound
         const uint32_t tn = __ldg(P.slot_tn + s);
         if (tn == TG_NONE) return;  // sink
+        if (dn[tn] <= cand) return;  // not improved (stale read is an upper bound)
         const uint32_t old = atomicMin(dn + tn, cand);
         if (cand >= old) return;    // not improved: the improver pushed tn
         push_node(P, q, tn);        // wait propagation + other out-edges next round

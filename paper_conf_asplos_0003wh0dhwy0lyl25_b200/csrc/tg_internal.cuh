@@ -86,6 +86,19 @@ struct ChainGraph {
     uint32_t *chain_first = nullptr;
 };
 
+// Device-side round control of one GAC loop (no host round trip per round):
+// round r reads frontier buffer r&1 with count cnt[r&3][0], appends to buffer
+// (r+1)&1 / cnt[(r+1)&3][0]; cnt[r&3][1..2] count big chunks / chain walks.  The
+// last block of a round's last kernel advances `round`, bumps `stamp` and clears
+// the ring slots the next round will write.
+struct RoundCtl {
+    uint32_t round;
+    uint32_t stamp;
+    uint32_t done_blocks;
+    uint32_t pad;
+    uint32_t cnt[4][4];
+};
+
 struct QueryScratch {
     uint32_t S = 0;          // sources per sub-batch this scratch was sized for
     uint32_t n = 0;
@@ -95,7 +108,8 @@ struct QueryScratch {
     unsigned long long *st = nullptr;  // [S][n] packed (time << 32 | pred)
     uint32_t *act = nullptr;           // [S][n] last activated time
     uint32_t *mark = nullptr;          // [S][n] (EAT) or [S][nnodes] (SP/FP) frontier dedupe stamp
-    uint32_t *entry = nullptr;         // [S][nlong] first entered position per long chain
+    uint32_t *bits = nullptr;          // [S][ceil(m/32)] "slot relaxed" bits (interior slots of long chains)
+    uint64_t bit_words = 0;            // words per query
     uint32_t *dnode = nullptr;         // [S][nnodes] SP/FP node state
     uint32_t *vout = nullptr;          // [S][n] SP/FP per-vertex output
     unsigned long long *fr[2] = {nullptr, nullptr};  // frontier items (q << 32 | vertex-or-node)
@@ -104,7 +118,8 @@ struct QueryScratch {
     uint64_t bigcap = 0;
     uint4 *chq = nullptr;    // long chain walks {q, s_begin, s_end, -}
     uint64_t chcap = 0;
-    uint32_t *ctr = nullptr;   // counters [2][4]
+    uint32_t *ctr = nullptr;   // counters [2][4] (SP/FP host-driven loop)
+    struct RoundCtl *ctl = nullptr;  // device-side round control (EAT family)
     uint32_t *h_ctr = nullptr; // pinned host mirror
     uint32_t *srcs = nullptr;  // [S] sources of the sub-batch
     unsigned long long *relax_cnt = nullptr;  // [S]

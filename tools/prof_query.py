@@ -1,0 +1,41 @@
+"""Profiling driver: build a config graph once and run query batches (for ncu).
+
+    python tools/prof_query.py --config C2 --problem eat --k 64 --reps 1
+"""
+import argparse
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import tgsynth  # noqa: E402
+import paper_conf_asplos_0003wh0dhwy0lyl25_b200 as tg  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="C2")
+ap.add_argument("--problem", default="eat")
+ap.add_argument("--k", type=int, default=64)
+ap.add_argument("--reps", type=int, default=1)
+ap.add_argument("--sub-batch", type=int, default=0)
+ap.add_argument("--shortcuts", type=int, default=1)
+a = ap.parse_args()
+
+ge = tgsynth.make_graph(a.config, device="cuda")
+cfg = tgsynth.CONFIGS[a.config]
+w = ge.w if cfg["kind"] == "wikitalk" else None
+g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, w, device=0).build()
+if a.sub_batch:
+    g.set_option("sub_batch", a.sub_batch)
+g.set_option("shortcuts", a.shortcuts)
+src = tgsynth.config_sources(a.config, ge, k=a.k)
+win = cfg["windows"][0]
+out = torch.empty((len(src), ge.n), dtype=torch.int32, device="cuda")
+for i in range(a.reps):
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    g.query(a.problem, src, win, out=out)
+    torch.cuda.synchronize()
+    print(f"rep {i}: {(time.perf_counter() - t0) * 1e3:.2f} ms  stats={g.last_stats()}", flush=True)
