@@ -33,6 +33,8 @@
 #include <cooperative_groups.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 #include "tg_internal.cuh"
@@ -52,13 +54,13 @@ struct EatP {
     const uint2 *lc;
     const int4 *sc;
     unsigned long long *st;
-    uint32_t *act, *mark, *bits;
+    uint32_t *act, *bits;
     uint64_t bit_words;
-    uint32_t n;
+    uint32_t n, S, vwords;
     uint32_t alpha, omega;
     int use_sc, stats;
     RoundCtl *ctl;
-    unsigned long long *fr0, *fr1;
+    uint32_t *fb0, *fb1;  // dense frontier bitmaps [S][vwords], by round parity
     uint4 *bigq;
     uint64_t bigcap;
     uint4 *chq;
@@ -68,23 +70,22 @@ struct EatP {
 
 // per-round view derived from the device-side round control
 struct RoundV {
-    uint32_t stamp;
-    const unsigned long long *fin;
+    uint32_t *fin;   // this round's frontier bitmap (consumed: words are cleared)
     uint32_t fin_n;
-    unsigned long long *fout;
-    uint32_t *fout_cnt, *big_cnt, *ch_cnt;
+    uint32_t *fout;  // next round's frontier bitmap
+    uint32_t *fout_cnt, *big_cnt, *ch_cnt, *words_cnt;
 };
 
 __device__ __forceinline__ RoundV round_view(const EatP &P) {
     RoundV R;
     const uint32_t r = *(volatile uint32_t *)&P.ctl->round;
-    R.stamp = *(volatile uint32_t *)&P.ctl->stamp;
-    R.fin = (r & 1) ? P.fr1 : P.fr0;
-    R.fout = (r & 1) ? P.fr0 : P.fr1;
+    R.fin = (r & 1) ? P.fb1 : P.fb0;
+    R.fout = (r & 1) ? P.fb0 : P.fb1;
     R.fin_n = *(volatile uint32_t *)&P.ctl->cnt[r & 3][0];
     R.fout_cnt = &P.ctl->cnt[(r + 1) & 3][0];
     R.big_cnt = &P.ctl->cnt[r & 3][1];
     R.ch_cnt = &P.ctl->cnt[r & 3][2];
+    R.words_cnt = &P.ctl->cnt[r & 3][3];
     return R;
 }
 
@@ -107,9 +108,12 @@ __device__ __forceinline__ void round_advance(RoundCtl *ctl) {
     }
 }
 
+// Layouts interleave the S queries of a sub-batch (query index fastest):
+//   st / act [v * S + q], frontier words [(v >> 5) * S + q], claim words [(slot >> 5) * S + q],
+// so the queries of a sub-batch that touch the same vertex or slot touch adjacent words.
 __device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t v, uint32_t arr,
                                           uint32_t id) {
-    const size_t i = (size_t)q * P.n + v;
+    const size_t i = (size_t)v * P.S + q;
     const unsigned long long pk = ((unsigned long long)arr << 32) | id;
     if (P.stats) atomicAdd(P.relax_cnt + q, 1ull);
     // States only decrease: a stale cached read is an upper bound, so when it is
@@ -117,20 +121,27 @@ __device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32
     if (P.st[i] <= pk) return;
     const unsigned long long old = atomicMin(P.st + i, pk);
     if (arr < (uint32_t)(old >> 32)) {
-        if (atomicExch(P.mark + i, R.stamp) != R.stamp) {
-            cg::coalesced_group g = cg::coalesced_threads();
-            uint32_t base = 0;
-            if (g.thread_rank() == 0) base = atomicAdd(R.fout_cnt, g.size());
-            base = g.shfl(base, 0);
-            R.fout[base + g.thread_rank()] = ((unsigned long long)q << 32) | v;
-        }
+        // arrival improved: v joins the next round's frontier (bitmap: duplicates merge;
+        // no shared counter -- the next activation counts the non-empty words it finds)
+        atomicOr(R.fout + (size_t)(v >> 5) * P.S + q, 1u << (v & 31));
     }
+}
+
+// Same, with the filter value already loaded (batched loads, see eat_edges).
+__device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, uint32_t q, uint32_t v, uint32_t arr,
+                                              uint32_t id, unsigned long long cur) {
+    const unsigned long long pk = ((unsigned long long)arr << 32) | id;
+    if (P.stats) atomicAdd(P.relax_cnt + q, 1ull);
+    if (cur <= pk) return;
+    const size_t i = (size_t)v * P.S + q;
+    const unsigned long long old = atomicMin(P.st + i, pk);
+    if (arr < (uint32_t)(old >> 32)) atomicOr(R.fout + (size_t)(v >> 5) * P.S + q, 1u << (v & 31));
 }
 
 // test-and-set of slot s's claim bit for query q; true if this caller claimed it
 __device__ __forceinline__ bool claim(const EatP &P, uint32_t q, uint32_t s) {
     const uint32_t bit = 1u << (s & 31);
-    return (atomicOr(P.bits + (size_t)q * P.bit_words + (s >> 5), bit) & bit) == 0;
+    return (atomicOr(P.bits + (size_t)(s >> 5) * P.S + q, bit) & bit) == 0;
 }
 
 // sequential walk over slots [s, s_end): claim, relax, continue; stop at a slot
@@ -144,20 +155,12 @@ __device__ __forceinline__ void eat_walk(const EatP &P, const RoundV &R, uint32_
     }
 }
 
-// A newly usable occurrence p (sorted-edge position) for query q.
-__device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_t q, uint32_t p) {
-    const uint32_t s = __ldg(P.occ_slot + p);
-    const int4 sl = tg_ld_slot(P.slots + s);
-    const uint32_t arr = (uint32_t)sl.y;
-    if (arr > P.omega) return;
-    if ((uint32_t)sl.w == TG_SINGLE) {
-        eat_relax(P, R, q, (uint32_t)sl.x, arr, (uint32_t)sl.z);
-        return;
-    }
+// A newly usable occurrence at slot s (already loaded) of a long chain.
+__device__ __forceinline__ void eat_long(const EatP &P, const RoundV &R, uint32_t q, uint32_t s, int4 sl) {
     const uint32_t l = (uint32_t)sl.w;
     const uint2 info = __ldg(P.lc + l);  // {first slot, length}
     if (s != info.x && !claim(P, q, s)) return;  // a walker from an earlier entry got here first
-    eat_relax(P, R, q, (uint32_t)sl.x, arr, (uint32_t)sl.z);
+    eat_relax(P, R, q, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     uint32_t s_end = info.x + info.y;
     if (s + 1 >= s_end) return;
     if (P.use_sc) {
@@ -178,67 +181,108 @@ __device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_
     eat_walk(P, R, q, s + 1, s_end);
 }
 
+// A newly usable occurrence p (sorted-edge position) for query q.
+__device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_t q, uint32_t p) {
+    const uint32_t s = __ldg(P.occ_slot + p);
+    const int4 sl = tg_ld_slot(P.slots + s);
+    if ((uint32_t)sl.y > P.omega) return;
+    if ((uint32_t)sl.w == TG_SINGLE) eat_relax(P, R, q, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+    else eat_long(P, R, q, s, sl);
+}
+
+// Activation over the dense frontier bitmap: a warp loads 32 consecutive words
+// (one vertex word for up to 32 queries of the sub-batch), then for each non-empty
+// word handles its 32 consecutive vertices (lane = vertex).  Consecutive words
+// revisit the same vertices' node index and edge ranges for other queries, which
+// then hit in L1/L2.
 __global__ void __launch_bounds__(QT) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
-    const uint32_t F = R.fin_n;
+    __shared__ uint32_t s_words;
+    if (threadIdx.x == 0) s_words = 0;
+    __syncthreads();
+    uint32_t my_words = 0;
+    const uint32_t W = P.S * P.vwords;
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
-    for (uint32_t base = gw * 32; base < F; base += nw * 32) {
-        const uint32_t i = base + lane;
-        uint32_t q = 0, e0 = 0, cnt = 0;
-        if (i < F) {
-            const unsigned long long it = R.fin[i];
-            q = (uint32_t)(it >> 32);
-            const uint32_t u = (uint32_t)it;
-            const size_t si = (size_t)q * P.n + u;
-            const uint32_t now = (uint32_t)(__ldcg(P.st + si) >> 32);
-            const uint32_t a = __ldg(P.vnode_off + u), b = __ldg(P.vnode_off + u + 1);
-            const uint32_t lo_t = max(now, P.alpha);
-            const uint32_t j0 = tg_lower_bound(P.node_t, a, b, lo_t);
-            const uint32_t elo = __ldg(P.node_eoff + j0);
-            // previous boundary: edges at index >= act were activated before; the first
-            // activation starts from the window end (t + duration <= omega needs t < omega)
-            const uint32_t prev = atomicMin(P.act + si, elo);
-            if (elo < prev) {
-                uint32_t ehi = prev;
-                if (prev == TG_NONE) ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, j0, b, P.omega));
-                if (elo < ehi) { e0 = elo; cnt = ehi - elo; }
+    for (uint32_t wb = gw * 32; wb < W; wb += nw * 32) {
+        const uint32_t wi = wb + lane;
+        uint32_t word = (wi < W) ? R.fin[wi] : 0u;
+        if (word) R.fin[wi] = 0u;  // consume
+        uint32_t pending = __ballot_sync(0xffffffffu, word != 0);
+        my_words += (lane == 0) ? __popc(pending) : 0u;
+        while (pending) {
+            const int sl = __ffs(pending) - 1;
+            pending &= pending - 1;
+            const uint32_t bitsw = __shfl_sync(0xffffffffu, word, sl);
+            const uint32_t widx = wb + sl;
+            const uint32_t vw = widx / P.S;
+            const uint32_t q = widx - vw * P.S;
+            const uint32_t u = vw * 32 + lane;
+            uint32_t e0 = 0, cnt = 0;
+            if ((bitsw >> lane) & 1u) {
+                const size_t si = (size_t)u * P.S + q;
+                const uint32_t now = (uint32_t)(__ldcg(P.st + si) >> 32);
+                const uint32_t a = __ldg(P.vnode_off + u), b = __ldg(P.vnode_off + u + 1);
+                const uint32_t lo_t = max(now, P.alpha);
+                const uint32_t j0 = tg_lower_bound(P.node_t, a, b, lo_t);
+                const uint32_t elo = __ldg(P.node_eoff + j0);
+                // previous boundary: edges at index >= act were activated before; the first
+                // activation starts from the window end (t + duration <= omega needs t < omega)
+                const uint32_t prev = atomicMin(P.act + si, elo);
+                if (elo < prev) {
+                    uint32_t ehi = prev;
+                    if (prev == TG_NONE) ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, j0, b, P.omega));
+                    if (elo < ehi) { e0 = elo; cnt = ehi - elo; }
+                }
             }
-        }
-        if (cnt > BIG_T) {
-            const uint32_t nch = (cnt + CHUNK - 1) / CHUNK;
-            const uint32_t k = atomicAdd(R.big_cnt, nch);
-            for (uint32_t c = 0; c < nch; c++) {
-                const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
-                if (k + c < P.bigcap) P.bigq[k + c] = make_uint4(q, b0, b1, 0);
-                else for (uint32_t p = b0; p < b1; p++) eat_edge(P, R, q, p);  // bigcap is a bound
-            }
-            cnt = 0;
-        }
-        uint32_t incl = cnt;
+            {   // large ranges -> chunk queue, one reservation per warp
+                uint32_t nch = (cnt > BIG_T) ? (cnt + CHUNK - 1) / CHUNK : 0u;
+                uint32_t ci = nch;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += y;
-        }
-        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-        const uint32_t excl = incl - cnt;
-        for (uint32_t gb = 0; gb < total; gb += 32) {
-            const uint32_t g = gb + lane;
-            uint32_t own = 0;  // number of lanes whose inclusive prefix <= g == owner lane
-#pragma unroll
-            for (int bb = 16; bb; bb >>= 1) {
-                const uint32_t v = __shfl_sync(0xffffffffu, incl, own + bb - 1);
-                if (v <= g) own += bb;
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, ci, o);
+                    if (lane >= o) ci += y;
+                }
+                const uint32_t ctot = __shfl_sync(0xffffffffu, ci, 31);
+                if (ctot) {
+                    uint32_t kb = 0;
+                    if (lane == 0) kb = atomicAdd(R.big_cnt, ctot);
+                    kb = __shfl_sync(0xffffffffu, kb, 0) + ci - nch;
+                    for (uint32_t c = 0; c < nch; c++) {
+                        const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
+                        if (kb + c < P.bigcap) P.bigq[kb + c] = make_uint4(q, b0, b1, 0);
+                        else for (uint32_t p = b0; p < b1; p++) eat_edge(P, R, q, p);  // bigcap is a bound
+                    }
+                    if (nch) cnt = 0;
+                }
             }
-            own &= 31;
-            const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
-            const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
-            const uint32_t oq = __shfl_sync(0xffffffffu, q, own);
-            if (g < total) eat_edge(P, R, oq, oe0 + (g - oex));
+            uint32_t incl = cnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += y;
+            }
+            const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+            const uint32_t excl = incl - cnt;
+            for (uint32_t gb = 0; gb < total; gb += 32) {
+                const uint32_t g = gb + lane;
+                uint32_t own = 0;  // number of lanes whose inclusive prefix <= g == owner lane
+#pragma unroll
+                for (int bb = 16; bb; bb >>= 1) {
+                    const uint32_t v = __shfl_sync(0xffffffffu, incl, own + bb - 1);
+                    if (v <= g) own += bb;
+                }
+                own &= 31;
+                const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
+                const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
+                if (g < total) eat_edge(P, R, q, oe0 + (g - oex));
+            }
         }
     }
+    if (my_words) atomicAdd(&s_words, my_words);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_words) atomicAdd(R.words_cnt, s_words);
 }
 
 __global__ void __launch_bounds__(QT) k_eat_big(EatP P) {
@@ -286,11 +330,12 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
 
 // VInitial (Table 1): every state INF (memset), the source = (alpha, no pred),
 // frontier = the sources; round control reset for a new loop.
-__global__ void k_eat_init(unsigned long long *st, uint32_t n, const uint32_t *srcs, uint32_t S, uint32_t alpha,
-                           unsigned long long *fr1, RoundCtl *ctl, int push) {
+__global__ void k_eat_init(unsigned long long *st, uint32_t n, uint32_t vwords, const uint32_t *srcs, uint32_t S,
+                           uint32_t alpha, uint32_t *fb1, RoundCtl *ctl, int push) {
     for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < S; q += gridDim.x * blockDim.x) {
-        st[(size_t)q * n + srcs[q]] = ((unsigned long long)alpha << 32) | TG_NONE;
-        if (push) fr1[q] = ((unsigned long long)q << 32) | srcs[q];
+        const uint32_t x = srcs[q];
+        st[(size_t)x * S + q] = ((unsigned long long)alpha << 32) | TG_NONE;
+        if (push) fb1[(size_t)(x >> 5) * S + q] = 1u << (x & 31);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         for (int i = 0; i < 4; i++)
@@ -302,28 +347,47 @@ __global__ void k_eat_init(unsigned long long *st, uint32_t n, const uint32_t *s
     }
 }
 
-// mode 0 = EAT, 1 = LD (mirror: value = C - time; target = omega), 2 = REACH
-__global__ void k_eat_extract(const unsigned long long *__restrict__ st, uint32_t n, const uint32_t *__restrict__ srcs,
-                              int mode, uint32_t C, uint32_t omega, uint32_t *__restrict__ out,
-                              uint32_t *__restrict__ pred) {
-    const uint32_t q = blockIdx.y;
-    const uint32_t src = srcs[q];
-    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-        const size_t i = (size_t)q * n + v;
-        const unsigned long long pk = st[i];
-        const bool reached = pk != ~0ull;
-        const uint32_t t = (uint32_t)(pk >> 32), id = (uint32_t)pk;
-        uint32_t val, pr = reached ? id : TG_NONE;
-        if (mode == 0) {
-            val = reached ? t : TG_UNREACHED;
-        } else if (mode == 1) {
-            val = (v == src) ? omega : (reached ? C - t : TG_UNREACHED);
-            if (v == src) pr = TG_NONE;
-        } else {
-            val = reached ? 1u : 0u;
+// mode 0 = EAT, 1 = LD (mirror: value = C - time; target = omega), 2 = REACH.
+// st is [v][q]; out rows are [q][v]: a block transposes a tile of 32 vertices x S
+// queries through shared memory so both the read and the writes are coalesced.
+__global__ void __launch_bounds__(256) k_eat_extract(const unsigned long long *__restrict__ st, uint32_t n, uint32_t S,
+                                                     const uint32_t *__restrict__ srcs, int mode, uint32_t C,
+                                                     uint32_t omega, uint32_t *__restrict__ out,
+                                                     uint32_t *__restrict__ pred) {
+    __shared__ unsigned long long tile[32 * 65];
+    const uint32_t nt = (n + 31) / 32;
+    for (uint32_t tb = blockIdx.x; tb < nt; tb += gridDim.x) {
+        const uint32_t v0 = tb * 32;
+        for (uint32_t q0 = 0; q0 < S; q0 += 64) {
+            const uint32_t qs = min(64u, S - q0);
+            __syncthreads();
+            for (uint32_t i = threadIdx.x; i < 32 * qs; i += blockDim.x) {
+                const uint32_t dv = i / qs, dq = i - dv * qs;
+                const uint32_t v = v0 + dv;
+                tile[dv * 65 + dq] = (v < n) ? st[(size_t)v * S + q0 + dq] : ~0ull;
+            }
+            __syncthreads();
+            for (uint32_t i = threadIdx.x; i < 32 * qs; i += blockDim.x) {
+                const uint32_t dq = i / 32, dv = i - dq * 32;
+                const uint32_t v = v0 + dv, q = q0 + dq;
+                if (v >= n) continue;
+                const unsigned long long pk = tile[dv * 65 + dq];
+                const bool reached = pk != ~0ull;
+                const uint32_t t = (uint32_t)(pk >> 32), id = (uint32_t)pk;
+                uint32_t val, pr = reached ? id : TG_NONE;
+                const uint32_t src = srcs[q];
+                if (mode == 0) {
+                    val = reached ? t : TG_UNREACHED;
+                } else if (mode == 1) {
+                    val = (v == src) ? omega : (reached ? C - t : TG_UNREACHED);
+                    if (v == src) pr = TG_NONE;
+                } else {
+                    val = reached ? 1u : 0u;
+                }
+                out[(size_t)q * n + v] = val;
+                if (pred) pred[(size_t)q * n + v] = pr;
+            }
         }
-        out[i] = val;
-        if (pred) pred[i] = pr;
     }
 }
 
@@ -344,14 +408,21 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     DevArena &A = Q.arena;
     TG_TRY(A.alloc((void **)&Q.st, S * n * 8));
     TG_TRY(A.alloc((void **)&Q.act, S * n * 4));
-    const uint64_t mark_len = S * std::max<uint64_t>(n, nodes_state ? nnodes : 0);
-    TG_TRY(A.alloc((void **)&Q.mark, mark_len * 4));
-    TG_TRY_CUDA(cudaMemset(Q.mark, 0, mark_len * 4));
+    Q.vwords = (uint32_t)((n + 31) / 32);
+    TG_TRY(A.alloc((void **)&Q.fb[0], S * Q.vwords * 4));
+    TG_TRY(A.alloc((void **)&Q.fb[1], S * Q.vwords * 4));
+    if (nodes_state) {
+        const uint64_t mark_len = S * nnodes;
+        TG_TRY(A.alloc((void **)&Q.mark, std::max<uint64_t>(mark_len, 1) * 4));
+        TG_TRY_CUDA(cudaMemset(Q.mark, 0, std::max<uint64_t>(mark_len, 1) * 4));
+    }
     Q.bit_words = (m + 31) / 32 + 1;
     TG_TRY(A.alloc((void **)&Q.bits, S * Q.bit_words * 4));
-    Q.fcap = S * std::max<uint64_t>(n, nodes_state ? nnodes : 0) + 64;
-    TG_TRY(A.alloc((void **)&Q.fr[0], Q.fcap * 8));
-    TG_TRY(A.alloc((void **)&Q.fr[1], Q.fcap * 8));
+    if (nodes_state) {
+        Q.fcap = S * nnodes + 64;
+        TG_TRY(A.alloc((void **)&Q.fr[0], Q.fcap * 8));
+        TG_TRY(A.alloc((void **)&Q.fr[1], Q.fcap * 8));
+    }
     Q.bigcap = S * (m / CHUNK + std::max<uint64_t>(n, nnodes) / BIG_T + 2) + 1024;
     TG_TRY(A.alloc((void **)&Q.bigq, Q.bigcap * 16));
     Q.chcap = S * (m / (INLINE_WALK + 1)) + (1u << 16);
@@ -376,7 +447,7 @@ uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
     if (g->opt_sub_batch > 0) return (uint32_t)std::min<int64_t>(g->opt_sub_batch, k);
     const uint64_t n = g->n;
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
-    uint64_t hot = n * (8 + 4 + 4) + g->m / 8 + 64;
+    uint64_t hot = n * (8 + 4) + n / 4 + g->m / 8 + 64;
     if (nodes_state) hot = nnodes * (4 + 4) + n * 4 + 64;
     const uint64_t budget = 64ull << 20;
     uint64_t S = std::max<uint64_t>(1, budget / hot);
@@ -394,21 +465,25 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, S * n * 8, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, S * n * 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, S * Q.bit_words * 4, s));
+    TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, (uint64_t)S * Q.vwords * 4, s));
+    TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, (uint64_t)S * Q.vwords * 4, s));
     if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8, s));
     const bool work = any_work && g->m > 0 && alpha < omega;
-    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, Q.srcs, S, alpha, Q.fr[1], Q.ctl, work ? 1 : 0);
+    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, Q.vwords, Q.srcs, S, alpha, Q.fb[1], Q.ctl,
+              work ? 1 : 0);
     uint32_t rounds = 0;
     if (work) {
         EatP P{};
         P.vnode_off = cgr.vnode_off; P.node_t = cgr.node_t; P.node_eoff = cgr.node_eoff; P.occ_slot = cgr.occ_slot;
         P.slots = cgr.slots; P.lc = cgr.lc; P.sc = cgr.sc;
-        P.st = Q.st; P.act = Q.act; P.mark = Q.mark; P.bits = Q.bits; P.bit_words = Q.bit_words;
-        P.n = g->n; P.alpha = alpha; P.omega = omega;
+        P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
+        P.n = g->n; P.S = S; P.vwords = Q.vwords; P.alpha = alpha; P.omega = omega;
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
-        P.ctl = Q.ctl; P.fr0 = Q.fr[0]; P.fr1 = Q.fr[1];
+        P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1];
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         const uint32_t grid = tg_grid_persistent(8);
-        const int group = (int)std::max<int64_t>(1, g->opt_round_group);
+        static const bool trace = getenv("TG_TRACE") != nullptr;
+        const int group = trace ? 1 : (int)std::max<int64_t>(1, g->opt_round_group);
         for (;;) {
             for (int k = 0; k < group; k++) {
                 TG_LAUNCH(k_eat_activate, grid, QT, 0, s, P);
@@ -418,7 +493,12 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
             TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
             const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
-            if (h->cnt[h->round & 3][0] == 0) { rounds = h->round - 1; break; }
+            const uint32_t last = h->round - 1;  // the round just finished
+            if (trace)
+                fprintf(stderr, "[tg] S=%u round %u: frontier words %u big-chunks %u chain-walks %u\n", S, last,
+                        h->cnt[last & 3][3], h->cnt[last & 3][1], h->cnt[last & 3][2]);
+            // a round whose frontier bitmap was empty ends the loop (it did no work)
+            if (h->cnt[last & 3][3] == 0) { rounds = last - 1; break; }
             if (h->round > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
         }
     }
@@ -461,8 +541,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         g->last.sub_batches++;
         uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
         uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
-        dim3 grid((unsigned)std::min<uint64_t>((n + 255) / 256, 1024), Sb);
-        TG_LAUNCH(k_eat_extract, grid, 256, 0, s, Q.st, g->n, Q.srcs, mode, C, w.t_omega, o, pr);
+        const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
+        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr);
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (g->opt_stats) {

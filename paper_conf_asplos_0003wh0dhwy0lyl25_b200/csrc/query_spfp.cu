@@ -47,31 +47,66 @@ struct SpP {
     uint32_t *dnode, *vout, *mark;
     uint32_t n;
     uint64_t nnodes;
-    uint32_t alpha, omega, stamp;
+    uint32_t alpha, omega;
     int use_sc;
-    const unsigned long long *fin;
-    const uint32_t *fin_cnt;
-    unsigned long long *fout;
-    uint32_t *fout_cnt;
+    RoundCtl *ctl;
+    unsigned long long *fr0, *fr1;
     uint4 *bigq;
-    uint32_t *big_cnt;
     uint64_t bigcap;
 };
 
-__device__ __forceinline__ void push_node(const SpP &P, uint32_t q, uint32_t j) {
+struct RoundV {
+    uint32_t stamp;
+    const unsigned long long *fin;
+    uint32_t fin_n;
+    unsigned long long *fout;
+    uint32_t *fout_cnt, *big_cnt;
+};
+
+__device__ __forceinline__ RoundV round_view(const SpP &P) {
+    RoundV R;
+    const uint32_t r = *(volatile uint32_t *)&P.ctl->round;
+    R.stamp = *(volatile uint32_t *)&P.ctl->stamp;
+    R.fin = (r & 1) ? P.fr1 : P.fr0;
+    R.fout = (r & 1) ? P.fr0 : P.fr1;
+    R.fin_n = *(volatile uint32_t *)&P.ctl->cnt[r & 3][0];
+    R.fout_cnt = &P.ctl->cnt[(r + 1) & 3][0];
+    R.big_cnt = &P.ctl->cnt[r & 3][1];
+    return R;
+}
+
+__device__ __forceinline__ void round_advance(RoundCtl *ctl) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const uint32_t d = atomicAdd(&ctl->done_blocks, 1u);
+        if (d == gridDim.x - 1) {
+            const uint32_t r = ctl->round;
+            for (int i = 0; i < 4; i++) ctl->cnt[(r + 2) & 3][i] = 0;
+            ctl->cnt[(r + 1) & 3][1] = 0;
+            ctl->cnt[(r + 1) & 3][2] = 0;
+            ctl->done_blocks = 0;
+            ctl->stamp = ctl->stamp + 1;
+            ctl->round = r + 1;
+            __threadfence();
+        }
+    }
+}
+
+__device__ __forceinline__ void push_node(const SpP &P, const RoundV &R, uint32_t q, uint32_t j) {
     const size_t i = (size_t)q * P.nnodes + j;
-    if (atomicExch(P.mark + i, P.stamp) != P.stamp) {
+    if (atomicExch(P.mark + i, R.stamp) != R.stamp) {
         cg::coalesced_group g = cg::coalesced_threads();
         uint32_t base = 0;
-        if (g.thread_rank() == 0) base = atomicAdd(P.fout_cnt, g.size());
+        if (g.thread_rank() == 0) base = atomicAdd(R.fout_cnt, g.size());
         base = g.shfl(base, 0);
-        P.fout[base + g.thread_rank()] = ((unsigned long long)q << 32) | j;
+        R.fout[base + g.thread_rank()] = ((unsigned long long)q << 32) | j;
     }
 }
 
 // Walk the chain from slot s (entered with head-node value cur).
 template <bool FP>
-__device__ void spfp_walk(const SpP &P, uint32_t q, uint32_t s, uint32_t s_end, uint32_t cur) {
+__device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s, uint32_t s_end, uint32_t cur) {
     uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
     uint32_t *vo = P.vout + (size_t)q * P.n;
     for (; s < s_end; s++) {
@@ -93,13 +128,13 @@ __device__ void spfp_walk(const SpP &P, uint32_t q, uint32_t s, uint32_t s_end, 
         if (dn[tn] <= cand) return;  // not improved (stale read is an upper bound)
         const uint32_t old = atomicMin(dn + tn, cand);
         if (cand >= old) return;    // not improved: the improver pushed tn
-        push_node(P, q, tn);        // wait propagation + other out-edges next round
+        push_node(P, R, q, tn);     // wait propagation + other out-edges next round
         cur = cand;
     }
 }
 
 template <bool FP>
-__device__ __forceinline__ void spfp_edge(const SpP &P, uint32_t q, uint32_t p) {
+__device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_t q, uint32_t p) {
     const uint32_t s = __ldg(P.occ_slot + p);
     const uint32_t j = __ldg(P.occ_node + p);
     const uint32_t cur = __ldcg(P.dnode + (size_t)q * P.nnodes + j);
@@ -126,17 +161,18 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, uint32_t q, uint32_t p) 
                 }
                 if (tn != TG_NONE) {
                     const uint32_t old = atomicMin(P.dnode + (size_t)q * P.nnodes + tn, cand);
-                    if (cand < old) push_node(P, q, tn);
+                    if (cand < old) push_node(P, R, q, tn);
                 }
             }
         }
     }
-    spfp_walk<FP>(P, q, s, s_end, cur);
+    spfp_walk<FP>(P, R, q, s, s_end, cur);
 }
 
 template <bool FP>
 __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
-    const uint32_t F = *P.fin_cnt;
+    const RoundV R = round_view(P);
+    const uint32_t F = R.fin_n;
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
@@ -144,7 +180,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
         const uint32_t i = base + lane;
         uint32_t q = 0, e0 = 0, cnt = 0;
         if (i < F) {
-            const unsigned long long it = P.fin[i];
+            const unsigned long long it = R.fin[i];
             q = (uint32_t)(it >> 32);
             const uint32_t j = (uint32_t)it;
             uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
@@ -157,18 +193,18 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
                 if (__ldg(P.node_t + jend) >= P.omega) break;  // no valid out-edge departs at >= omega
                 const uint32_t old = atomicMin(dn + jend, d);
                 if (old <= d) break;
-                if (steps == WAIT_MAX) { push_node(P, q, jend); break; }  // continue next round
+                if (steps == WAIT_MAX) { push_node(P, R, q, jend); break; }  // continue next round
             }
             e0 = __ldg(P.node_eoff + j);
             cnt = __ldg(P.node_eoff + jend) - e0;
         }
         if (cnt > BIG_T) {
             const uint32_t nch = (cnt + CHUNK - 1) / CHUNK;
-            const uint32_t k = atomicAdd(P.big_cnt, nch);
+            const uint32_t k = atomicAdd(R.big_cnt, nch);
             for (uint32_t c = 0; c < nch; c++) {
                 const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
                 if (k + c < P.bigcap) P.bigq[k + c] = make_uint4(q, b0, b1, 0);
-                else for (uint32_t p = b0; p < b1; p++) spfp_edge<FP>(P, q, p);
+                else for (uint32_t p = b0; p < b1; p++) spfp_edge<FP>(P, R, q, p);
             }
             cnt = 0;
         }
@@ -192,26 +228,43 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
             const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
             const uint32_t oq = __shfl_sync(0xffffffffu, q, own);
-            if (g < total) spfp_edge<FP>(P, oq, oe0 + (g - oex));
+            if (g < total) spfp_edge<FP>(P, R, oq, oe0 + (g - oex));
         }
     }
 }
 
 template <bool FP>
 __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
-    const uint32_t B = (uint32_t)min((uint64_t)*P.big_cnt, P.bigcap);
+    const RoundV R = round_view(P);
+    const uint32_t B = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.big_cnt, P.bigcap);
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
-        for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<FP>(P, c.x, p);
+        for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<FP>(P, R, c.x, p);
     }
+    round_advance(P.ctl);
 }
 
 // VInitial: the source's departure nodes tau >= alpha get 0 (SP) / LS = tau (FP).
+// round control for a new loop (before k_spfp_init pushes into buffer 1)
+__global__ void k_spfp_ctl_init(RoundCtl *ctl) {
+    for (int i = 0; i < 4; i++)
+        for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
+    ctl->round = 0;  // k_spfp_init pushes with round 0's view: output buffer 1, count cnt[1][0]
+    ctl->done_blocks = 0;
+    ctl->stamp = ctl->stamp + 1;
+}
+
+__global__ void k_spfp_ctl_start(RoundCtl *ctl) {
+    ctl->round = 1;
+    ctl->stamp = ctl->stamp + 1;
+}
+
 template <bool FP>
 __global__ void k_spfp_init(SpP P, const uint32_t *srcs, uint32_t S) {
+    const RoundV R = round_view(P);
     const uint32_t q = blockIdx.y;
     if (q >= S) return;
     const uint32_t x = srcs[q];
@@ -221,7 +274,7 @@ __global__ void k_spfp_init(SpP P, const uint32_t *srcs, uint32_t S) {
         const uint32_t tau = P.node_t[j];
         if (tau >= P.omega) break;
         P.dnode[(size_t)q * P.nnodes + j] = FP ? (0xFFFFFFFEu - tau) : 0u;
-        push_node(P, q, j);
+        push_node(P, R, q, j);
     }
 }
 
@@ -245,7 +298,6 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     const uint64_t n = g->n, nn = c.nnodes;
     TG_TRY_CUDA(cudaMemsetAsync(Q.vout, 0xFF, Sb * n * 4, s));
     if (nn) TG_TRY_CUDA(cudaMemsetAsync(Q.dnode, 0xFF, Sb * nn * 4, s));
-    uint32_t rounds = 0;
     if (g->m == 0 || alpha >= omega) { *rounds_out = 0; return TG_OK; }
     SpP P{};
     P.vnode_off = c.vnode_off; P.node_t = c.node_t; P.node_u = c.node_u; P.node_eoff = c.node_eoff;
@@ -253,44 +305,28 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     P.lc = c.lc; P.sc = c.sc; P.sc_sumw = c.sc_sumw;
     P.dnode = Q.dnode; P.vout = Q.vout; P.mark = Q.mark; P.n = g->n; P.nnodes = nn;
     P.alpha = alpha; P.omega = omega; P.use_sc = (int)g->opt_shortcuts;
+    P.ctl = Q.ctl; P.fr0 = Q.fr[0]; P.fr1 = Q.fr[1];
     P.bigq = Q.bigq; P.bigcap = Q.bigcap;
-    // round 1 input = buffer 1
-    TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + 4, 0, 4, s));
-    if (++g->qs_epoch == 0) {
-        TG_TRY_CUDA(cudaMemsetAsync(Q.mark, 0, (uint64_t)Q.S * std::max<uint64_t>(n, nn) * 4, s));
-        g->qs_epoch = 1;
-    }
-    P.stamp = g->qs_epoch;
-    P.fout = Q.fr[1]; P.fout_cnt = Q.ctr + 4;
+    TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl);
     {
         dim3 grid(4, Sb);
         TG_LAUNCH(k_spfp_init<FP>, grid, 256, 0, s, P, Q.srcs, Sb);
     }
+    TG_LAUNCH(k_spfp_ctl_start, 1, 1, 0, s, Q.ctl);
     const uint32_t grid = tg_grid_persistent(8);
     const int group = (int)std::max<int64_t>(1, g->opt_round_group);
-    uint32_t r = 1;
+    uint32_t rounds = 0;
     for (;;) {
-        for (int k = 0; k < group; k++, r++) {
-            const int in = r & 1, outp = (r + 1) & 1;
-            TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + outp * 4, 0, 4, s));
-            TG_TRY_CUDA(cudaMemsetAsync(Q.ctr + in * 4 + 1, 0, 8, s));
-            if (++g->qs_epoch == 0) {
-                TG_TRY_CUDA(cudaMemsetAsync(Q.mark, 0, (uint64_t)Q.S * std::max<uint64_t>(n, nn) * 4, s));
-                g->qs_epoch = 1;
-            }
-            P.stamp = g->qs_epoch;
-            P.fin = Q.fr[in]; P.fin_cnt = Q.ctr + in * 4;
-            P.fout = Q.fr[outp]; P.fout_cnt = Q.ctr + outp * 4;
-            P.big_cnt = Q.ctr + in * 4 + 1;
+        for (int k = 0; k < group; k++) {
             TG_LAUNCH(k_spfp_activate<FP>, grid, QT, 0, s, P);
             TG_LAUNCH(k_spfp_big<FP>, grid, QT, 0, s, P);
         }
-        TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctr, 32, cudaMemcpyDeviceToHost, s));
+        TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
         TG_TRY_CUDA(cudaStreamSynchronize(s));
-        if (Q.h_ctr[(r & 1) * 4] == 0) break;
-        if (r > 10000000) { tg_set_error("SP/FP rounds did not converge"); return TG_ERR_CUDA; }
+        const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
+        if (h->cnt[h->round & 3][0] == 0) { rounds = h->round - 1; break; }
+        if (h->round > 10000000) { tg_set_error("SP/FP rounds did not converge"); return TG_ERR_CUDA; }
     }
-    rounds = r - 1;
     *rounds_out = rounds;
     return TG_OK;
 }

@@ -112,7 +112,9 @@ struct QueryScratch {
     uint64_t bit_words = 0;            // words per query
     uint32_t *dnode = nullptr;         // [S][nnodes] SP/FP node state
     uint32_t *vout = nullptr;          // [S][n] SP/FP per-vertex output
-    unsigned long long *fr[2] = {nullptr, nullptr};  // frontier items (q << 32 | vertex-or-node)
+    unsigned long long *fr[2] = {nullptr, nullptr};  // SP/FP frontier items (q << 32 | node)
+    uint32_t *fb[2] = {nullptr, nullptr};            // EAT-family dense frontier bitmaps [S][vwords]
+    uint32_t vwords = 0;
     uint64_t fcap = 0;
     uint4 *bigq = nullptr;   // big activation chunks {q, e_begin, e_end, -}
     uint64_t bigcap = 0;
