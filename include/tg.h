@@ -186,6 +186,11 @@ TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
 /* Total kernels this library has launched in this process (all handles). */
 TG_API uint64_t tg_kernel_launch_count(void);
 
+/* Device memory released by destroyed graphs is cached per device and reused by
+ * later graphs / queries (no cudaMalloc / cudaFree per create-build-query cycle).
+ * This returns every cached block to the CUDA driver. */
+TG_API void tg_release_cached_memory(void);
+
 /* Per-kernel timing for measurement: when enabled, every launch is bracketed by
  * a CUDA event pair recorded on the launching stream.  tg_profile_report
  * synchronises on the recorded events and folds them into a per-kernel table;

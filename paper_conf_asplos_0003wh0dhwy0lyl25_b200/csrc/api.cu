@@ -1,5 +1,6 @@
 // api.cu -- the C-ABI entry points of include/tg.h.
 #include <algorithm>
+#include <mutex>
 #include <chrono>
 #include <cstdio>
 #include <cstring>
@@ -39,26 +40,84 @@ void tg_prof_end(const char *name, cudaStream_t s, cudaEvent_t ev0) {
 
 void tg_set_error(const std::string &msg) { t_err = msg; }
 
+// ----------------------------------------------------------------------------- caching allocator
+// Device blocks released by a graph / query scratch are kept in a per-device free
+// list and handed out again for requests of a similar size (<= 2x), so repeated
+// create/build/query cycles do not pay cudaMalloc/cudaFree (which synchronises).
+namespace {
+struct CachedBlk { void *p; size_t bytes; int dev; };
+std::vector<CachedBlk> g_cache;
+std::mutex g_cache_mu;
+size_t round_bytes(size_t b) { return (b + 511) & ~size_t(511); }
+}  // namespace
+
+static void *cache_take(size_t bytes, int dev, size_t *got) {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    size_t best = (size_t)-1;
+    int bi = -1;
+    for (size_t i = 0; i < g_cache.size(); i++) {
+        const CachedBlk &c = g_cache[i];
+        if (c.dev == dev && c.bytes >= bytes && c.bytes <= 2 * bytes + (1u << 20) && c.bytes < best) {
+            best = c.bytes;
+            bi = (int)i;
+        }
+    }
+    if (bi < 0) return nullptr;
+    void *p = g_cache[bi].p;
+    *got = g_cache[bi].bytes;
+    g_cache.erase(g_cache.begin() + bi);
+    return p;
+}
+
+static void cache_release_all(int dev) {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    for (size_t i = 0; i < g_cache.size();) {
+        if (dev < 0 || g_cache[i].dev == dev) {
+            cudaFree(g_cache[i].p);
+            g_cache.erase(g_cache.begin() + i);
+        } else {
+            i++;
+        }
+    }
+}
+
 tg_status DevArena::alloc(void **p, size_t bytes) {
     *p = nullptr;
     if (nb >= (int)(sizeof(blks) / sizeof(blks[0]))) {
         tg_set_error("DevArena: too many blocks");
         return TG_ERR_NOMEM;
     }
-    if (bytes == 0) bytes = 16;
-    cudaError_t e = cudaMalloc(p, bytes);
-    if (e != cudaSuccess) {
-        cudaGetLastError();
-        tg_set_error(std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
-        return TG_ERR_NOMEM;
+    bytes = round_bytes(bytes ? bytes : 16);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    size_t got = bytes;
+    void *q = cache_take(bytes, dev, &got);
+    if (!q) {
+        got = bytes;
+        cudaError_t e = cudaMalloc(&q, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            cache_release_all(dev);  // return cached blocks to the driver and retry once
+            e = cudaMalloc(&q, bytes);
+        }
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            tg_set_error(std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+            return TG_ERR_NOMEM;
+        }
     }
-    blks[nb++] = {*p, bytes};
-    total += bytes;
+    *p = q;
+    blks[nb++] = {q, got};
+    total += got;
     return TG_OK;
 }
 
 void DevArena::free_all() {
-    for (int i = 0; i < nb; i++) cudaFree(blks[i].p);
+    // callers synchronise before releasing (blocks may be reused by the next owner at once)
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    for (int i = 0; i < nb; i++) g_cache.push_back({blks[i].p, blks[i].bytes, dev});
     nb = 0;
     total = 0;
 }
@@ -114,6 +173,11 @@ const char *tg_status_string(tg_status s) {
 const char *tg_last_error(void) { return t_err.c_str(); }
 
 uint64_t tg_kernel_launch_count(void) { return g_tg_launches; }
+
+void tg_release_cached_memory(void) {
+    cudaDeviceSynchronize();
+    cache_release_all(-1);
+}
 
 void tg_profile_enable(int on) { g_tg_profile = on ? 1 : 0; }
 

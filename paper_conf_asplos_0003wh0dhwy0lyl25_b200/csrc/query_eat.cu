@@ -397,6 +397,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     QueryScratch &Q = g->qs;
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
     if (Q.S >= S && Q.n == g->n && (!nodes_state || Q.nodes_state)) return TG_OK;
+    TG_TRY_CUDA(cudaDeviceSynchronize());  // blocks go back to the cache for immediate reuse
     Q.arena.free_all();
     if (Q.h_ctr) { cudaFreeHost(Q.h_ctr); Q.h_ctr = nullptr; }
     Q = QueryScratch{};
@@ -445,6 +446,10 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
 // frontier stamps, claim bits) of a sub-batch should stay resident in the 126 MB L2.
 uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
     if (g->opt_sub_batch > 0) return (uint32_t)std::min<int64_t>(g->opt_sub_batch, k);
+    // EAT family: the interleaved [v][q] layouts share vertex / slot lines across the
+    // queries of a sub-batch, so larger sub-batches are better (64: one frontier word
+    // group per vertex word); SP/FP: keep the per-query node state near L2 size.
+    if (!nodes_state) return std::min<uint32_t>(k, 64);
     const uint64_t n = g->n;
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
     uint64_t hot = n * (8 + 4) + n / 4 + g->m / 8 + 64;

@@ -26,7 +26,7 @@ TG_TMAX = 0x7FFFFFFE
 
 EXPORTED = ["tg_graph_create", "tg_build_chains", "tg_query", "tg_graph_destroy", "tg_status_string",
             "tg_last_error", "tg_graph_info", "tg_export_chains", "tg_last_query_stats", "tg_set_option",
-            "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report"]
+            "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report", "tg_release_cached_memory"]
 
 
 class TGError(RuntimeError):
@@ -87,6 +87,8 @@ def load_library(path: str = LIB_PATH):
     lib.tg_set_option.argtypes = [P, ctypes.c_char_p, i64]
     lib.tg_kernel_launch_count.restype = u64
     lib.tg_kernel_launch_count.argtypes = []
+    lib.tg_release_cached_memory.restype = None
+    lib.tg_release_cached_memory.argtypes = []
     lib.tg_profile_enable.restype = None
     lib.tg_profile_enable.argtypes = [ctypes.c_int]
     lib.tg_profile_report.restype = ctypes.c_int
@@ -184,6 +186,10 @@ def tg_set_option(g, key: str, value: int):
 
 def tg_kernel_launch_count() -> int:
     return int(load_library().tg_kernel_launch_count())
+
+
+def tg_release_cached_memory():
+    load_library().tg_release_cached_memory()
 
 
 def tg_profile_enable(on: bool = True):
