@@ -44,8 +44,8 @@ namespace cg = cooperative_groups;
 namespace {
 
 constexpr int QT = 256;                 // threads per block
-constexpr uint32_t BIG_T = 256;         // ranges above this are split into chunks
-constexpr uint32_t CHUNK = 1024;        // edges per chunk (one warp)
+constexpr uint32_t BIG_T = 128;         // unions longer than this are split into chunks
+constexpr uint32_t CHUNK = 128;         // edges per chunk (one warp)
 constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in the activating thread
 
 struct EatP {
@@ -56,11 +56,13 @@ struct EatP {
     unsigned long long *st;
     uint32_t *act, *bits;
     uint64_t bit_words;
-    uint32_t n, S, vwords;
+    uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
     uint32_t alpha, omega;
     int use_sc, stats;
     RoundCtl *ctl;
-    uint32_t *fb0, *fb1;  // dense frontier bitmaps [S][vwords], by round parity
+    uint32_t *fb0, *fb1;  // frontier masks [n][G] (bit = query within the group), by round parity
+    uint2 *recs;          // big-unit records: 32 per-query ranges each
+    uint64_t reccap;
     uint4 *bigq;
     uint64_t bigcap;
     uint4 *chq;
@@ -73,7 +75,7 @@ struct RoundV {
     uint32_t *fin;   // this round's frontier bitmap (consumed: words are cleared)
     uint32_t fin_n;
     uint32_t *fout;  // next round's frontier bitmap
-    uint32_t *fout_cnt, *big_cnt, *ch_cnt, *words_cnt;
+    uint32_t *rec_cnt, *big_cnt, *ch_cnt, *words_cnt;
 };
 
 __device__ __forceinline__ RoundV round_view(const EatP &P) {
@@ -81,8 +83,8 @@ __device__ __forceinline__ RoundV round_view(const EatP &P) {
     const uint32_t r = *(volatile uint32_t *)&P.ctl->round;
     R.fin = (r & 1) ? P.fb1 : P.fb0;
     R.fout = (r & 1) ? P.fb0 : P.fb1;
-    R.fin_n = *(volatile uint32_t *)&P.ctl->cnt[r & 3][0];
-    R.fout_cnt = &P.ctl->cnt[(r + 1) & 3][0];
+    R.fin_n = 0;
+    R.rec_cnt = &P.ctl->cnt[r & 3][0];
     R.big_cnt = &P.ctl->cnt[r & 3][1];
     R.ch_cnt = &P.ctl->cnt[r & 3][2];
     R.words_cnt = &P.ctl->cnt[r & 3][3];
@@ -109,7 +111,7 @@ __device__ __forceinline__ void round_advance(RoundCtl *ctl) {
 }
 
 // Layouts interleave the S queries of a sub-batch (query index fastest):
-//   st / act [v * S + q], frontier words [(v >> 5) * S + q], claim words [(slot >> 5) * S + q],
+//   st / act [v * S + q], frontier masks [v * G + q / 32] (bit q % 32), claim words [(slot >> 5) * S + q],
 // so the queries of a sub-batch that touch the same vertex or slot touch adjacent words.
 __device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t v, uint32_t arr,
                                           uint32_t id) {
@@ -123,7 +125,7 @@ __device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32
     if (arr < (uint32_t)(old >> 32)) {
         // arrival improved: v joins the next round's frontier (bitmap: duplicates merge;
         // no shared counter -- the next activation counts the non-empty words it finds)
-        atomicOr(R.fout + (size_t)(v >> 5) * P.S + q, 1u << (v & 31));
+        atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
     }
 }
 
@@ -135,7 +137,7 @@ __device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, ui
     if (cur <= pk) return;
     const size_t i = (size_t)v * P.S + q;
     const unsigned long long old = atomicMin(P.st + i, pk);
-    if (arr < (uint32_t)(old >> 32)) atomicOr(R.fout + (size_t)(v >> 5) * P.S + q, 1u << (v & 31));
+    if (arr < (uint32_t)(old >> 32)) atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
 }
 
 // test-and-set of slot s's claim bit for query q; true if this caller claimed it
@@ -190,102 +192,152 @@ __device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_
     else eat_long(P, R, q, s, sl);
 }
 
-// Activation over the dense frontier bitmap: a warp loads 32 consecutive words
-// (one vertex word for up to 32 queries of the sub-batch), then for each non-empty
-// word handles its 32 consecutive vertices (lane = vertex).  Consecutive words
-// revisit the same vertices' node index and edge ranges for other queries, which
-// then hit in L1/L2.
-__global__ void __launch_bounds__(QT) k_eat_activate(EatP P) {
+// Edge-major relaxation of one frontier unit (vertex v, query group g) over the
+// edge positions [pbeg, pend).  Lane k holds query g*32+k's newly usable range
+// [lo, hi) (empty: lo = hi).  Per block of 32 edges each lane loads one edge's
+// occurrence and slot once; a ballot per edge gives the queries for which that
+// edge is new; the (edge, query) pairs are compacted edge-major over the lanes,
+// so the queries of one edge read adjacent state words in one request.
+__device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint32_t g, uint32_t lo, uint32_t hi,
+                                           uint32_t pbeg, uint32_t pend) {
+    const int lane = threadIdx.x & 31;
+    for (uint32_t pb = pbeg; pb < pend; pb += 32) {
+        const uint32_t p = pb + lane;
+        uint32_t s = 0;
+        int4 sl = make_int4(0, -1, 0, 0);
+        if (p < pend) {
+            s = __ldg(P.occ_slot + p);
+            sl = tg_ld_slot(P.slots + s);
+        }
+        // mask of queries for which edge pb+k is newly usable (lane k keeps its own)
+        uint32_t mask = 0;
+#pragma unroll 8
+        for (int k = 0; k < 32; k++) {
+            const uint32_t pk = pb + k;
+            const uint32_t m = __ballot_sync(0xffffffffu, lo <= pk && pk < hi);
+            if (lane == k) mask = m;
+        }
+        if (p >= pend || (uint32_t)sl.y > P.omega) mask = 0;  // past the window end: never usable
+        const uint32_t cnt = __popc(mask);
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+        const uint32_t excl = incl - cnt;
+        for (uint32_t tb = 0; tb < total; tb += 32) {
+            const uint32_t t = tb + lane;
+            uint32_t own = 0;  // edge lane owning pair t
+#pragma unroll
+            for (int bb = 16; bb; bb >>= 1) {
+                const uint32_t v = __shfl_sync(0xffffffffu, incl, own + bb - 1);
+                if (v <= t) own += bb;
+            }
+            own &= 31;
+            const uint32_t om = __shfl_sync(0xffffffffu, mask, own);
+            const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
+            const uint32_t os = __shfl_sync(0xffffffffu, s, own);
+            int4 osl;
+            osl.x = __shfl_sync(0xffffffffu, sl.x, own);
+            osl.y = __shfl_sync(0xffffffffu, sl.y, own);
+            osl.z = __shfl_sync(0xffffffffu, sl.z, own);
+            osl.w = __shfl_sync(0xffffffffu, sl.w, own);
+            if (t < total) {
+                const uint32_t ql = __fns(om, 0, (int)(t - oex) + 1);  // (t-oex)-th set bit of the edge's mask
+                const uint32_t q = g * 32 + ql;
+                if ((uint32_t)osl.w == TG_SINGLE) eat_relax(P, R, q, (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
+                else eat_long(P, R, q, os, osl);
+            }
+        }
+    }
+}
+
+// Activation ("skeleton engine"): a warp loads the frontier masks of 32
+// consecutive units, then for each non-empty unit (vertex v, group g) lane k
+// computes query g*32+k's newly usable out-edge range of v: [first edge departing
+// at >= max(EAT(v), alpha), previous boundary), the boundary kept per (v, q) as
+// an edge index (atomicMin makes concurrent activations disjoint).  The union of
+// the lanes' ranges is relaxed edge-major (unit_range); long unions are split into
+// chunks for k_eat_big.
+__global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
-    __shared__ uint32_t s_words;
-    if (threadIdx.x == 0) s_words = 0;
+    __shared__ uint32_t s_units;
+    if (threadIdx.x == 0) s_units = 0;
     __syncthreads();
-    uint32_t my_words = 0;
-    const uint32_t W = P.S * P.vwords;
+    uint32_t my_units = 0;
+    const uint32_t NU = P.n * P.G;
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
-    for (uint32_t wb = gw * 32; wb < W; wb += nw * 32) {
-        const uint32_t wi = wb + lane;
-        uint32_t word = (wi < W) ? R.fin[wi] : 0u;
-        if (word) R.fin[wi] = 0u;  // consume
+    for (uint32_t ub = gw * 32; ub < NU; ub += nw * 32) {
+        const uint32_t ui = ub + lane;
+        uint32_t word = (ui < NU) ? R.fin[ui] : 0u;
+        if (word) R.fin[ui] = 0u;  // consume
         uint32_t pending = __ballot_sync(0xffffffffu, word != 0);
-        my_words += (lane == 0) ? __popc(pending) : 0u;
+        my_units += (lane == 0) ? __popc(pending) : 0u;
         while (pending) {
             const int sl = __ffs(pending) - 1;
             pending &= pending - 1;
-            const uint32_t bitsw = __shfl_sync(0xffffffffu, word, sl);
-            const uint32_t widx = wb + sl;
-            const uint32_t vw = widx / P.S;
-            const uint32_t q = widx - vw * P.S;
-            const uint32_t u = vw * 32 + lane;
-            uint32_t e0 = 0, cnt = 0;
-            if ((bitsw >> lane) & 1u) {
-                const size_t si = (size_t)u * P.S + q;
+            const uint32_t qm = __shfl_sync(0xffffffffu, word, sl);
+            const uint32_t unit = ub + sl;
+            const uint32_t v = unit / P.G;
+            const uint32_t g = unit - v * P.G;
+            const uint32_t q = g * 32 + lane;
+            uint32_t lo = 0, hi = 0;
+            if ((qm >> lane) & 1u) {
+                const size_t si = (size_t)v * P.S + q;
                 const uint32_t now = (uint32_t)(__ldcg(P.st + si) >> 32);
-                const uint32_t a = __ldg(P.vnode_off + u), b = __ldg(P.vnode_off + u + 1);
-                const uint32_t lo_t = max(now, P.alpha);
-                const uint32_t j0 = tg_lower_bound(P.node_t, a, b, lo_t);
+                const uint32_t a = __ldg(P.vnode_off + v), b = __ldg(P.vnode_off + v + 1);
+                const uint32_t j0 = tg_lower_bound(P.node_t, a, b, max(now, P.alpha));
                 const uint32_t elo = __ldg(P.node_eoff + j0);
-                // previous boundary: edges at index >= act were activated before; the first
+                // edges at index >= the boundary were activated before; the first
                 // activation starts from the window end (t + duration <= omega needs t < omega)
                 const uint32_t prev = atomicMin(P.act + si, elo);
                 if (elo < prev) {
                     uint32_t ehi = prev;
                     if (prev == TG_NONE) ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, j0, b, P.omega));
-                    if (elo < ehi) { e0 = elo; cnt = ehi - elo; }
+                    if (elo < ehi) { lo = elo; hi = ehi; }
                 }
             }
-            {   // large ranges -> chunk queue, one reservation per warp
-                uint32_t nch = (cnt > BIG_T) ? (cnt + CHUNK - 1) / CHUNK : 0u;
-                uint32_t ci = nch;
+            uint32_t ulo = (lo < hi) ? lo : 0xFFFFFFFFu, uhi = hi;
 #pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint32_t y = __shfl_up_sync(0xffffffffu, ci, o);
-                    if (lane >= o) ci += y;
+            for (int o = 16; o; o >>= 1) {
+                ulo = min(ulo, __shfl_xor_sync(0xffffffffu, ulo, o));
+                uhi = max(uhi, __shfl_xor_sync(0xffffffffu, uhi, o));
+            }
+            if (ulo >= uhi) continue;
+            if (uhi - ulo > BIG_T) {
+                // long union: record the 32 ranges once, queue chunks of CHUNK edges
+                uint32_t rec = 0, k0 = 0;
+                const uint32_t nch = (uhi - ulo + CHUNK - 1) / CHUNK;
+                if (lane == 0) {
+                    rec = atomicAdd(R.rec_cnt, 1u);
+                    k0 = atomicAdd(R.big_cnt, nch);
                 }
-                const uint32_t ctot = __shfl_sync(0xffffffffu, ci, 31);
-                if (ctot) {
-                    uint32_t kb = 0;
-                    if (lane == 0) kb = atomicAdd(R.big_cnt, ctot);
-                    kb = __shfl_sync(0xffffffffu, kb, 0) + ci - nch;
-                    for (uint32_t c = 0; c < nch; c++) {
-                        const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
-                        if (kb + c < P.bigcap) P.bigq[kb + c] = make_uint4(q, b0, b1, 0);
-                        else for (uint32_t p = b0; p < b1; p++) eat_edge(P, R, q, p);  // bigcap is a bound
+                rec = __shfl_sync(0xffffffffu, rec, 0);
+                k0 = __shfl_sync(0xffffffffu, k0, 0);
+                if (rec < P.reccap && k0 + nch <= P.bigcap) {
+                    P.recs[(size_t)rec * 32 + lane] = make_uint2(lo, hi);
+                    for (uint32_t c = lane; c < nch; c += 32) {
+                        const uint32_t b0 = ulo + c * CHUNK;
+                        P.bigq[k0 + c] = make_uint4(rec, b0, min(uhi, b0 + CHUNK), g);
                     }
-                    if (nch) cnt = 0;
+                    continue;
                 }
+                // capacity exceeded (not expected: both are bounds): relax in place
             }
-            uint32_t incl = cnt;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-                if (lane >= o) incl += y;
-            }
-            const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-            const uint32_t excl = incl - cnt;
-            for (uint32_t gb = 0; gb < total; gb += 32) {
-                const uint32_t g = gb + lane;
-                uint32_t own = 0;  // number of lanes whose inclusive prefix <= g == owner lane
-#pragma unroll
-                for (int bb = 16; bb; bb >>= 1) {
-                    const uint32_t v = __shfl_sync(0xffffffffu, incl, own + bb - 1);
-                    if (v <= g) own += bb;
-                }
-                own &= 31;
-                const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
-                const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
-                if (g < total) eat_edge(P, R, q, oe0 + (g - oex));
-            }
+            unit_range(P, R, g, lo, hi, ulo, uhi);
         }
     }
-    if (my_words) atomicAdd(&s_words, my_words);
+    if (lane == 0 && my_units) atomicAdd(&s_units, my_units);
     __syncthreads();
-    if (threadIdx.x == 0 && s_words) atomicAdd(R.words_cnt, s_words);
+    if (threadIdx.x == 0 && s_units) atomicAdd(R.words_cnt, s_units);
 }
 
-__global__ void __launch_bounds__(QT) k_eat_big(EatP P) {
+// Chunks of long unions: one warp per chunk, the unit's 32 query ranges from its record.
+__global__ void __launch_bounds__(QT, 8) k_eat_big(EatP P) {
     const RoundV R = round_view(P);
     const uint32_t B = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.big_cnt, P.bigcap);
     const int lane = threadIdx.x & 31;
@@ -293,7 +345,8 @@ __global__ void __launch_bounds__(QT) k_eat_big(EatP P) {
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
-        for (uint32_t p = c.y + lane; p < c.z; p += 32) eat_edge(P, R, c.x, p);
+        const uint2 r = P.recs[(size_t)c.x * 32 + lane];
+        unit_range(P, R, c.w, r.x, r.y, c.y, c.z);
     }
 }
 
@@ -330,17 +383,16 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
 
 // VInitial (Table 1): every state INF (memset), the source = (alpha, no pred),
 // frontier = the sources; round control reset for a new loop.
-__global__ void k_eat_init(unsigned long long *st, uint32_t n, uint32_t vwords, const uint32_t *srcs, uint32_t S,
+__global__ void k_eat_init(unsigned long long *st, uint32_t n, uint32_t G, const uint32_t *srcs, uint32_t S,
                            uint32_t alpha, uint32_t *fb1, RoundCtl *ctl, int push) {
     for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < S; q += gridDim.x * blockDim.x) {
         const uint32_t x = srcs[q];
         st[(size_t)x * S + q] = ((unsigned long long)alpha << 32) | TG_NONE;
-        if (push) fb1[(size_t)(x >> 5) * S + q] = 1u << (x & 31);
+        if (push) atomicOr(fb1 + (size_t)x * G + (q >> 5), 1u << (q & 31));
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         for (int i = 0; i < 4; i++)
             for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
-        ctl->cnt[1][0] = push ? S : 0;
         ctl->round = 1;
         ctl->done_blocks = 0;
         ctl->stamp = ctl->stamp + 1;  // stamps only grow: marks from earlier loops never match
@@ -409,9 +461,9 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     DevArena &A = Q.arena;
     TG_TRY(A.alloc((void **)&Q.st, S * n * 8));
     TG_TRY(A.alloc((void **)&Q.act, S * n * 4));
-    Q.vwords = (uint32_t)((n + 31) / 32);
-    TG_TRY(A.alloc((void **)&Q.fb[0], S * Q.vwords * 4));
-    TG_TRY(A.alloc((void **)&Q.fb[1], S * Q.vwords * 4));
+    Q.vwords = (uint32_t)((S + 31) / 32);  // query groups per vertex
+    TG_TRY(A.alloc((void **)&Q.fb[0], n * Q.vwords * 4));
+    TG_TRY(A.alloc((void **)&Q.fb[1], n * Q.vwords * 4));
     if (nodes_state) {
         const uint64_t mark_len = S * nnodes;
         TG_TRY(A.alloc((void **)&Q.mark, std::max<uint64_t>(mark_len, 1) * 4));
@@ -424,8 +476,12 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
         TG_TRY(A.alloc((void **)&Q.fr[0], Q.fcap * 8));
         TG_TRY(A.alloc((void **)&Q.fr[1], Q.fcap * 8));
     }
-    Q.bigcap = S * (m / CHUNK + std::max<uint64_t>(n, nnodes) / BIG_T + 2) + 1024;
+    // big-union chunks: per unit at most deg/CHUNK + 1; records: one per unit with a long union
+    Q.bigcap = std::max<uint64_t>(S * (m / CHUNK + std::max<uint64_t>(n, nnodes) / BIG_T + 2) + 1024,
+                                  (uint64_t)Q.vwords * (m / CHUNK + n / BIG_T + 2) + 1024);
     TG_TRY(A.alloc((void **)&Q.bigq, Q.bigcap * 16));
+    Q.reccap = (uint64_t)Q.vwords * (m / BIG_T + 2) + 1024;
+    TG_TRY(A.alloc((void **)&Q.recs, Q.reccap * 32 * 8));
     Q.chcap = S * (m / (INLINE_WALK + 1)) + (1u << 16);
     TG_TRY(A.alloc((void **)&Q.chq, Q.chcap * 16));
     TG_TRY(A.alloc((void **)&Q.ctr, 64));
@@ -470,11 +526,12 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, S * n * 8, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, S * n * 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, S * Q.bit_words * 4, s));
-    TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, (uint64_t)S * Q.vwords * 4, s));
-    TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, (uint64_t)S * Q.vwords * 4, s));
+    const uint32_t G = (S + 31) / 32;
+    TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
+    TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
     if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8, s));
     const bool work = any_work && g->m > 0 && alpha < omega;
-    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, Q.vwords, Q.srcs, S, alpha, Q.fb[1], Q.ctl,
+    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
     uint32_t rounds = 0;
     if (work) {
@@ -482,9 +539,9 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         P.vnode_off = cgr.vnode_off; P.node_t = cgr.node_t; P.node_eoff = cgr.node_eoff; P.occ_slot = cgr.occ_slot;
         P.slots = cgr.slots; P.lc = cgr.lc; P.sc = cgr.sc;
         P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
-        P.n = g->n; P.S = S; P.vwords = Q.vwords; P.alpha = alpha; P.omega = omega;
+        P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
-        P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1];
+        P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         const uint32_t grid = tg_grid_persistent(8);
         static const bool trace = getenv("TG_TRACE") != nullptr;

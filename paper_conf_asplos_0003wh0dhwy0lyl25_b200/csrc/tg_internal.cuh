@@ -113,8 +113,10 @@ struct QueryScratch {
     uint32_t *dnode = nullptr;         // [S][nnodes] SP/FP node state
     uint32_t *vout = nullptr;          // [S][n] SP/FP per-vertex output
     unsigned long long *fr[2] = {nullptr, nullptr};  // SP/FP frontier items (q << 32 | node)
-    uint32_t *fb[2] = {nullptr, nullptr};            // EAT-family dense frontier bitmaps [S][vwords]
-    uint32_t vwords = 0;
+    uint32_t *fb[2] = {nullptr, nullptr};            // EAT-family frontier masks [n][G]
+    uint32_t vwords = 0;                             // G = query groups of 32 (allocation)
+    uint2 *recs = nullptr;                           // big-unit records (32 ranges each)
+    uint64_t reccap = 0;
     uint64_t fcap = 0;
     uint4 *bigq = nullptr;   // big activation chunks {q, e_begin, e_end, -}
     uint64_t bigcap = 0;
