@@ -177,6 +177,11 @@ uint64_t tg_kernel_launch_count(void) { return g_tg_launches; }
 void tg_release_cached_memory(void) {
     cudaDeviceSynchronize();
     cache_release_all(-1);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
+    cudaGetLastError();
 }
 
 void tg_profile_enable(int on) { g_tg_profile = on ? 1 : 0; }
@@ -230,6 +235,21 @@ tg_status tg_graph_create(uint32_t n_vertices, uint64_t n_edges, const uint32_t 
     }
     if (device < 0 || device >= ndev) { tg_set_error("bad device ordinal"); return TG_ERR_INVALID; }
     DeviceGuard dg(device);
+    {
+        // keep the stream-ordered pool's memory between builds (the default release
+        // threshold of 0 returns it to the driver at every synchronisation, and the
+        // next cudaMallocAsync has to map it again)
+        static bool pool_set[64] = {false};
+        if (device < 64 && !pool_set[device]) {
+            cudaMemPool_t pool;
+            if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+                uint64_t thr = UINT64_MAX;
+                cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+            }
+            cudaGetLastError();
+            pool_set[device] = true;
+        }
+    }
     tg_graph *g = new tg_graph();
     g->device = device;
     g->n = n_vertices;
