@@ -45,6 +45,7 @@ extern "C" {
 #endif
 
 typedef struct tg_graph tg_graph; /* opaque; owned by the caller; free with tg_graph_destroy */
+typedef struct tg_comm tg_comm;   /* opaque NCCL communicator wrapper (multi-GPU only) */
 
 typedef enum {
     TG_OK = 0,
@@ -176,11 +177,33 @@ typedef struct {
  * relaxed exactly once, "first touch"). */
 TG_API tg_status tg_last_query_stats(const tg_graph *g, tg_query_stats *st, uint64_t *per_query_relax);
 
+/* ---------------------------------------------------------------- multi-GPU
+ * Two ways to use N GPUs; every rank calls the same functions with
+ * the same arguments (SPMD), one process per GPU.
+ *   mode 0 (replicate): each rank builds a full replica and answers its own block
+ *     of sources -- no communication on the data path; nothing to attach.
+ *   mode 1 (vertex range): ONE query batch is partitioned: rank r owns vertices
+ *     [n*r/N, n*(r+1)/N) and the chains of the edges leaving them (and, for LD,
+ *     of the mirror edges leaving them).  After every GAC round the packed
+ *     (arrival << 32 | pred) states are combined with ncclAllReduce(min) over
+ *     NVLink; `out`/`pred` are complete on every rank.  EAT / LD / REACH only.
+ * NCCL is loaded at run time (dlopen "libnccl.so.2"), sharing the process's copy. */
+
+/* 128-byte ncclUniqueId for tg_comm_create (rank 0 creates it, the caller broadcasts it). */
+TG_API tg_status tg_nccl_unique_id(void *out_id);
+/* Communicator for (rank, world) on `device`; world == 1 needs no NCCL. */
+TG_API tg_status tg_comm_create(const void *nccl_unique_id, int rank, int world, int device, tg_comm **out);
+TG_API void tg_comm_destroy(tg_comm *c); /* NULL-safe; destroy graphs that use it first */
+/* Attach before tg_build_chains; mode 0 = replicate, 1 = vertex range. */
+TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
+
 /* Tuning / debugging knobs (key, value):
  *   "sub_batch"  sources processed concurrently (0 = automatic)
  *   "stats"      1 = count relaxations per query (slower), 0 = off
  *   "shortcuts"  1 = relax chain tails through shortcuts on first entry (default), 0 = off
- *   "round_group" rounds launched between host convergence checks (default 4) */
+ *   "round_group" rounds launched between host convergence checks (default 4)
+ *   "partitions" logical vertex-range partitions on this GPU (1..16, before build):
+ *                runs the multi-GPU mode-1 algorithm inside one process (tests) */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
 
 /* Total kernels this library has launched in this process (all handles). */

@@ -83,10 +83,6 @@ static void cache_release_all(int dev) {
 
 tg_status DevArena::alloc(void **p, size_t bytes) {
     *p = nullptr;
-    if (nb >= (int)(sizeof(blks) / sizeof(blks[0]))) {
-        tg_set_error("DevArena: too many blocks");
-        return TG_ERR_NOMEM;
-    }
     bytes = round_bytes(bytes ? bytes : 16);
     int dev = 0;
     cudaGetDevice(&dev);
@@ -107,7 +103,7 @@ tg_status DevArena::alloc(void **p, size_t bytes) {
         }
     }
     *p = q;
-    blks[nb++] = {q, got};
+    blks.push_back({q, got});
     total += got;
     return TG_OK;
 }
@@ -117,8 +113,8 @@ void DevArena::free_all() {
     int dev = 0;
     cudaGetDevice(&dev);
     std::lock_guard<std::mutex> lk(g_cache_mu);
-    for (int i = 0; i < nb; i++) g_cache.push_back({blks[i].p, blks[i].bytes, dev});
-    nb = 0;
+    for (const Blk &b : blks) g_cache.push_back({b.p, b.bytes, dev});
+    blks.clear();
     total = 0;
 }
 
@@ -128,6 +124,10 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
                             uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
 tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                       bool out_dev, cudaStream_t s);
+tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
+                                 uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
+int tg_comm_rank(const tg_comm *c);
+int tg_comm_world(const tg_comm *c);
 
 static bool is_device_ptr(const void *p) {
     if (!p) return false;
@@ -278,8 +278,24 @@ tg_status tg_build_chains(tg_graph *g) {
     if (g->built) return TG_OK;
     DeviceGuard dg(g->device);
     auto t0 = std::chrono::steady_clock::now();
-    TG_TRY(tg_build_direction(g, &g->fwd, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, 0));
-    TG_TRY(tg_build_mirror(g, 0));
+    if (g->comm && g->comm_mode == 1) {
+        // this rank's vertex range of a single partitioned query batch
+        const int r = tg_comm_rank(g->comm), P = tg_comm_world(g->comm);
+        g->nparts = 1;
+        g->part_vb[0] = (uint32_t)((uint64_t)g->n * r / P);
+        g->part_vb[1] = (uint32_t)((uint64_t)g->n * (r + 1) / P);
+        TG_TRY(tg_build_partition(g, &g->pf[0], &g->pm[0], g->part_vb[0], g->part_vb[1], 0));
+    } else if (g->opt_partitions > 1) {
+        // logical vertex-range partitions on one GPU (same algorithm, shared state)
+        const int P = g->opt_partitions;
+        g->nparts = P;
+        for (int p = 0; p <= P; p++) g->part_vb[p] = (uint32_t)((uint64_t)g->n * p / P);
+        for (int p = 0; p < P; p++)
+            TG_TRY(tg_build_partition(g, &g->pf[p], &g->pm[p], g->part_vb[p], g->part_vb[p + 1], 0));
+    } else {
+        TG_TRY(tg_build_direction(g, &g->fwd, g->m, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, nullptr, 0));
+        TG_TRY(tg_build_mirror(g, 0));
+    }
     TG_TRY_CUDA(cudaDeviceSynchronize());
     g->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     g->built = true;
@@ -309,6 +325,13 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
     cudaStream_t s = (cudaStream_t)cuda_stream;
     const bool out_dev = is_device_ptr(out);
     const bool pred_dev = is_device_ptr(pred);
+    if (g->nparts > 0) {
+        if (!(p == TG_EAT || p == TG_LD || p == TG_REACH)) {
+            tg_set_error("vertex-range partitioned graphs answer TG_EAT / TG_LD / TG_REACH only");
+            return TG_ERR_STATE;
+        }
+        return tg_run_eat_partitioned(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
+    }
     if (p == TG_EAT || p == TG_LD || p == TG_REACH)
         return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     return tg_run_spfp(g, p, sources, n_sources, w, out, out_dev, s);
@@ -334,6 +357,12 @@ tg_status tg_graph_info(const tg_graph *g, tg_info *info) {
     info->n_chains = g->fwd.nchains;
     info->n_long_chains = g->fwd.nlong;
     info->max_chain_len = g->fwd.maxlen;
+    for (int p = 0; p < g->nparts; p++) {  // partitioned: totals over this process's partitions
+        info->n_nodes += g->pf[p].nnodes;
+        info->n_chains += g->pf[p].nchains;
+        info->n_long_chains += g->pf[p].nlong;
+        info->max_chain_len = std::max(info->max_chain_len, g->pf[p].maxlen);
+    }
     info->c_mirror = g->max_arr;
     info->device_bytes = g->arena.total + g->qs.arena.total;
     info->build_ms = g->build_ms;
@@ -346,6 +375,7 @@ tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off,
                            uint32_t *sc_tail_v, uint32_t *sc_arr, uint64_t *sc_sum_w, uint32_t *sc_elapsed) {
     if (!g || !chain_off || !chain_edges) { tg_set_error("NULL argument"); return TG_ERR_INVALID; }
     if (!g->built) { tg_set_error("graph not built"); return TG_ERR_STATE; }
+    if (g->nparts > 0) { tg_set_error("chain export is for unpartitioned graphs"); return TG_ERR_STATE; }
     DeviceGuard dg(g->device);
     const ChainGraph &c = mirrored ? g->mir : g->fwd;
     const uint64_t m = g->m, nc = c.nchains;
@@ -406,6 +436,11 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     else if (k == "stats") g->opt_stats = value;
     else if (k == "shortcuts") g->opt_shortcuts = value;
     else if (k == "round_group") g->opt_round_group = value;
+    else if (k == "partitions") {
+        if (g->built) { tg_set_error("set partitions before tg_build_chains"); return TG_ERR_STATE; }
+        if (value < 1 || value > TG_MAXP) { tg_set_error("partitions must be in [1, 16]"); return TG_ERR_RANGE; }
+        g->opt_partitions = (int)value;
+    }
     else { tg_set_error("unknown option " + k); return TG_ERR_INVALID; }
     return TG_OK;
 }

@@ -143,7 +143,8 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
                                 int4 *__restrict__ slots, uint32_t *__restrict__ slot_w,
                                 uint32_t *__restrict__ slot_tn, uint32_t *__restrict__ occ_slot,
                                 uint2 *__restrict__ lc, int4 *__restrict__ sc,
-                                unsigned long long *__restrict__ sc_sumw, uint32_t *__restrict__ sc_elapsed) {
+                                unsigned long long *__restrict__ sc_sumw, uint32_t *__restrict__ sc_elapsed,
+                                const uint32_t *__restrict__ id_map) {
     GRID_STRIDE(p, m) {
         if (!head[p]) continue;
         uint32_t c = cidx[p];
@@ -156,7 +157,7 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
         while (q != TG_NONE) {
             uint32_t e = sid[q];
             uint32_t w = Wt[e];
-            slots[s] = make_int4((int)s_v[q], (int)s_arr[q], (int)e, (int)l);
+            slots[s] = make_int4((int)s_v[q], (int)s_arr[q], (int)(id_map ? id_map[e] : e), (int)l);
             slot_w[s] = w;
             slot_tn[s] = tn[q];
             occ_slot[q] = s;
@@ -167,7 +168,8 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
         }
         if (len >= 2) {
             lc[l] = make_uint2(first, len);
-            sc[l] = make_int4((int)s_v[last], (int)s_arr[last], (int)sid[last], (int)node_of[p]);
+            const uint32_t lid = id_map ? id_map[sid[last]] : sid[last];
+            sc[l] = make_int4((int)s_v[last], (int)s_arr[last], (int)lid, (int)node_of[p]);
             sc_sumw[l] = sumw;
             sc_elapsed[l] = s_arr[last] - T[sid[p]];
         }
@@ -203,6 +205,25 @@ __global__ void k_validate(const uint32_t *__restrict__ u, const uint32_t *__res
         atomicMax(&res[2], ma);
         atomicMax(&res[3], mw);
         atomicMin(&res[4], mn);
+    }
+}
+
+// vertex-range partitions: keep edges whose key vertex (u forward, v mirror) is in [vb, ve)
+__global__ void k_range_flags(const uint32_t *__restrict__ key, uint64_t m, uint32_t vb, uint32_t ve,
+                              uint32_t *__restrict__ flag) {
+    GRID_STRIDE(i, m) flag[i] = (key[i] >= vb && key[i] < ve) ? 1u : 0u;
+}
+
+__global__ void k_range_compact(const uint32_t *__restrict__ key, uint64_t m, uint32_t vb, uint32_t ve,
+                                const uint32_t *__restrict__ pos, const uint32_t *__restrict__ u,
+                                const uint32_t *__restrict__ v, const uint32_t *__restrict__ t,
+                                const uint32_t *__restrict__ dur, const uint32_t *__restrict__ w,
+                                uint32_t *__restrict__ ou, uint32_t *__restrict__ ov, uint32_t *__restrict__ ot,
+                                uint32_t *__restrict__ odur, uint32_t *__restrict__ ow, uint32_t *__restrict__ oid) {
+    GRID_STRIDE(i, m) {
+        if (key[i] < vb || key[i] >= ve) continue;
+        const uint32_t j = pos[i];
+        ou[j] = u[i]; ov[j] = v[i]; ot[j] = t[i]; odur[j] = dur[i]; ow[j] = w[i]; oid[j] = (uint32_t)i;
     }
 }
 
@@ -245,9 +266,9 @@ static int bits_for(uint64_t x) {  // bits to represent values in [0, x]
     return std::max(b, 1);
 }
 
-tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, const uint32_t *u, const uint32_t *v, const uint32_t *t,
-                             const uint32_t *dur, const uint32_t *w, cudaStream_t s) {
-    const uint64_t m = g->m;
+tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
+                             const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
+                             cudaStream_t s) {
     const uint32_t n = g->n;
     cg->n = n;
     cg->m = m;
@@ -373,7 +394,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, const uint32_t *u, con
     TG_TRY(A.alloc((void **)&cg->sc_elapsed, std::max<uint64_t>(L, 1) * 4));
     TG_LAUNCH(k_chain_scatter, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, cg->chain_first, chain_len, lidx, sid,
               s_v, s_arr, tn, node_of, t, w, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
-              cg->sc_sumw, cg->sc_elapsed);
+              cg->sc_sumw, cg->sc_elapsed, id_map);
 
     for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)s_v, (void *)s_arr, (void *)hub,
                     (void *)head, (void *)succ, (void *)cidx, (void *)chain_len, (void *)lidx})
@@ -384,12 +405,54 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, const uint32_t *u, con
 
 tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {
     // reading A5: G^R maps (u, v, t, lam) to (v, u, C - (t + lam), lam), C = max(t + lam)
-    if (g->m == 0) return tg_build_direction(g, &g->mir, g->d_v, g->d_u, g->d_t, g->d_dur, g->d_w, s);
+    if (g->m == 0) return tg_build_direction(g, &g->mir, 0, g->d_v, g->d_u, g->d_t, g->d_dur, g->d_w, nullptr, s);
     uint32_t *mt = nullptr;
     TG_TRY_CUDA(cudaMallocAsync((void **)&mt, g->m * 4, s));
     TG_LAUNCH(k_mirror, blocks_for(g->m, 4), BT, 0, s, g->d_t, g->d_dur, g->m, g->max_arr, mt);
-    tg_status st = tg_build_direction(g, &g->mir, g->d_v, g->d_u, mt, g->d_dur, g->d_w, s);
+    tg_status st = tg_build_direction(g, &g->mir, g->m, g->d_v, g->d_u, mt, g->d_dur, g->d_w, nullptr, s);
     cudaFreeAsync(mt, s);
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     return st;
+}
+
+// One vertex-range partition [vb, ve): forward chains over the edges leaving the
+// range, mirror chains over the edges entering it (the mirror's sources).
+// Slots keep the original edge ids (id map).
+tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s) {
+    const uint64_t m = g->m;
+    uint32_t *mt = nullptr, *flag = nullptr, *cnt = nullptr;
+    TG_TRY_CUDA(cudaMallocAsync((void **)&mt, std::max<uint64_t>(m, 1) * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&flag, std::max<uint64_t>(m, 1) * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&cnt, 4, s));
+    if (m) TG_LAUNCH(k_mirror, blocks_for(m, 4), BT, 0, s, g->d_t, g->d_dur, m, g->max_arr, mt);
+    for (int dir = 0; dir < 2; dir++) {
+        // forward: (u, v, t); mirror: (v, u, C - t - dur)
+        const uint32_t *key = dir == 0 ? g->d_u : g->d_v;
+        const uint32_t *uu = dir == 0 ? g->d_u : g->d_v;
+        const uint32_t *vv = dir == 0 ? g->d_v : g->d_u;
+        const uint32_t *tt = dir == 0 ? g->d_t : mt;
+        uint32_t ms = 0;
+        if (m) {
+            TG_LAUNCH(k_range_flags, blocks_for(m, 4), BT, 0, s, key, m, vb, ve, flag);
+            TG_TRY(tg_exclusive_scan_u32(flag, flag, m, cnt, s, nullptr));
+            TG_TRY_CUDA(cudaMemcpyAsync(&ms, cnt, 4, cudaMemcpyDeviceToHost, s));
+            TG_TRY_CUDA(cudaStreamSynchronize(s));
+        }
+        uint32_t *sub = nullptr;  // 6 arrays of ms
+        TG_TRY_CUDA(cudaMallocAsync((void **)&sub, std::max<uint64_t>(ms, 1) * 4 * 6, s));
+        uint32_t *su = sub, *sv = sub + ms, *st = sub + 2 * (uint64_t)ms, *sd = sub + 3 * (uint64_t)ms,
+                 *sw = sub + 4 * (uint64_t)ms, *sid = sub + 5 * (uint64_t)ms;
+        if (ms)
+            TG_LAUNCH(k_range_compact, blocks_for(m, 4), BT, 0, s, key, m, vb, ve, flag, uu, vv, tt, g->d_dur, g->d_w,
+                      su, sv, st, sd, sw, sid);
+        tg_status r = tg_build_direction(g, dir == 0 ? fwd : mir, ms, su, sv, st, sd, sw, sid, s);
+        TG_TRY_CUDA(cudaStreamSynchronize(s));
+        cudaFreeAsync(sub, s);
+        if (r != TG_OK) return r;
+    }
+    cudaFreeAsync(mt, s);
+    cudaFreeAsync(flag, s);
+    cudaFreeAsync(cnt, s);
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    return TG_OK;
 }

@@ -57,6 +57,7 @@ struct EatP {
     uint32_t *act, *bits;
     uint64_t bit_words;
     uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
+    uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
     uint32_t alpha, omega;
     int use_sc, stats;
     RoundCtl *ctl;
@@ -267,11 +268,11 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
     if (threadIdx.x == 0) s_units = 0;
     __syncthreads();
     uint32_t my_units = 0;
-    const uint32_t NU = P.n * P.G;
+    const uint32_t NU = P.ub1;
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
-    for (uint32_t ub = gw * 32; ub < NU; ub += nw * 32) {
+    for (uint32_t ub = P.ub0 + gw * 32; ub < NU; ub += nw * 32) {
         const uint32_t ui = ub + lane;
         uint32_t word = (ui < NU) ? R.fin[ui] : 0u;
         if (word) R.fin[ui] = 0u;  // consume
@@ -443,12 +444,47 @@ __global__ void __launch_bounds__(256) k_eat_extract(const unsigned long long *_
     }
 }
 
+// Vertex-range partitions: after the state exchange, each partition derives the
+// next frontier of ITS vertices from the state itself (bits set by relaxations are
+// discarded): (v, q) is active iff its arrival dropped below the last activated one.
+// One thread per unit bit, so a warp assembles one frontier word with a ballot.
+__global__ void k_part_frontier(const unsigned long long *__restrict__ st, uint32_t *__restrict__ lat,
+                                uint32_t *__restrict__ fnext, uint32_t S, uint32_t G, uint32_t vb, uint32_t ve,
+                                uint32_t *__restrict__ count) {
+    uint32_t mine = 0;
+    const uint64_t u0 = (uint64_t)vb * G, u1 = (uint64_t)ve * G;  // frontier units of the range
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t unit = u0 + gw; unit < u1; unit += nw) {  // warp per unit: lane = query bit
+        const uint32_t v = (uint32_t)(unit / G), g = (uint32_t)(unit - (uint64_t)v * G);
+        const uint32_t q = g * 32 + lane;
+        bool on = false;
+        if (q < S) {
+            const size_t si = (size_t)v * S + q;
+            const uint32_t now = (uint32_t)(st[si] >> 32);
+            if (now < lat[si]) { lat[si] = now; on = true; }
+        }
+        const uint32_t w = __ballot_sync(0xffffffffu, on);
+        if (lane == 0) { fnext[unit] = w; mine += __popc(w); }
+    }
+    if (lane == 0 && mine) atomicAdd(count, mine);
+}
+
+__global__ void k_ctl_reset(RoundCtl *ctl) {
+    for (int i = 0; i < 4; i++)
+        for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
+    ctl->round = 1;
+    ctl->done_blocks = 0;
+    ctl->stamp = ctl->stamp + 1;
+}
+
 }  // namespace
 
 static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     QueryScratch &Q = g->qs;
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
-    if (Q.S >= S && Q.n == g->n && (!nodes_state || Q.nodes_state)) return TG_OK;
+    if (Q.S >= S && Q.n == g->n && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat)) return TG_OK;
     TG_TRY_CUDA(cudaDeviceSynchronize());  // blocks go back to the cache for immediate reuse
     Q.arena.free_all();
     if (Q.h_ctr) { cudaFreeHost(Q.h_ctr); Q.h_ctr = nullptr; }
@@ -469,7 +505,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
         TG_TRY(A.alloc((void **)&Q.mark, std::max<uint64_t>(mark_len, 1) * 4));
         TG_TRY_CUDA(cudaMemset(Q.mark, 0, std::max<uint64_t>(mark_len, 1) * 4));
     }
-    Q.bit_words = (m + 31) / 32 + 1;
+    Q.bit_words = (m + 31) / 32 + TG_MAXP + 1;  // partitions get word-aligned regions
     TG_TRY(A.alloc((void **)&Q.bits, S * Q.bit_words * 4));
     if (nodes_state) {
         Q.fcap = S * nnodes + 64;
@@ -486,8 +522,12 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     TG_TRY(A.alloc((void **)&Q.chq, Q.chcap * 16));
     TG_TRY(A.alloc((void **)&Q.ctr, 64));
     TG_TRY_CUDA(cudaMemset(Q.ctr, 0, 64));
-    TG_TRY(A.alloc((void **)&Q.ctl, sizeof(RoundCtl)));
-    TG_TRY_CUDA(cudaMemset(Q.ctl, 0, sizeof(RoundCtl)));
+    TG_TRY(A.alloc((void **)&Q.ctl, sizeof(RoundCtl) * TG_MAXP));
+    TG_TRY_CUDA(cudaMemset(Q.ctl, 0, sizeof(RoundCtl) * TG_MAXP));
+    if (g->nparts > 0) {
+        TG_TRY(A.alloc((void **)&Q.lat, S * n * 4));
+        TG_TRY(A.alloc((void **)&Q.pcount, 64));
+    }
     TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
     TG_TRY(A.alloc((void **)&Q.srcs, S * 4));
     TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8));
@@ -540,6 +580,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         P.slots = cgr.slots; P.lc = cgr.lc; P.sc = cgr.sc;
         P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
         P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
+        P.ub0 = 0; P.ub1 = g->n * G;
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
@@ -599,6 +640,131 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources + b0, Sb * 4, cudaMemcpyHostToDevice, s));
         uint32_t rounds = 0;
         TG_TRY(eat_rounds(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
+        g->last.rounds = std::max(g->last.rounds, rounds);
+        g->last.sub_batches++;
+        uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
+        uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
+        const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
+        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr);
+        if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
+        if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
+        if (g->opt_stats) {
+            std::vector<unsigned long long> h(Sb);
+            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, Sb * 8, cudaMemcpyDeviceToHost, s));
+            TG_TRY_CUDA(cudaStreamSynchronize(s));
+            for (uint32_t q = 0; q < Sb; q++) { g->last_relax[b0 + q] = h[q]; g->last.slots_relaxed += h[q]; }
+        }
+    }
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    g->last.kernel_launches = g_tg_launches - launches0;
+    return TG_OK;
+}
+
+// ============================================================================ vertex-range partitions
+tg_status tg_comm_allreduce_min_u64(tg_comm *c, unsigned long long *buf, uint64_t count, cudaStream_t s);
+tg_status tg_comm_allreduce_sum_u32(tg_comm *c, uint32_t *buf, uint64_t count, cudaStream_t s);
+
+// Single query batch partitioned by vertex range (SURVEY §8(e) mode 2).  Every
+// partition p (one per rank with NCCL, or g->nparts logical partitions on one GPU)
+// activates only its own vertices and relaxes its own chains; after the round the
+// packed states are combined with a min-allreduce (NCCL) -- on one GPU the logical
+// partitions share one state array -- and each partition derives its next
+// frontier from the combined state (k_part_frontier).
+tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
+                                 uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s) {
+    const bool ld = (p == TG_LD);
+    uint32_t alpha = w.t_alpha, omega = w.t_omega;
+    bool any_work = true;
+    const uint32_t C = g->max_arr;
+    if (ld) {
+        if (alpha > C) { any_work = false; alpha = 0; omega = 0; }
+        else { uint32_t a2 = (omega >= C) ? 0u : C - omega; omega = C - alpha; alpha = a2; }
+    }
+    const uint32_t S = tg_pick_sub_batch(g, k, false);
+    TG_TRY(ensure_scratch(g, S, false));
+    QueryScratch &Q = g->qs;
+    const uint64_t n = g->n;
+    if (!out_dev && !Q.out_stage) TG_TRY(Q.arena.alloc((void **)&Q.out_stage, (uint64_t)Q.S * n * 4));
+    if (pred && !pred_dev && !Q.pred_stage) TG_TRY(Q.arena.alloc((void **)&Q.pred_stage, (uint64_t)Q.S * n * 4));
+    g->last = tg_query_stats{};
+    if (g->opt_stats) {
+        delete[] g->last_relax;
+        g->last_relax = new uint64_t[k];
+        g->last_relax_len = k;
+    }
+    const uint64_t launches0 = g_tg_launches;
+    const int mode = ld ? 1 : (p == TG_REACH ? 2 : 0);
+    const uint32_t grid = tg_grid_persistent(8);
+    for (uint32_t b0 = 0; b0 < k; b0 += S) {
+        const uint32_t Sb = std::min(S, k - b0);
+        const uint32_t G = (Sb + 31) / 32;
+        TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources + b0, Sb * 4, cudaMemcpyHostToDevice, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, Sb * n * 8, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, Sb * n * 4, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.lat, 0xFF, Sb * n * 4, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, Sb * Q.bit_words * 4, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
+        if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8, s));
+        TG_LAUNCH(k_eat_init, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs, Sb, alpha, Q.fb[1], Q.ctl, 0);
+        const bool work = any_work && g->m > 0 && alpha < omega;
+        uint32_t rounds = 0;
+        if (work) {
+            EatP base{};
+            base.st = Q.st; base.act = Q.act; base.bits = Q.bits; base.bit_words = Q.bit_words;
+            base.n = g->n; base.S = Sb; base.G = G; base.alpha = alpha; base.omega = omega;
+            base.use_sc = (int)g->opt_shortcuts; base.stats = (int)g->opt_stats;
+            base.fb0 = Q.fb[0]; base.fb1 = Q.fb[1]; base.recs = Q.recs; base.reccap = Q.reccap;
+            base.bigq = Q.bigq; base.bigcap = Q.bigcap; base.chq = Q.chq; base.chcap = Q.chcap;
+            base.relax_cnt = Q.relax_cnt;
+            EatP parts[TG_MAXP];
+            uint64_t bit_off = 0;  // claim bits: each partition numbers its own slots from 0
+            for (int pi = 0; pi < g->nparts; pi++) {
+                const ChainGraph &cg = ld ? g->pm[pi] : g->pf[pi];
+                EatP P = base;
+                P.bits = Q.bits + bit_off * Sb;
+                bit_off += (cg.m + 31) / 32;
+                P.vnode_off = cg.vnode_off; P.node_t = cg.node_t; P.node_eoff = cg.node_eoff; P.occ_slot = cg.occ_slot;
+                P.slots = cg.slots; P.lc = cg.lc; P.sc = cg.sc;
+                P.ctl = Q.ctl + pi;
+                P.ub0 = g->part_vb[pi] * G;
+                P.ub1 = g->part_vb[pi + 1] * G;
+                parts[pi] = P;
+                TG_LAUNCH(k_ctl_reset, 1, 1, 0, s, Q.ctl + pi);
+                // round 1's frontier: the sources, derived from the state like every later one
+                TG_LAUNCH(k_part_frontier, grid, 256, 0, s, Q.st, Q.lat, Q.fb[1], Sb, G, g->part_vb[pi],
+                          g->part_vb[pi + 1], Q.pcount);
+            }
+            if (g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
+            uint32_t r = 1;
+            for (;;) {
+                TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.pcount, 4, cudaMemcpyDeviceToHost, s));
+                TG_TRY_CUDA(cudaStreamSynchronize(s));
+                if (Q.h_ctr[0] == 0) break;
+                if (r > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
+                TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
+                for (int pi = 0; pi < g->nparts; pi++) {
+                    if (parts[pi].ub0 == parts[pi].ub1) {
+                        // an empty range still has to advance its round counter in lockstep
+                        TG_LAUNCH(k_eat_chain, grid, QT, 0, s, parts[pi]);
+                        continue;
+                    }
+                    TG_LAUNCH(k_eat_activate, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH(k_eat_big, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH(k_eat_chain, grid, QT, 0, s, parts[pi]);
+                }
+                // exchange: every rank ends the round with the elementwise min of all ranks' states
+                if (g->comm) TG_TRY(tg_comm_allreduce_min_u64(g->comm, Q.st, (uint64_t)Sb * n, s));
+                uint32_t *fnext = ((r + 1) & 1) ? Q.fb[1] : Q.fb[0];
+                for (int pi = 0; pi < g->nparts; pi++)
+                    TG_LAUNCH(k_part_frontier, grid, 256, 0, s, Q.st, Q.lat, fnext, Sb, G, g->part_vb[pi],
+                              g->part_vb[pi + 1], Q.pcount);
+                if (g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
+                r++;
+                rounds = r - 1;
+            }
+        }
         g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;
         uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;

@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "../../include/tg.h"
 
@@ -51,8 +52,7 @@ void tg_prof_end(const char *name, cudaStream_t s, cudaEvent_t ev0);
 // Simple owning device buffer list for a graph handle.
 struct DevArena {
     struct Blk { void *p; size_t bytes; };
-    Blk blks[96];
-    int nb = 0;
+    std::vector<Blk> blks;
     size_t total = 0;
     tg_status alloc(void **p, size_t bytes);
     void free_all();
@@ -123,13 +123,19 @@ struct QueryScratch {
     uint4 *chq = nullptr;    // long chain walks {q, s_begin, s_end, -}
     uint64_t chcap = 0;
     uint32_t *ctr = nullptr;   // counters [2][4] (SP/FP host-driven loop)
-    struct RoundCtl *ctl = nullptr;  // device-side round control (EAT family)
+    struct RoundCtl *ctl = nullptr;  // device-side round control (EAT family), [TG_MAXP]
+    uint32_t *lat = nullptr;         // partitioned mode: last activated arrival [v][q]
+    uint32_t *pcount = nullptr;      // partitioned mode: frontier bits of the next round
     uint32_t *h_ctr = nullptr; // pinned host mirror
     uint32_t *srcs = nullptr;  // [S] sources of the sub-batch
     unsigned long long *relax_cnt = nullptr;  // [S]
     uint32_t *out_stage = nullptr, *pred_stage = nullptr;  // [S][n] when out is host memory
     DevArena arena;
 };
+
+#define TG_MAXP 16  // logical vertex-range partitions per process (tests / one rank's share)
+
+struct tg_comm;  // comm.cu: NCCL communicator (loaded with dlopen)
 
 struct tg_graph {
     int device = 0;
@@ -141,6 +147,14 @@ struct tg_graph {
     bool built = false;
     double build_ms = 0;
     ChainGraph fwd, mir;
+    // vertex-range partitions (multi-GPU mode 1, or logical partitions on one GPU):
+    // partition p owns vertices [part_vb[p], part_vb[p+1]); pf/pm hold its chains
+    int nparts = 0;                 // 0 = not partitioned
+    int opt_partitions = 1;         // logical partitions requested via tg_set_option
+    uint32_t part_vb[TG_MAXP + 1] = {0};
+    ChainGraph pf[TG_MAXP], pm[TG_MAXP];
+    tg_comm *comm = nullptr;
+    int comm_mode = 0;              // 0 replicated (source sharding), 1 vertex range
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
@@ -163,8 +177,10 @@ tg_status tg_exclusive_scan_u32(const uint32_t *in, uint32_t *out, uint64_t coun
 tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
                               unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s);
 
-tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, const uint32_t *u, const uint32_t *v,
-                             const uint32_t *t, const uint32_t *dur, const uint32_t *w, cudaStream_t s);
+tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
+                             const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
+                             cudaStream_t s);
+tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s);
 
 tg_status tg_run_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                        uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);

@@ -26,7 +26,8 @@ TG_TMAX = 0x7FFFFFFE
 
 EXPORTED = ["tg_graph_create", "tg_build_chains", "tg_query", "tg_graph_destroy", "tg_status_string",
             "tg_last_error", "tg_graph_info", "tg_export_chains", "tg_last_query_stats", "tg_set_option",
-            "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report", "tg_release_cached_memory"]
+            "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report", "tg_release_cached_memory",
+            "tg_nccl_unique_id", "tg_comm_create", "tg_comm_destroy", "tg_graph_attach_comm"]
 
 
 class TGError(RuntimeError):
@@ -87,6 +88,14 @@ def load_library(path: str = LIB_PATH):
     lib.tg_set_option.argtypes = [P, ctypes.c_char_p, i64]
     lib.tg_kernel_launch_count.restype = u64
     lib.tg_kernel_launch_count.argtypes = []
+    lib.tg_nccl_unique_id.restype = st
+    lib.tg_nccl_unique_id.argtypes = [P]
+    lib.tg_comm_create.restype = st
+    lib.tg_comm_create.argtypes = [P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.POINTER(P)]
+    lib.tg_comm_destroy.restype = None
+    lib.tg_comm_destroy.argtypes = [P]
+    lib.tg_graph_attach_comm.restype = st
+    lib.tg_graph_attach_comm.argtypes = [P, P, ctypes.c_int]
     lib.tg_release_cached_memory.restype = None
     lib.tg_release_cached_memory.argtypes = []
     lib.tg_profile_enable.restype = None
@@ -186,6 +195,27 @@ def tg_set_option(g, key: str, value: int):
 
 def tg_kernel_launch_count() -> int:
     return int(load_library().tg_kernel_launch_count())
+
+
+def tg_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(load_library().tg_nccl_unique_id(buf))
+    return buf.raw
+
+
+def tg_comm_create(unique_id: bytes, rank: int, world: int, device: int):
+    h = ctypes.c_void_p()
+    buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+    _check(load_library().tg_comm_create(buf, int(rank), int(world), int(device), ctypes.byref(h)))
+    return h
+
+
+def tg_comm_destroy(c):
+    load_library().tg_comm_destroy(c)
+
+
+def tg_graph_attach_comm(g, c, mode: int):
+    _check(load_library().tg_graph_attach_comm(g, c, int(mode)))
 
 
 def tg_release_cached_memory():

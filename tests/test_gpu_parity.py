@@ -256,3 +256,53 @@ def test_abi_errors_on_gpu(tg):
     with pytest.raises(tg.TGError) as e:
         tg.tg_query(g.h, tg.TG_SHORTEST, [0], (0, 10), out, pred=out)
     assert e.value.status == 1
+
+
+# --------------------------------------------------------------------------- vertex-range partitions
+@pytest.mark.parametrize("parts", [2, 3, 5])
+def test_logical_partitions_random(tg, parts):
+    """Multi-GPU mode 1 (vertex-range partitions + state exchange) run as logical
+    partitions on one GPU: bit-exact, including preds and first-touch W."""
+    for seed in range(6):
+        rng = np.random.default_rng(seed + 77)
+        n, m = 400, 5000
+        u = rng.integers(0, n, m).astype(np.uint32); v = rng.integers(0, n, m).astype(np.uint32)
+        t = rng.integers(0, 300, m).astype(np.uint32); lam = rng.integers(1, 6, m).astype(np.uint32)
+        g = _gpu_graph(tg, n, u, v, t, lam, partitions=parts, stats=1)
+        og = oracle.Graph(n, u, v, t, lam)
+        srcs = [int(x) for x in rng.choice(n, 40, replace=False)]
+        for win in [(0, 10**6), (30, 200)]:
+            for p in ("eat", "ld", "reach"):
+                _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
+
+
+def test_logical_partitions_c1(tg):
+    ge = tgsynth.make_graph("C1")
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, w, partitions=4)
+    og = oracle.Graph(n, u, v, t, d, w)
+    for win in tgsynth.CONFIGS["C1"]["windows"]:
+        _check_rows(tg, g, og, "eat", [0, 5, 99], win)
+        _check_rows(tg, g, og, "ld", [0, 5], win)
+    with pytest.raises(tg.TGError):
+        g.query("sp", [0], (0, 10))  # partitioned graphs answer EAT/LD/REACH only
+
+
+def test_nccl_comm_world1_vertex_range(tg):
+    """The NCCL path of mode 1 with world = 1 (one GPU available): communicator
+    creation, attach, per-round ncclAllReduce(min) and the count reduction."""
+    import torch
+    from paper_conf_asplos_0003wh0dhwy0lyl25_b200 import distributed as tgd
+    ge = tgsynth.make_graph("C2", scale_shift=-6)
+    n, u, v, t, d, w = ge.numpy()
+    comm = tgd.make_comm(0, 1, 0)
+    f = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.uint32).view(np.int32)).cuda()
+    g = tg.Graph(n, f(u), f(v), f(t), f(d), device=0)
+    tg.tg_graph_attach_comm(g.h, comm, 1)
+    g.build()
+    og = oracle.Graph(n, u, v, t, d)
+    srcs = tgsynth.config_sources("C2", ge, k=8)
+    _check_rows(tg, g, og, "eat", srcs, (0, 10**9))
+    _check_rows(tg, g, og, "ld", srcs, (0, 10**9))
+    g.close()
+    tg.tg_comm_destroy(comm)
