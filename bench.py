@@ -48,6 +48,11 @@ def parse_args():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-profile", action="store_true", help="do not bracket kernels with CUDA events")
     ap.add_argument("--query-only", action="store_true", help="time only tg_query (graph built once)")
+    ap.add_argument("--mode", choices=["replicate", "vertex"], default="replicate",
+                    help="multi-GPU mode: replicate = source sharding (weak scaling); vertex = one batch "
+                         "partitioned by vertex range with per-round ncclAllReduce(min) (strong scaling)")
+    ap.add_argument("--partitions", type=int, default=1, help="logical vertex-range partitions per GPU")
+    ap.add_argument("--cpu-queries", type=int, default=2, help="oracle queries per problem in cpu_baseline")
     return ap.parse_args()
 
 
@@ -112,15 +117,25 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------------------- workload
-def workload(cfg_name, k_per_rank, rank, world, device):
+def default_k(cfg_name, cfg):
+    # per-rank sources per problem: the config's batch, capped at 64 (C4's 1024 are
+    # answered 64 per rank per step, weak scaling)
+    return min(cfg["k"], 64)
+
+
+def workload(cfg_name, k_per_rank, rank, world, device, mode="replicate"):
     import tgsynth
+    from paper_conf_asplos_0003wh0dhwy0lyl25_b200.distributed import shard_sources
     cfg = tgsynth.CONFIGS[cfg_name]
     ge = tgsynth.make_graph(cfg_name, device=device)
-    k = k_per_rank if k_per_rank else cfg["k"]
-    all_src = tgsynth.config_sources(cfg_name, ge, k=k * world)
-    if len(all_src) < k * world:  # small graphs: cycle
-        all_src = (all_src * (k * world // max(1, len(all_src)) + 1))[: k * world]
-    mine = all_src[rank * k:(rank + 1) * k]
+    k = k_per_rank if k_per_rank else default_k(cfg_name, cfg)
+    if mode == "vertex":  # one batch, every rank answers all of it cooperatively
+        mine = tgsynth.config_sources(cfg_name, ge, k=k)
+    else:
+        all_src = tgsynth.config_sources(cfg_name, ge, k=k * world)
+        if len(all_src) < k * world:  # small graphs: cycle
+            all_src = (all_src * (k * world // max(1, len(all_src)) + 1))[: k * world]
+        mine = shard_sources(all_src, rank, world)
     problems = [p for p in cfg["problems"] if p in ("eat", "ld")] or ["eat"]
     win = cfg["windows"][0]
     weighted = cfg["kind"] == "wikitalk"
@@ -154,17 +169,27 @@ def run_ours(a, rank, world, local_rank):
     dev = torch.device("cuda", local_rank)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
-    ge, mine, problems, win, weighted, cfg = workload(a.config, a.k, rank, world, dev)
+    ge, mine, problems, win, weighted, cfg = workload(a.config, a.k, rank, world, dev, a.mode)
     k = len(mine)
     n, m = ge.n, ge.m
     w_arg = ge.w if weighted else None
     outs = {p: torch.empty((k, n), dtype=torch.int32, device=dev) for p in problems}
     torch.cuda.synchronize()
+    comm = None
+    if a.mode == "vertex":
+        from paper_conf_asplos_0003wh0dhwy0lyl25_b200.distributed import make_comm
+        comm = make_comm(rank, world, local_rank, bcast_device=dev)
 
     def make_graph():
         g = tg.Graph(n, ge.u, ge.v, ge.t, ge.dur, w_arg, device=local_rank)
         if a.sub_batch:
             g.set_option("sub_batch", a.sub_batch)
+        if "ld" not in problems:
+            g.set_option("mirror", 0)
+        if a.partitions > 1:
+            g.set_option("partitions", a.partitions)
+        if comm is not None:
+            tg.tg_graph_attach_comm(g.h, comm, 1)
         return g.build()
 
     persistent = make_graph() if a.query_only else None
@@ -230,7 +255,7 @@ def run_ours(a, rank, world, local_rank):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
 
-    queries_per_step = k * len(problems) * world
+    queries_per_step = k * len(problems) * (world if a.mode == "replicate" else 1)
     value = queries_per_step / (ms / 1e3)
 
     # roofline of the dominant kernel group
@@ -243,6 +268,8 @@ def run_ours(a, rank, world, local_rank):
         dom = max(kprof.items(), key=lambda kv: kv[1][1])
         total_kernel_ms = sum(v[1] for v in kprof.values())
         W_total = sum(W_by_problem.values()) * a.steps
+        if a.mode == "vertex" and world > 1:
+            W_total = W_total / world  # per-rank relax kernels see ~1/N of the batch's work
         relax_bytes = 28 * W_total
         roof = {
             "bound": "hbm",
@@ -265,12 +292,12 @@ def run_ours(a, rank, world, local_rank):
         }
 
     e2e = None
-    if not a.no_e2e:
+    if not a.no_e2e and comm is None:
         e2e = run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev)
 
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
-        cpu = cpu_baseline(ge, mine, problems, win, weighted)
+        cpu = cpu_baseline(ge, mine, problems, win, weighted, n_sample=a.cpu_queries)
 
     res = {
         "metric": "EAT (+LD) temporal-path queries/s; temporal-edges/s and relax-phase HBM GB/s in extras",
@@ -281,13 +308,15 @@ def run_ours(a, rank, world, local_rank):
         "warmup": a.warmup,
         "ms_per_step": ms,
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "weak" if a.mode == "replicate" else "strong",
         "vs_baseline": None,
         "dtype": "u32",
         "data": "synthetic",
         "config": {
             "workload": describe(a.config, ge, k, problems, win),
-            "parallelism": f"source-sharded x{world} (replicated graph, no data-path collective)",
+            "parallelism": (f"source-sharded x{world} (replicated graph, no data-path collective)"
+                            if a.mode == "replicate" else
+                            f"vertex-range x{world} (one batch; per-round ncclAllReduce(min) of packed states)"),
             "step": "create+validate, build_chains (fwd+mirror), " + " + ".join(f"{p} x{k}" for p in problems),
             "query_only": a.query_only,
             "l2": "inputs larger than L2 (edge list %.0f MB, chain structure %.0f MB > 126 MB)" % (
@@ -295,7 +324,7 @@ def run_ours(a, rank, world, local_rank):
             "sub_batch": a.sub_batch or "auto",
         },
         "teps_graph": value * m / 1.0,  # queries/s x |E|: the paper-comparable |E|-normalised rate
-        "teps_work": (sum(W_by_problem.values()) * world) / (ms / 1e3),
+        "teps_work": (sum(W_by_problem.values()) * (world if a.mode == "replicate" else 1)) / (ms / 1e3),
         "W_per_query": {p: W_by_problem[p] / k for p in problems},
         "rounds": rounds,
         "graph": {"n": n, "m": m, "nodes": info["n_nodes"], "chains": info["n_chains"],
@@ -309,11 +338,14 @@ def run_ours(a, rank, world, local_rank):
     }
     if rank == 0:
         print(json.dumps(res), flush=True)
+    if comm is not None:
+        tg.tg_comm_destroy(comm)
     if world > 1:
         dist.destroy_process_group()
 
 
 def run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev):
+    # (not run in vertex mode: there every rank needs the communicator on its graph)
     """Same metric through the public C-ABI with HOST buffers: pinned host edge arrays
     -> tg_graph_create (H2D inside) -> build -> tg_query into pinned host outputs (D2H inside)."""
     import torch
@@ -327,6 +359,8 @@ def run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev):
         g = tg.Graph(n, hu, hv, ht, hd, hw, device=dev.index)
         if a.sub_batch:
             g.set_option("sub_batch", a.sub_batch)
+        if "ld" not in problems:
+            g.set_option("mirror", 0)
         g.build()
         for p in problems:
             tg.tg_query(g.h, tg.PROBLEMS[p], mine, win, houts[p])

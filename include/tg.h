@@ -99,7 +99,8 @@ TG_API tg_status tg_graph_create(uint32_t n_vertices, uint64_t n_edges,
  * are departure nodes (v, tau) (reading A11), with hubs per Def. 2 (P:L174,
  * P:L225); generate one shortcut per chain (Alg. 2); build the vertex ->
  * occurrence index that replaces the paper's GPU hash table.  The same
- * is done for the time-mirrored graph used by TG_LD (reading A5).  Idempotent.
+ * is done for the time-mirrored graph used by TG_LD (reading A5) unless option
+ * "mirror" is 0, in which case the first TG_LD query builds it.  Idempotent.
  * Runs on the legacy default stream and returns when finished.
  */
 TG_API tg_status tg_build_chains(tg_graph *g);
@@ -202,6 +203,7 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *   "stats"      1 = count relaxations per query (slower), 0 = off
  *   "shortcuts"  1 = relax chain tails through shortcuts on first entry (default), 0 = off
  *   "round_group" rounds launched between host convergence checks (default 4)
+ *   "mirror"     1 = build the LD mirror in tg_build_chains (default), 0 = on first LD query
  *   "partitions" logical vertex-range partitions on this GPU (1..16, before build):
  *                runs the multi-GPU mode-1 algorithm inside one process (tests) */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);

@@ -294,7 +294,10 @@ tg_status tg_build_chains(tg_graph *g) {
             TG_TRY(tg_build_partition(g, &g->pf[p], &g->pm[p], g->part_vb[p], g->part_vb[p + 1], 0));
     } else {
         TG_TRY(tg_build_direction(g, &g->fwd, g->m, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, nullptr, 0));
-        TG_TRY(tg_build_mirror(g, 0));
+        if (g->opt_mirror) {
+            TG_TRY(tg_build_mirror(g, 0));
+            g->mirror_built = true;
+        }
     }
     TG_TRY_CUDA(cudaDeviceSynchronize());
     g->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
@@ -331,6 +334,10 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
             return TG_ERR_STATE;
         }
         return tg_run_eat_partitioned(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
+    }
+    if (p == TG_LD && !g->mirror_built) {  // lazily built mirror (option "mirror" = 0)
+        TG_TRY(tg_build_mirror(g, 0));
+        g->mirror_built = true;
     }
     if (p == TG_EAT || p == TG_LD || p == TG_REACH)
         return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
@@ -376,6 +383,7 @@ tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off,
     if (!g || !chain_off || !chain_edges) { tg_set_error("NULL argument"); return TG_ERR_INVALID; }
     if (!g->built) { tg_set_error("graph not built"); return TG_ERR_STATE; }
     if (g->nparts > 0) { tg_set_error("chain export is for unpartitioned graphs"); return TG_ERR_STATE; }
+    if (mirrored && !g->mirror_built) { tg_set_error("the mirror graph has not been built"); return TG_ERR_STATE; }
     DeviceGuard dg(g->device);
     const ChainGraph &c = mirrored ? g->mir : g->fwd;
     const uint64_t m = g->m, nc = c.nchains;
@@ -436,6 +444,7 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     else if (k == "stats") g->opt_stats = value;
     else if (k == "shortcuts") g->opt_shortcuts = value;
     else if (k == "round_group") g->opt_round_group = value;
+    else if (k == "mirror") g->opt_mirror = value ? 1 : 0;
     else if (k == "partitions") {
         if (g->built) { tg_set_error("set partitions before tg_build_chains"); return TG_ERR_STATE; }
         if (value < 1 || value > TG_MAXP) { tg_set_error("partitions must be in [1, 16]"); return TG_ERR_RANGE; }

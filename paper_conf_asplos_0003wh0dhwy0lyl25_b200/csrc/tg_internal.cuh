@@ -163,6 +163,8 @@ struct tg_graph {
     int64_t opt_stats = 0;
     int64_t opt_shortcuts = 1;
     int64_t opt_round_group = 4;
+    int opt_mirror = 1;        // build the LD mirror in tg_build_chains (else on the first LD query)
+    bool mirror_built = false;
     // last query statistics
     tg_query_stats last{};
     uint64_t *last_relax = nullptr;  // host, per query
