@@ -217,6 +217,13 @@ def run_ours(a, rank, world, local_rank):
     for p in problems:
         gstat.query(p, mine, win, out=outs[p])
         W_by_problem[p] = int(gstat.last_stats(k)["per_query_relax"].sum())
+    W_global = sum(W_by_problem.values())
+    if a.mode == "vertex" and world > 1:
+        t = torch.tensor([float(W_global)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t)
+        W_global = float(t.item())
+    elif a.mode == "replicate":
+        W_global *= world  # every rank answers its own block (same distribution)
     rounds = {p: None for p in problems}
     gstat.set_option("stats", 0)
     for p in problems:
@@ -267,9 +274,8 @@ def run_ours(a, rank, world, local_rank):
         relax_launches = sum(kprof[x][0] for x in relax_names)
         dom = max(kprof.items(), key=lambda kv: kv[1][1])
         total_kernel_ms = sum(v[1] for v in kprof.values())
+        # in vertex mode the stats counter counts this rank's relaxations (its partition)
         W_total = sum(W_by_problem.values()) * a.steps
-        if a.mode == "vertex" and world > 1:
-            W_total = W_total / world  # per-rank relax kernels see ~1/N of the batch's work
         relax_bytes = 28 * W_total
         roof = {
             "bound": "hbm",
@@ -324,7 +330,7 @@ def run_ours(a, rank, world, local_rank):
             "sub_batch": a.sub_batch or "auto",
         },
         "teps_graph": value * m / 1.0,  # queries/s x |E|: the paper-comparable |E|-normalised rate
-        "teps_work": (sum(W_by_problem.values()) * (world if a.mode == "replicate" else 1)) / (ms / 1e3),
+        "teps_work": W_global / (ms / 1e3),
         "W_per_query": {p: W_by_problem[p] / k for p in problems},
         "rounds": rounds,
         "graph": {"n": n, "m": m, "nodes": info["n_nodes"], "chains": info["n_chains"],
