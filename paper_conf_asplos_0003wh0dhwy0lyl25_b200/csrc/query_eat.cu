@@ -548,11 +548,12 @@ uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
     if (!nodes_state) return std::min<uint32_t>(k, 64);
     const uint64_t n = g->n;
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
-    uint64_t hot = n * (8 + 4) + n / 4 + g->m / 8 + 64;
-    if (nodes_state) hot = nnodes * (4 + 4) + n * 4 + 64;
-    const uint64_t budget = 64ull << 20;
+    // SP/FP: per query node state + stamps + output; rounds are shared by a sub-batch,
+    // so batch as many queries as a 4 GiB state budget allows (at most 32)
+    const uint64_t hot = nnodes * (4 + 4 + 8) + n * 4 + 64;
+    const uint64_t budget = 4ull << 30;
     uint64_t S = std::max<uint64_t>(1, budget / hot);
-    S = std::min<uint64_t>(S, 64);
+    S = std::min<uint64_t>(S, 32);
     return (uint32_t)std::min<uint64_t>(S, k);
 }
 

@@ -35,7 +35,7 @@ namespace {
 constexpr int QT = 256;
 constexpr uint32_t BIG_T = 256;
 constexpr uint32_t CHUNK = 1024;
-constexpr uint32_t WAIT_MAX = 64;  // wait-propagation steps per item per round
+constexpr uint32_t WAIT_MAX = 2048;  // wait-propagation steps per item per round
 
 struct SpP {
     const uint32_t *vnode_off, *node_t, *node_u, *node_eoff, *occ_slot, *occ_node;
