@@ -204,6 +204,9 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *   "shortcuts"  1 = relax chain tails through shortcuts on first entry (default), 0 = off
  *   "round_group" rounds launched between host convergence checks (default 4)
  *   "mirror"     1 = build the LD mirror in tg_build_chains (default), 0 = on first LD query
+ *   "walk_min"   chains with at least this many edges are walked by the chain engine
+ *                (default 6, min 2, before build); shorter chains are relaxed edge by
+ *                edge through their own occurrences (P:L322's RemoveChain, generalised)
  *   "partitions" logical vertex-range partitions on this GPU (1..16, before build):
  *                runs the multi-GPU mode-1 algorithm inside one process (tests) */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);

@@ -409,15 +409,16 @@ tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off,
             TG_TRY_CUDA(cudaMemcpy(dur.data(), g->d_dur, m * 4, cudaMemcpyDeviceToHost));
             for (uint64_t s = 0; s < m; s++) t[s] = (uint32_t)slots[s].y - dur[(uint32_t)slots[s].z];
         }
+        uint32_t l = 0;  // long-chain index: chains with >= 2 edges numbered in chain order
         for (uint64_t ch = 0; ch < nc; ch++) {
             uint32_t b = first[ch], e = first[ch + 1];
             int4 sl = slots[b];
             if (e - b >= 2) {
-                uint32_t l = (uint32_t)sl.w;
                 if (sc_tail_v) sc_tail_v[ch] = (uint32_t)sc[l].x;
                 if (sc_arr) sc_arr[ch] = (uint32_t)sc[l].y;
                 if (sc_sum_w) sc_sum_w[ch] = sumw[l];
                 if (sc_elapsed) sc_elapsed[ch] = el[l];
+                l++;
             } else {  // Alg. 2 line 8: a one-edge chain is its own shortcut
                 if (sc_tail_v) sc_tail_v[ch] = (uint32_t)sl.x;
                 if (sc_arr) sc_arr[ch] = (uint32_t)sl.y;
@@ -445,6 +446,11 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     else if (k == "shortcuts") g->opt_shortcuts = value;
     else if (k == "round_group") g->opt_round_group = value;
     else if (k == "mirror") g->opt_mirror = value ? 1 : 0;
+    else if (k == "exp") g->opt_exp = value;
+    else if (k == "walk_min") {
+        if (g->built) { tg_set_error("set walk_min before tg_build_chains"); return TG_ERR_STATE; }
+        g->opt_walk_min = value < 2 ? 2 : value;
+    }
     else if (k == "partitions") {
         if (g->built) { tg_set_error("set partitions before tg_build_chains"); return TG_ERR_STATE; }
         if (value < 1 || value > TG_MAXP) { tg_set_error("partitions must be in [1, 16]"); return TG_ERR_RANGE; }

@@ -144,20 +144,24 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
                                 uint32_t *__restrict__ slot_tn, uint32_t *__restrict__ occ_slot,
                                 uint2 *__restrict__ lc, int4 *__restrict__ sc,
                                 unsigned long long *__restrict__ sc_sumw, uint32_t *__restrict__ sc_elapsed,
-                                const uint32_t *__restrict__ id_map) {
+                                const uint32_t *__restrict__ id_map, uint32_t walk_min) {
     GRID_STRIDE(p, m) {
         if (!head[p]) continue;
         uint32_t c = cidx[p];
         uint32_t first = chain_first[c];
         uint32_t len = chain_len[c];
-        uint32_t l = (len >= 2) ? lidx[c] : TG_SINGLE;
+        const uint32_t l = (len >= 2) ? lidx[c] : TG_SINGLE;
+        // slots of chains shorter than walk_min are marked SINGLE: the query engines
+        // relax them edge by edge through their own occurrences (RemoveChain, P:L322,
+        // generalised); longer chains are walked.  lc/sc are generated for every chain.
+        const uint32_t cw = (len >= walk_min) ? l : TG_SINGLE;
         uint32_t s = first;
         uint32_t q = p, last = p;
         unsigned long long sumw = 0;
         while (q != TG_NONE) {
             uint32_t e = sid[q];
             uint32_t w = Wt[e];
-            slots[s] = make_int4((int)s_v[q], (int)s_arr[q], (int)(id_map ? id_map[e] : e), (int)l);
+            slots[s] = make_int4((int)s_v[q], (int)s_arr[q], (int)(id_map ? id_map[e] : e), (int)cw);
             slot_w[s] = w;
             slot_tn[s] = tn[q];
             occ_slot[q] = s;
@@ -394,7 +398,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_TRY(A.alloc((void **)&cg->sc_elapsed, std::max<uint64_t>(L, 1) * 4));
     TG_LAUNCH(k_chain_scatter, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, cg->chain_first, chain_len, lidx, sid,
               s_v, s_arr, tn, node_of, t, w, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
-              cg->sc_sumw, cg->sc_elapsed, id_map);
+              cg->sc_sumw, cg->sc_elapsed, id_map, (uint32_t)std::max<int64_t>(2, g->opt_walk_min));
 
     for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)s_v, (void *)s_arr, (void *)hub,
                     (void *)head, (void *)succ, (void *)cidx, (void *)chain_len, (void *)lidx})

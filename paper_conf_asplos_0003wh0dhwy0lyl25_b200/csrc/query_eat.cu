@@ -59,7 +59,8 @@ struct EatP {
     uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
     uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
     uint32_t alpha, omega;
-    int use_sc, stats;
+    int use_sc, stats, exp;
+  // exp: diagnostic variants for timing only (results invalid when != 0)
     RoundCtl *ctl;
     uint32_t *fb0, *fb1;  // frontier masks [n][G] (bit = query within the group), by round parity
     uint2 *recs;          // big-unit records: 32 per-query ranges each
@@ -248,7 +249,9 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
             if (t < total) {
                 const uint32_t ql = __fns(om, 0, (int)(t - oex) + 1);  // (t-oex)-th set bit of the edge's mask
                 const uint32_t q = g * 32 + ql;
-                if ((uint32_t)osl.w == TG_SINGLE) eat_relax(P, R, q, (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
+                if (P.exp == 2) continue;  // diagnostic: enumeration only
+                if ((uint32_t)osl.w == TG_SINGLE || P.exp == 1)
+                    eat_relax(P, R, q, (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
                 else eat_long(P, R, q, os, osl);
             }
         }
@@ -582,7 +585,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
         P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
         P.ub0 = 0; P.ub1 = g->n * G;
-        P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
+        P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats; P.exp = (int)g->opt_exp;
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         const uint32_t grid = tg_grid_persistent(8);

@@ -63,7 +63,7 @@ struct DevArena {
 //   departure nodes (v, tau) in (v, tau) order:   vnode_off[n+1], node_t[N], node_u[N], node_eoff[N+1]
 //   sorted edges (by (u, t, id)), "occurrences": occ_slot[m] -> slot index, occ_node[m] -> node
 //   slots in chain-major order (chains ordered by head (u, t, first id)):
-//       slots int4[m] = {v, arr = t + duration, edge id, long-chain index | TG_SINGLE}
+//       slots int4[m] = {v, arr = t + duration, edge id, long-chain index of a walked chain | TG_SINGLE}
 //       slot_w[m], slot_tn[m] (tail departure node or TG_NONE)   -- SP/FP only
 //   long chains (>= 2 edges): lc uint2[L] = {first slot, length}
 //                             sc int4[L]  = {tail v, tail arrival, tail edge id, head node}
@@ -163,7 +163,9 @@ struct tg_graph {
     int64_t opt_stats = 0;
     int64_t opt_shortcuts = 1;
     int64_t opt_round_group = 4;
-    int opt_mirror = 1;        // build the LD mirror in tg_build_chains (else on the first LD query)
+    int opt_mirror = 1;
+    int64_t opt_exp = 0;
+    int64_t opt_walk_min = 6;  // chains with fewer edges are not walked (RemoveChain threshold, build time)       // diagnostic kernel variants (timing experiments only)        // build the LD mirror in tg_build_chains (else on the first LD query)
     bool mirror_built = false;
     // last query statistics
     tg_query_stats last{};

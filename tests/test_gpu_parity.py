@@ -89,6 +89,18 @@ def test_tiny_random_all_problems(tg, seed):
             _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
 
 
+@pytest.mark.parametrize("walk_min", [2, 6])
+def test_walk_threshold(tg, walk_min):
+    """Every chain walked (walk_min = 2) and the default threshold give identical,
+    exact results and the same first-touch work."""
+    for seed in range(4):
+        n, u, v, t, lam, w = tgsynth.tiny_random(seed + 900, n_max=60, m_max=900, t_max=40, lam_max=4)
+        g = _gpu_graph(tg, n, u, v, t, lam, w, walk_min=walk_min, stats=1)
+        og = oracle.Graph(n, u, v, t, lam, w)
+        for p in ("eat", "ld", "sp", "fp"):
+            _check_rows(tg, g, og, p, list(range(min(n, 12))), (0, 10**6), stats=(p == "eat"))
+
+
 @pytest.mark.parametrize("seed", range(6))
 def test_medium_random(tg, seed):
     rng = np.random.default_rng(seed)
@@ -205,7 +217,7 @@ def test_long_chain_and_hub(tg):
     H = 20000
     u += [0] * H; v += list(np.random.default_rng(0).integers(1, L + 1, H)); t += [0] * H; lam += [3] * H
     u, v, t, lam = (np.array(a, np.uint32) for a in (u, v, t, lam))
-    g = _gpu_graph(tg, L + 1, u, v, t, lam, stats=1)
+    g = _gpu_graph(tg, L + 1, u, v, t, lam, stats=1, walk_min=2)
     og = oracle.Graph(L + 1, u, v, t, lam)
     for win in [(0, 10**6), (0, 2500), (7, 4000)]:
         for p in ("eat", "ld", "sp", "fp"):
