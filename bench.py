@@ -213,10 +213,12 @@ def run_ours(a, rank, world, local_rank):
     # work counts (untimed): W per query from the engine's first-touch counter (== oracle W, tested)
     gstat = persistent or make_graph()
     gstat.set_option("stats", 1)
-    W_by_problem = {}
+    W_by_problem, Wu_by_problem = {}, {}
     for p in problems:
         gstat.query(p, mine, win, out=outs[p])
-        W_by_problem[p] = int(gstat.last_stats(k)["per_query_relax"].sum())
+        st = gstat.last_stats(k)
+        W_by_problem[p] = int(st["per_query_relax"].sum())
+        Wu_by_problem[p] = int(st["slots_union"])
     W_global = sum(W_by_problem.values())
     if a.mode == "vertex" and world > 1:
         t = torch.tensor([float(W_global)], dtype=torch.float64, device=dev)
@@ -274,9 +276,14 @@ def run_ours(a, rank, world, local_rank):
         relax_launches = sum(kprof[x][0] for x in relax_names)
         dom = max(kprof.items(), key=lambda kv: kv[1][1])
         total_kernel_ms = sum(v[1] for v in kprof.values())
-        # in vertex mode the stats counter counts this rank's relaxations (its partition)
+        # SURVEY 8(d), batched with source lanes: every slot relaxed by some query of a
+        # sub-batch is read once (16 B slot + 4 B occurrence), every relaxation touches
+        # 8 B of packed state: B = W_union * 20 + sum_q W_q * 8.  (In vertex mode the
+        # counters are this rank's, i.e. its partition's relaxations.)
         W_total = sum(W_by_problem.values()) * a.steps
-        relax_bytes = 28 * W_total
+        Wu_total = sum(Wu_by_problem.values()) * a.steps
+        relax_bytes = 20 * Wu_total + 8 * W_total
+        single_source_bytes = 28 * W_total
         roof = {
             "bound": "hbm",
             "kernel": "relax phase (k_eat_activate + k_eat_big + k_eat_chain: activation with inline "
@@ -288,6 +295,9 @@ def run_ours(a, rank, world, local_rank):
             "traffic": None,
             "peak_source": peak_src,
             "algorithmic_bytes_per_step": relax_bytes / a.steps,
+            "algorithmic_bytes_formula": "20 B x W_union + 8 B x sum_q W_q (SURVEY 8(d), batched source lanes)",
+            "W_union_per_step": Wu_total / a.steps,
+            "single_source_formula_GBps": single_source_bytes / (relax_ms / 1e3) / 1e9 if relax_ms else None,
             "relax_ms_per_step": relax_ms / a.steps,
             "relax_launches_per_step": relax_launches / a.steps,
             "relax_share_of_kernel_time": relax_ms / total_kernel_ms if total_kernel_ms else None,
@@ -332,6 +342,7 @@ def run_ours(a, rank, world, local_rank):
         "teps_graph": value * m / 1.0,  # queries/s x |E|: the paper-comparable |E|-normalised rate
         "teps_work": W_global / (ms / 1e3),
         "W_per_query": {p: W_by_problem[p] / k for p in problems},
+        "W_union": Wu_by_problem,
         "rounds": rounds,
         "graph": {"n": n, "m": m, "nodes": info["n_nodes"], "chains": info["n_chains"],
                   "long_chains": info["n_long_chains"], "max_chain_len": info["max_chain_len"],

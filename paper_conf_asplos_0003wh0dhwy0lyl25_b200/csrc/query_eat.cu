@@ -55,6 +55,7 @@ struct EatP {
     const int4 *sc;
     unsigned long long *st;
     uint32_t *act, *bits;
+    uint32_t *touched;  // stats: slots relaxed by any query of the sub-batch
     uint64_t bit_words;
     uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
     uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
@@ -115,11 +116,14 @@ __device__ __forceinline__ void round_advance(RoundCtl *ctl) {
 // Layouts interleave the S queries of a sub-batch (query index fastest):
 //   st / act [v * S + q], frontier masks [v * G + q / 32] (bit q % 32), claim words [(slot >> 5) * S + q],
 // so the queries of a sub-batch that touch the same vertex or slot touch adjacent words.
-__device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t v, uint32_t arr,
-                                          uint32_t id) {
+__device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t slot, uint32_t v,
+                                          uint32_t arr, uint32_t id) {
     const size_t i = (size_t)v * P.S + q;
     const unsigned long long pk = ((unsigned long long)arr << 32) | id;
-    if (P.stats) atomicAdd(P.relax_cnt + q, 1ull);
+    if (P.stats) {  // work counters: relaxations per query, distinct slots of the sub-batch
+        atomicAdd(P.relax_cnt + q, 1ull);
+        atomicOr(P.touched + (slot >> 5), 1u << (slot & 31));
+    }
     // States only decrease: a stale cached read is an upper bound, so when it is
     // already <= pk the atomic cannot change anything (most relaxations, W >> n).
     if (P.st[i] <= pk) return;
@@ -129,17 +133,6 @@ __device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32
         // no shared counter -- the next activation counts the non-empty words it finds)
         atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
     }
-}
-
-// Same, with the filter value already loaded (batched loads, see eat_edges).
-__device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, uint32_t q, uint32_t v, uint32_t arr,
-                                              uint32_t id, unsigned long long cur) {
-    const unsigned long long pk = ((unsigned long long)arr << 32) | id;
-    if (P.stats) atomicAdd(P.relax_cnt + q, 1ull);
-    if (cur <= pk) return;
-    const size_t i = (size_t)v * P.S + q;
-    const unsigned long long old = atomicMin(P.st + i, pk);
-    if (arr < (uint32_t)(old >> 32)) atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
 }
 
 // test-and-set of slot s's claim bit for query q; true if this caller claimed it
@@ -155,7 +148,7 @@ __device__ __forceinline__ void eat_walk(const EatP &P, const RoundV &R, uint32_
         const int4 sl = tg_ld_slot(P.slots + s);
         if ((uint32_t)sl.y > P.omega) return;  // arrivals increase strictly along a chain
         if (!claim(P, q, s)) return;
-        eat_relax(P, R, q, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+        eat_relax(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     }
 }
 
@@ -164,14 +157,14 @@ __device__ __forceinline__ void eat_long(const EatP &P, const RoundV &R, uint32_
     const uint32_t l = (uint32_t)sl.w;
     const uint2 info = __ldg(P.lc + l);  // {first slot, length}
     if (s != info.x && !claim(P, q, s)) return;  // a walker from an earlier entry got here first
-    eat_relax(P, R, q, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+    eat_relax(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     uint32_t s_end = info.x + info.y;
     if (s + 1 >= s_end) return;
     if (P.use_sc) {
         // skeleton: Propagate along the shortcut head -> tail (Alg. 2 / Alg. 3 line 6)
         const int4 scv = __ldg(P.sc + l);
         if ((uint32_t)scv.y <= P.omega && claim(P, q, s_end - 1)) {
-            eat_relax(P, R, q, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
+            eat_relax(P, R, q, s_end - 1, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
             s_end -= 1;
         }
     }
@@ -190,7 +183,7 @@ __device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_
     const uint32_t s = __ldg(P.occ_slot + p);
     const int4 sl = tg_ld_slot(P.slots + s);
     if ((uint32_t)sl.y > P.omega) return;
-    if ((uint32_t)sl.w == TG_SINGLE) eat_relax(P, R, q, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+    if ((uint32_t)sl.w == TG_SINGLE) eat_relax(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     else eat_long(P, R, q, s, sl);
 }
 
@@ -251,7 +244,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
                 const uint32_t q = g * 32 + ql;
                 if (P.exp == 2) continue;  // diagnostic: enumeration only
                 if ((uint32_t)osl.w == TG_SINGLE || P.exp == 1)
-                    eat_relax(P, R, q, (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
+                    eat_relax(P, R, q, os, (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
                 else eat_long(P, R, q, os, osl);
             }
         }
@@ -373,7 +366,7 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
                 if ((uint32_t)sl.y > P.omega) {
                     past = true;
                 } else if (claim(P, c.x, s)) {
-                    eat_relax(P, R, c.x, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+                    eat_relax(P, R, c.x, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
                     cont = true;
                 }
             }
@@ -474,6 +467,14 @@ __global__ void k_part_frontier(const unsigned long long *__restrict__ st, uint3
     if (lane == 0 && mine) atomicAdd(count, mine);
 }
 
+__global__ void k_popcount(const uint32_t *__restrict__ w, uint64_t nw, unsigned long long *__restrict__ out) {
+    unsigned long long c = 0;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x)
+        c += __popc(w[i]);
+    for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(out, c);
+}
+
 __global__ void k_ctl_reset(RoundCtl *ctl) {
     for (int i = 0; i < 4; i++)
         for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
@@ -533,7 +534,8 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     }
     TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
     TG_TRY(A.alloc((void **)&Q.srcs, S * 4));
-    TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8));
+    TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8 + 8));  // [S] per query + [S] = distinct slots
+    TG_TRY(A.alloc((void **)&Q.touched, ((m + 31) / 32 + TG_MAXP + 1) * 4));
     if (nodes_state) {
         TG_TRY(A.alloc((void **)&Q.dnode, std::max<uint64_t>(S * nnodes, 1) * 4));
         TG_TRY(A.alloc((void **)&Q.vout, S * n * 4));
@@ -573,7 +575,10 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     const uint32_t G = (S + 31) / 32;
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
-    if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8, s));
+    if (g->opt_stats) {
+        TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8 + 8, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
+    }
     const bool work = any_work && g->m > 0 && alpha < omega;
     TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
@@ -588,6 +593,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats; P.exp = (int)g->opt_exp;
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
+        P.touched = Q.touched;
         const uint32_t grid = tg_grid_persistent(8);
         static const bool trace = getenv("TG_TRACE") != nullptr;
         const int group = trace ? 1 : (int)std::max<int64_t>(1, g->opt_round_group);
@@ -653,10 +659,14 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (g->opt_stats) {
-            std::vector<unsigned long long> h(Sb);
-            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, Sb * 8, cudaMemcpyDeviceToHost, s));
+            const uint64_t tw = (g->m + 31) / 32 + TG_MAXP + 1;
+            TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, Q.touched, tw,
+                      Q.relax_cnt + Sb);
+            std::vector<unsigned long long> h(Sb + 1);
+            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, (Sb + 1) * 8, cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
             for (uint32_t q = 0; q < Sb; q++) { g->last_relax[b0 + q] = h[q]; g->last.slots_relaxed += h[q]; }
+            g->last.slots_union += h[Sb];
         }
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
@@ -710,7 +720,10 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
-        if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8, s));
+        if (g->opt_stats) {
+            TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8 + 8, s));
+            TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
+        }
         TG_LAUNCH(k_eat_init, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs, Sb, alpha, Q.fb[1], Q.ctl, 0);
         const bool work = any_work && g->m > 0 && alpha < omega;
         uint32_t rounds = 0;
@@ -728,6 +741,7 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 const ChainGraph &cg = ld ? g->pm[pi] : g->pf[pi];
                 EatP P = base;
                 P.bits = Q.bits + bit_off * Sb;
+                P.touched = Q.touched + bit_off;
                 bit_off += (cg.m + 31) / 32;
                 P.vnode_off = cg.vnode_off; P.node_t = cg.node_t; P.node_eoff = cg.node_eoff; P.occ_slot = cg.occ_slot;
                 P.slots = cg.slots; P.lc = cg.lc; P.sc = cg.sc;
@@ -778,10 +792,14 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (g->opt_stats) {
-            std::vector<unsigned long long> h(Sb);
-            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, Sb * 8, cudaMemcpyDeviceToHost, s));
+            const uint64_t tw = (g->m + 31) / 32 + TG_MAXP + 1;
+            TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, Q.touched, tw,
+                      Q.relax_cnt + Sb);
+            std::vector<unsigned long long> h(Sb + 1);
+            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, (Sb + 1) * 8, cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
             for (uint32_t q = 0; q < Sb; q++) { g->last_relax[b0 + q] = h[q]; g->last.slots_relaxed += h[q]; }
+            g->last.slots_union += h[Sb];
         }
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));

@@ -128,7 +128,8 @@ struct QueryScratch {
     uint32_t *pcount = nullptr;      // partitioned mode: frontier bits of the next round
     uint32_t *h_ctr = nullptr; // pinned host mirror
     uint32_t *srcs = nullptr;  // [S] sources of the sub-batch
-    unsigned long long *relax_cnt = nullptr;  // [S]
+    unsigned long long *relax_cnt = nullptr;  // [S] + distinct-slot count
+    uint32_t *touched = nullptr;              // stats: slots relaxed by any query of the sub-batch
     uint32_t *out_stage = nullptr, *pred_stage = nullptr;  // [S][n] when out is host memory
     DevArena arena;
 };

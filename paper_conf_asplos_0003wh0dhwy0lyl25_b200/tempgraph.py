@@ -50,7 +50,8 @@ class tg_info(ctypes.Structure):
 
 class tg_query_stats(ctypes.Structure):
     _fields_ = [("rounds", ctypes.c_uint32), ("sub_batches", ctypes.c_uint32),
-                ("slots_relaxed", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64)]
+                ("slots_relaxed", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64),
+                ("slots_union", ctypes.c_uint64)]
 
 
 _lib = None

@@ -160,6 +160,26 @@ def test_c2_small_batch(tg):
         _check_rows(tg, g, og, "ld", srcs[:16], win)
 
 
+def test_union_work_count(tg):
+    """W_union (distinct slots relaxed by any query of the sub-batch, the bench's
+    algorithmic-bytes input) equals the union of the oracle's usable valid edges."""
+    ge = tgsynth.make_graph("C2", scale_shift=-5)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, w, stats=1)
+    og = oracle.Graph(n, u, v, t, d, w)
+    srcs = tgsynth.config_sources("C2", ge, k=40)
+    win = (1000, 50000)
+    g.query("eat", srcs, win)
+    st = g.last_stats(len(srcs))
+    used = np.zeros(len(u), bool)
+    valid = (t >= win[0]) & (t.astype(np.int64) + d <= win[1])
+    for x in srcs:
+        A, _, _ = oracle.eat(og, x, *win)
+        used |= valid & (A[u] != NONE) & (A[u] <= t)
+    assert st["slots_union"] == int(used.sum())
+    assert st["slots_relaxed"] >= st["slots_union"]
+
+
 def test_c3_small_all_problems(tg):
     """configs[2] shape at 1/16 scale: wiki-talk-shaped, all four problems."""
     ge = tgsynth.make_graph("C3", scale_shift=-4)
