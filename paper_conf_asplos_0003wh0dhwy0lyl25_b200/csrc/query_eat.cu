@@ -193,8 +193,16 @@ __device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_
 // occurrence and slot once; a ballot per edge gives the queries for which that
 // edge is new; the (edge, query) pairs are compacted edge-major over the lanes,
 // so the queries of one edge read adjacent state words in one request.
+// Per-warp shared-memory staging of one 32-edge block: the (edge, query) pairs
+// as 16-bit (edge lane << 5 | query bit) entries, and the block's slots.
+struct WarpStage {
+    uint16_t pairs[1024];
+    int4 slot[32];
+    uint32_t sidx[32];
+};
+
 __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint32_t g, uint32_t lo, uint32_t hi,
-                                           uint32_t pbeg, uint32_t pend) {
+                                           uint32_t pbeg, uint32_t pend, WarpStage &ws) {
     const int lane = threadIdx.x & 31;
     for (uint32_t pb = pbeg; pb < pend; pb += 32) {
         const uint32_t p = pb + lane;
@@ -221,33 +229,28 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
             if (lane >= o) incl += y;
         }
         const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-        const uint32_t excl = incl - cnt;
-        for (uint32_t tb = 0; tb < total; tb += 32) {
-            const uint32_t t = tb + lane;
-            uint32_t own = 0;  // edge lane owning pair t
-#pragma unroll
-            for (int bb = 16; bb; bb >>= 1) {
-                const uint32_t v = __shfl_sync(0xffffffffu, incl, own + bb - 1);
-                if (v <= t) own += bb;
-            }
-            own &= 31;
-            const uint32_t om = __shfl_sync(0xffffffffu, mask, own);
-            const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
-            const uint32_t os = __shfl_sync(0xffffffffu, s, own);
-            int4 osl;
-            osl.x = __shfl_sync(0xffffffffu, sl.x, own);
-            osl.y = __shfl_sync(0xffffffffu, sl.y, own);
-            osl.z = __shfl_sync(0xffffffffu, sl.z, own);
-            osl.w = __shfl_sync(0xffffffffu, sl.w, own);
-            if (t < total) {
-                const uint32_t ql = __fns(om, 0, (int)(t - oex) + 1);  // (t-oex)-th set bit of the edge's mask
-                const uint32_t q = g * 32 + ql;
-                if (P.exp == 2) continue;  // diagnostic: enumeration only
-                if ((uint32_t)osl.w == TG_SINGLE || P.exp == 1)
-                    eat_relax(P, R, q, os, (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
-                else eat_long(P, R, q, os, osl);
-            }
+        if (total == 0) continue;
+        // expand: edge lane k writes its pairs at [incl - cnt, incl) in edge-major order
+        ws.slot[lane] = sl;
+        ws.sidx[lane] = s;
+        uint32_t pos = incl - cnt, mm = mask;
+        while (mm) {
+            const uint32_t bq = __ffs(mm) - 1;
+            mm &= mm - 1;
+            ws.pairs[pos++] = (uint16_t)((lane << 5) | bq);
         }
+        __syncwarp();
+        for (uint32_t t = lane; t < total; t += 32) {
+            const uint32_t e = ws.pairs[t];
+            const uint32_t k = e >> 5;
+            const uint32_t q = g * 32 + (e & 31);
+            const int4 osl = ws.slot[k];
+            if ((uint32_t)osl.w == TG_SINGLE)
+                eat_relax(P, R, q, ws.sidx[k], (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
+            else
+                eat_long(P, R, q, ws.sidx[k], osl);
+        }
+        __syncwarp();
     }
 }
 
@@ -260,6 +263,8 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
 // chunks for k_eat_big.
 __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
+    __shared__ WarpStage stage[QT / 32];
+    WarpStage &ws = stage[threadIdx.x >> 5];
     __shared__ uint32_t s_units;
     if (threadIdx.x == 0) s_units = 0;
     __syncthreads();
@@ -325,7 +330,7 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
                 }
                 // capacity exceeded (not expected: both are bounds): relax in place
             }
-            unit_range(P, R, g, lo, hi, ulo, uhi);
+            unit_range(P, R, g, lo, hi, ulo, uhi, ws);
         }
     }
     if (lane == 0 && my_units) atomicAdd(&s_units, my_units);
@@ -336,6 +341,8 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
 // Chunks of long unions: one warp per chunk, the unit's 32 query ranges from its record.
 __global__ void __launch_bounds__(QT, 8) k_eat_big(EatP P) {
     const RoundV R = round_view(P);
+    __shared__ WarpStage stage[QT / 32];
+    WarpStage &ws = stage[threadIdx.x >> 5];
     const uint32_t B = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.big_cnt, P.bigcap);
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -343,7 +350,7 @@ __global__ void __launch_bounds__(QT, 8) k_eat_big(EatP P) {
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
         const uint2 r = P.recs[(size_t)c.x * 32 + lane];
-        unit_range(P, R, c.w, r.x, r.y, c.y, c.z);
+        unit_range(P, R, c.w, r.x, r.y, c.y, c.z, ws);
     }
 }
 
