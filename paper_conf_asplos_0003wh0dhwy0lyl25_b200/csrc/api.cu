@@ -293,7 +293,7 @@ tg_status tg_build_chains(tg_graph *g) {
         for (int p = 0; p < P; p++)
             TG_TRY(tg_build_partition(g, &g->pf[p], &g->pm[p], g->part_vb[p], g->part_vb[p + 1], 0));
     } else {
-        TG_TRY(tg_build_direction(g, &g->fwd, g->m, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, nullptr, 0));
+        TG_TRY(tg_build_direction(g, &g->fwd, g->m, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, nullptr, g->max_t, 0));
         if (g->opt_mirror) {
             TG_TRY(tg_build_mirror(g, 0));
             g->mirror_built = true;

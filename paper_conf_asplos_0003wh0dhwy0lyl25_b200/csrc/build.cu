@@ -72,23 +72,26 @@ __global__ void k_vnode_off(const uint32_t *__restrict__ node_u, uint64_t nn, ui
     }
 }
 
+// AoS edge records in input order, {v, arrival, w, t}: one 16-byte gather per
+// sorted edge instead of several 4-byte ones
+__global__ void k_records(const uint32_t *__restrict__ V, const uint32_t *__restrict__ T,
+                          const uint32_t *__restrict__ DUR, const uint32_t *__restrict__ W, uint64_t m,
+                          uint4 *__restrict__ rec) {
+    GRID_STRIDE(i, m) rec[i] = make_uint4(V[i], T[i] + DUR[i], W[i], T[i]);
+}
+
 // snap each sorted edge to its tail departure node; count in-degrees
-__global__ void k_snap(const uint32_t *__restrict__ sid, uint64_t m, const uint32_t *__restrict__ V,
-                       const uint32_t *__restrict__ T, const uint32_t *__restrict__ DUR,
+__global__ void k_snap(const uint32_t *__restrict__ sid, uint64_t m, const uint4 *__restrict__ rec,
                        const uint32_t *__restrict__ vnode_off, const uint32_t *__restrict__ node_t,
-                       uint32_t *__restrict__ tn, uint32_t *__restrict__ s_v, uint32_t *__restrict__ s_arr,
-                       uint32_t *__restrict__ indeg) {
+                       uint32_t *__restrict__ tn, uint32_t *__restrict__ indeg) {
     GRID_STRIDE(p, m) {
-        uint32_t e = sid[p];
-        uint32_t v = V[e];
-        uint32_t arr = T[e] + DUR[e];
-        uint32_t lo = vnode_off[v], hi = vnode_off[v + 1];
-        uint32_t j = tg_lower_bound(node_t, lo, hi, arr);
-        uint32_t r = (j < hi) ? j : TG_NONE;
-        tn[p] = r;
-        s_v[p] = v;
-        s_arr[p] = arr;
-        if (r != TG_NONE) atomicAdd(&indeg[r], 1u);
+        const uint4 r = rec[sid[p]];
+        const uint32_t v = r.x, arr = r.y;
+        const uint32_t lo = vnode_off[v], hi = vnode_off[v + 1];
+        const uint32_t j = tg_lower_bound(node_t, lo, hi, arr);
+        const uint32_t x = (j < hi) ? j : TG_NONE;
+        tn[p] = x;
+        if (x != TG_NONE) atomicAdd(&indeg[x], 1u);
     }
 }
 
@@ -137,9 +140,8 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
                                 const uint32_t *__restrict__ succ, uint64_t m,
                                 const uint32_t *__restrict__ chain_first, const uint32_t *__restrict__ chain_len,
                                 const uint32_t *__restrict__ lidx, const uint32_t *__restrict__ sid,
-                                const uint32_t *__restrict__ s_v, const uint32_t *__restrict__ s_arr,
+                                const uint4 *__restrict__ rec,
                                 const uint32_t *__restrict__ tn, const uint32_t *__restrict__ node_of,
-                                const uint32_t *__restrict__ T, const uint32_t *__restrict__ Wt,
                                 int4 *__restrict__ slots, uint32_t *__restrict__ slot_w,
                                 uint32_t *__restrict__ slot_tn, uint32_t *__restrict__ occ_slot,
                                 uint2 *__restrict__ lc, int4 *__restrict__ sc,
@@ -156,26 +158,28 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
         // generalised); longer chains are walked.  lc/sc are generated for every chain.
         const uint32_t cw = (len >= walk_min) ? l : TG_SINGLE;
         uint32_t s = first;
-        uint32_t q = p, last = p;
+        uint32_t q = p;
         unsigned long long sumw = 0;
+        uint4 r0 = make_uint4(0, 0, 0, 0), r = r0;
+        uint32_t e = 0;
         while (q != TG_NONE) {
-            uint32_t e = sid[q];
-            uint32_t w = Wt[e];
-            slots[s] = make_int4((int)s_v[q], (int)s_arr[q], (int)(id_map ? id_map[e] : e), (int)cw);
-            slot_w[s] = w;
+            e = sid[q];
+            r = rec[e];
+            if (q == p) r0 = r;
+            slots[s] = make_int4((int)r.x, (int)r.y, (int)(id_map ? id_map[e] : e), (int)cw);
+            slot_w[s] = r.z;
             slot_tn[s] = tn[q];
             occ_slot[q] = s;
-            sumw += w;  // GenerateShortcut: accumulate W_e (Alg. 2 line 5)
-            last = q;
+            sumw += r.z;  // GenerateShortcut: accumulate W_e (Alg. 2 line 5)
             s++;
             q = succ[q];
         }
-        if (len >= 2) {
+        if (len >= 2) {  // r / e now hold the chain's last edge
             lc[l] = make_uint2(first, len);
-            const uint32_t lid = id_map ? id_map[sid[last]] : sid[last];
-            sc[l] = make_int4((int)s_v[last], (int)s_arr[last], (int)lid, (int)node_of[p]);
+            const uint32_t lid = id_map ? id_map[e] : e;
+            sc[l] = make_int4((int)r.x, (int)r.y, (int)lid, (int)node_of[p]);
             sc_sumw[l] = sumw;
-            sc_elapsed[l] = s_arr[last] - T[sid[p]];
+            sc_elapsed[l] = r.y - r0.w;
         }
     }
 }
@@ -272,7 +276,7 @@ static int bits_for(uint64_t x) {  // bits to represent values in [0, x]
 
 tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
                              const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
-                             cudaStream_t s) {
+                             uint32_t tmax, cudaStream_t s) {
     const uint32_t n = g->n;
     cg->n = n;
     cg->m = m;
@@ -284,21 +288,8 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
         TG_TRY_CUDA(cudaMemsetAsync(cg->chain_first, 0, 4, s));
         return TG_OK;
     }
-    // ---- 1. sort by (u, t, id)
-    uint32_t maxt = 0;
-    {
-        // max over this direction's t (mirror times differ from forward ones)
-        uint32_t *res = nullptr;
-        TG_TRY_CUDA(cudaMallocAsync((void **)&res, 5 * 4, s));
-        uint32_t init[5] = {0, 0, 0, 0, 0xFFFFFFFFu};
-        TG_TRY_CUDA(cudaMemcpyAsync(res, init, sizeof(init), cudaMemcpyHostToDevice, s));
-        TG_LAUNCH(k_validate, blocks_for(m, 4), BT, 0, s, u, v, t, dur, w, m, n, res);
-        uint32_t h[5];
-        TG_TRY_CUDA(cudaMemcpyAsync(h, res, sizeof(h), cudaMemcpyDeviceToHost, s));
-        TG_TRY_CUDA(cudaStreamSynchronize(s));
-        TG_TRY_CUDA(cudaFreeAsync(res, s));
-        maxt = h[1];
-    }
+    // ---- 1. sort by (u, t, id); tmax bounds this direction's t (known from validation)
+    const uint32_t maxt = tmax;
     const int tbits = bits_for(maxt);
     const int ubits = bits_for(n - 1);
     unsigned long long *keys = nullptr;
@@ -347,15 +338,16 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_TRY_CUDA(cudaFreeAsync(keys, s));
 
     // ---- 3./4. snap, in-degree, hubs
-    uint32_t *tn = nullptr, *s_v = nullptr, *s_arr = nullptr, *indeg = nullptr;
+    uint32_t *tn = nullptr, *indeg = nullptr;
+    uint4 *rec = nullptr;
     unsigned char *hub = nullptr;
     TG_TRY_CUDA(cudaMallocAsync((void **)&tn, m * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&s_v, m * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&s_arr, m * 4, s));
+    TG_TRY_CUDA(cudaMallocAsync((void **)&rec, m * 16, s));
+    TG_LAUNCH(k_records, blocks_for(m, 4), BT, 0, s, v, t, dur, w, m, rec);
     TG_TRY_CUDA(cudaMallocAsync((void **)&indeg, nn * 4, s));
     TG_TRY_CUDA(cudaMallocAsync((void **)&hub, nn, s));
     TG_TRY_CUDA(cudaMemsetAsync(indeg, 0, nn * 4, s));
-    TG_LAUNCH(k_snap, blocks_for(m, 4), BT, 0, s, sid, m, v, t, dur, cg->vnode_off, cg->node_t, tn, s_v, s_arr, indeg);
+    TG_LAUNCH(k_snap, blocks_for(m, 4), BT, 0, s, sid, m, rec, cg->vnode_off, cg->node_t, tn, indeg);
     TG_LAUNCH(k_hubs, blocks_for(nn, 4), BT, 0, s, indeg, cg->node_eoff, nn, hub);
     TG_TRY_CUDA(cudaFreeAsync(indeg, s));
 
@@ -397,10 +389,10 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_TRY(A.alloc((void **)&cg->sc_sumw, std::max<uint64_t>(L, 1) * 8));
     TG_TRY(A.alloc((void **)&cg->sc_elapsed, std::max<uint64_t>(L, 1) * 4));
     TG_LAUNCH(k_chain_scatter, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, cg->chain_first, chain_len, lidx, sid,
-              s_v, s_arr, tn, node_of, t, w, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
+              rec, tn, node_of, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
               cg->sc_sumw, cg->sc_elapsed, id_map, (uint32_t)std::max<int64_t>(2, g->opt_walk_min));
 
-    for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)s_v, (void *)s_arr, (void *)hub,
+    for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)rec, (void *)hub,
                     (void *)head, (void *)succ, (void *)cidx, (void *)chain_len, (void *)lidx})
         TG_TRY_CUDA(cudaFreeAsync(p, s));
     TG_TRY_CUDA(cudaStreamSynchronize(s));
@@ -409,11 +401,13 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
 
 tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {
     // reading A5: G^R maps (u, v, t, lam) to (v, u, C - (t + lam), lam), C = max(t + lam)
-    if (g->m == 0) return tg_build_direction(g, &g->mir, 0, g->d_v, g->d_u, g->d_t, g->d_dur, g->d_w, nullptr, s);
+    // mirrored departures C - (t + lam) <= C - min_t - 1
+    const uint32_t mir_tmax = g->max_arr - g->min_t;
+    if (g->m == 0) return tg_build_direction(g, &g->mir, 0, g->d_v, g->d_u, g->d_t, g->d_dur, g->d_w, nullptr, 0, s);
     uint32_t *mt = nullptr;
     TG_TRY_CUDA(cudaMallocAsync((void **)&mt, g->m * 4, s));
     TG_LAUNCH(k_mirror, blocks_for(g->m, 4), BT, 0, s, g->d_t, g->d_dur, g->m, g->max_arr, mt);
-    tg_status st = tg_build_direction(g, &g->mir, g->m, g->d_v, g->d_u, mt, g->d_dur, g->d_w, nullptr, s);
+    tg_status st = tg_build_direction(g, &g->mir, g->m, g->d_v, g->d_u, mt, g->d_dur, g->d_w, nullptr, mir_tmax, s);
     cudaFreeAsync(mt, s);
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     return st;
@@ -449,7 +443,8 @@ tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint
         if (ms)
             TG_LAUNCH(k_range_compact, blocks_for(m, 4), BT, 0, s, key, m, vb, ve, flag, uu, vv, tt, g->d_dur, g->d_w,
                       su, sv, st, sd, sw, sid);
-        tg_status r = tg_build_direction(g, dir == 0 ? fwd : mir, ms, su, sv, st, sd, sw, sid, s);
+        tg_status r = tg_build_direction(g, dir == 0 ? fwd : mir, ms, su, sv, st, sd, sw, sid,
+                                         dir == 0 ? g->max_t : g->max_arr - g->min_t, s);
         TG_TRY_CUDA(cudaStreamSynchronize(s));
         cudaFreeAsync(sub, s);
         if (r != TG_OK) return r;

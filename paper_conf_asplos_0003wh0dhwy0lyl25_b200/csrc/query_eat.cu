@@ -178,21 +178,6 @@ __device__ __forceinline__ void eat_long(const EatP &P, const RoundV &R, uint32_
     eat_walk(P, R, q, s + 1, s_end);
 }
 
-// A newly usable occurrence p (sorted-edge position) for query q.
-__device__ __forceinline__ void eat_edge(const EatP &P, const RoundV &R, uint32_t q, uint32_t p) {
-    const uint32_t s = __ldg(P.occ_slot + p);
-    const int4 sl = tg_ld_slot(P.slots + s);
-    if ((uint32_t)sl.y > P.omega) return;
-    if ((uint32_t)sl.w == TG_SINGLE) eat_relax(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
-    else eat_long(P, R, q, s, sl);
-}
-
-// Edge-major relaxation of one frontier unit (vertex v, query group g) over the
-// edge positions [pbeg, pend).  Lane k holds query g*32+k's newly usable range
-// [lo, hi) (empty: lo = hi).  Per block of 32 edges each lane loads one edge's
-// occurrence and slot once; a ballot per edge gives the queries for which that
-// edge is new; the (edge, query) pairs are compacted edge-major over the lanes,
-// so the queries of one edge read adjacent state words in one request.
 // Per-warp shared-memory staging of one 32-edge block: the (edge, query) pairs
 // as 16-bit (edge lane << 5 | query bit) entries, and the block's slots.
 struct WarpStage {

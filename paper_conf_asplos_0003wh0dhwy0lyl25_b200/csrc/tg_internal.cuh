@@ -184,7 +184,7 @@ tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t
 
 tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
                              const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
-                             cudaStream_t s);
+                             uint32_t tmax, cudaStream_t s);
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s);
 
 tg_status tg_run_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
