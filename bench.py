@@ -269,6 +269,10 @@ def run_ours(a, rank, world, local_rank):
 
     # roofline of the dominant kernel group
     peak, peak_src = peaks()
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "round1", f"relax_traffic_{a.config}.json")
+    if os.path.exists(tf) and a.mode == "replicate" and a.partitions == 1 and k == 64:
+        traffic = json.load(open(tf))  # measured with ncu on this code for this workload
     roof = None
     if kprof:
         relax_names = [x for x in kprof if x.startswith(("k_eat_activate", "k_eat_big", "k_eat_chain"))]
@@ -292,7 +296,9 @@ def run_ours(a, rank, world, local_rank):
             "peak": peak,
             "unit": "GB/s",
             "frac": (relax_bytes / (relax_ms / 1e3) / 1e9 / peak) if relax_ms else None,
-            "traffic": None,
+            "traffic": traffic["bytes_per_step"] if traffic else None,
+            "traffic_unit": "DRAM bytes per step (relax kernels, ncu)",
+            "traffic_source": (traffic["source"] + " -- " + os.path.relpath(tf, ROOT)) if traffic else None,
             "peak_source": peak_src,
             "algorithmic_bytes_per_step": relax_bytes / a.steps,
             "algorithmic_bytes_formula": "20 B x W_union + 8 B x sum_q W_q (SURVEY 8(d), batched source lanes)",
