@@ -81,6 +81,21 @@ static void cache_release_all(int dev) {
     }
 }
 
+cudaError_t tg_malloc_async(void **p, size_t bytes, cudaStream_t s) {
+    cudaError_t e = cudaMallocAsync(p, bytes, s);
+    if (e == cudaErrorMemoryAllocation) {
+        cudaGetLastError();
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaStreamSynchronize(s);
+        cache_release_all(dev);
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
+        e = cudaMallocAsync(p, bytes, s);
+    }
+    return e;
+}
+
 tg_status DevArena::alloc(void **p, size_t bytes) {
     *p = nullptr;
     bytes = round_bytes(bytes ? bytes : 16);

@@ -245,7 +245,7 @@ __global__ void k_mirror(const uint32_t *__restrict__ t, const uint32_t *__restr
 
 tg_status tg_validate_edges(tg_graph *g, cudaStream_t s) {
     uint32_t *res = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&res, 5 * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&res, 5 * 4, s));
     uint32_t init[5] = {0, 0, 0, 0, 0xFFFFFFFFu};
     TG_TRY_CUDA(cudaMemcpyAsync(res, init, sizeof(init), cudaMemcpyHostToDevice, s));
     if (g->m) TG_LAUNCH(k_validate, blocks_for(g->m, 4), BT, 0, s, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, g->m, g->n, res);
@@ -294,8 +294,8 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     const int ubits = bits_for(n - 1);
     unsigned long long *keys = nullptr;
     uint32_t *sid = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&keys, m * 8, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&sid, m * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&keys, m * 8, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&sid, m * 4, s));
     TG_LAUNCH(k_make_keys, blocks_for(m, 4), BT, 0, s, u, t, m, tbits, keys, sid);
     unsigned long long *sk;
     uint32_t *sv;
@@ -305,7 +305,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     uint32_t *node_of = nullptr, *d_cnt = nullptr;
     TG_TRY(A.alloc((void **)&cg->occ_node, m * 4));
     node_of = cg->occ_node;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&d_cnt, 16, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&d_cnt, 16, s));
     TG_LAUNCH(k_node_flags, blocks_for(m, 4), BT, 0, s, keys, m, node_of);
     TG_TRY(tg_exclusive_scan_u32(node_of, node_of, m, d_cnt, s, nullptr));
     uint32_t h_cnt = 0;
@@ -341,11 +341,11 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     uint32_t *tn = nullptr, *indeg = nullptr;
     uint4 *rec = nullptr;
     unsigned char *hub = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&tn, m * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&rec, m * 16, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&tn, m * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&rec, m * 16, s));
     TG_LAUNCH(k_records, blocks_for(m, 4), BT, 0, s, v, t, dur, w, m, rec);
-    TG_TRY_CUDA(cudaMallocAsync((void **)&indeg, nn * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&hub, nn, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&indeg, nn * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&hub, nn, s));
     TG_TRY_CUDA(cudaMemsetAsync(indeg, 0, nn * 4, s));
     TG_LAUNCH(k_snap, blocks_for(m, 4), BT, 0, s, sid, m, rec, cg->vnode_off, cg->node_t, tn, indeg);
     TG_LAUNCH(k_hubs, blocks_for(nn, 4), BT, 0, s, indeg, cg->node_eoff, nn, hub);
@@ -353,9 +353,9 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
 
     // ---- 5. heads / successors; chain ids in (head u, head t, first id) order
     uint32_t *head = nullptr, *succ = nullptr, *cidx = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&head, m * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&succ, m * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&cidx, m * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&head, m * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&succ, m * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&cidx, m * 4, s));
     TG_LAUNCH(k_succ, blocks_for(m, 4), BT, 0, s, node_of, tn, m, hub, cg->node_eoff, head, succ);
     TG_TRY(tg_exclusive_scan_u32(head, cidx, m, d_cnt, s, nullptr));
     uint32_t nch = 0;
@@ -365,8 +365,8 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
 
     // ---- 6. chain lengths, slot offsets, long-chain numbering
     uint32_t *chain_len = nullptr, *lidx = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&chain_len, (uint64_t)nch * 4 + 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&lidx, (uint64_t)nch * 4 + 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&chain_len, (uint64_t)nch * 4 + 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&lidx, (uint64_t)nch * 4 + 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(d_cnt + 2, 0, 4, s));
     TG_LAUNCH(k_chain_len, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, chain_len, d_cnt + 2);
     TG_TRY(A.alloc((void **)&cg->chain_first, ((uint64_t)nch + 1) * 4));
@@ -405,7 +405,7 @@ tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {
     const uint32_t mir_tmax = g->max_arr - g->min_t;
     if (g->m == 0) return tg_build_direction(g, &g->mir, 0, g->d_v, g->d_u, g->d_t, g->d_dur, g->d_w, nullptr, 0, s);
     uint32_t *mt = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&mt, g->m * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&mt, g->m * 4, s));
     TG_LAUNCH(k_mirror, blocks_for(g->m, 4), BT, 0, s, g->d_t, g->d_dur, g->m, g->max_arr, mt);
     tg_status st = tg_build_direction(g, &g->mir, g->m, g->d_v, g->d_u, mt, g->d_dur, g->d_w, nullptr, mir_tmax, s);
     cudaFreeAsync(mt, s);
@@ -419,9 +419,9 @@ tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s) {
     const uint64_t m = g->m;
     uint32_t *mt = nullptr, *flag = nullptr, *cnt = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&mt, std::max<uint64_t>(m, 1) * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&flag, std::max<uint64_t>(m, 1) * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&cnt, 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&mt, std::max<uint64_t>(m, 1) * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&flag, std::max<uint64_t>(m, 1) * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&cnt, 4, s));
     if (m) TG_LAUNCH(k_mirror, blocks_for(m, 4), BT, 0, s, g->d_t, g->d_dur, m, g->max_arr, mt);
     for (int dir = 0; dir < 2; dir++) {
         // forward: (u, v, t); mirror: (v, u, C - t - dur)
@@ -437,7 +437,7 @@ tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint
             TG_TRY_CUDA(cudaStreamSynchronize(s));
         }
         uint32_t *sub = nullptr;  // 6 arrays of ms
-        TG_TRY_CUDA(cudaMallocAsync((void **)&sub, std::max<uint64_t>(ms, 1) * 4 * 6, s));
+        TG_TRY_CUDA(tg_malloc_async((void **)&sub, std::max<uint64_t>(ms, 1) * 4 * 6, s));
         uint32_t *su = sub, *sv = sub + ms, *st = sub + 2 * (uint64_t)ms, *sd = sub + 3 * (uint64_t)ms,
                  *sw = sub + 4 * (uint64_t)ms, *sid = sub + 5 * (uint64_t)ms;
         if (ms)

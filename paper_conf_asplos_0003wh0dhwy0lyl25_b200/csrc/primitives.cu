@@ -86,7 +86,7 @@ tg_status tg_exclusive_scan_u32(const uint32_t *in, uint32_t *out, uint64_t coun
         return TG_OK;
     }
     uint32_t *sums = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&sums, tiles * sizeof(uint32_t), s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&sums, tiles * sizeof(uint32_t), s));
     TG_LAUNCH(k_scan_reduce, (unsigned)tiles, SCAN_THREADS, 0, s, in, count, sums);
     tg_status st = tg_exclusive_scan_u32(sums, sums, tiles, nullptr, s, nullptr);
     if (st != TG_OK) { cudaFreeAsync(sums, s); return st; }
@@ -225,9 +225,9 @@ tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t
     }
     unsigned long long *k2 = nullptr;
     uint32_t *v2 = nullptr, *counts = nullptr;
-    TG_TRY_CUDA(cudaMallocAsync((void **)&k2, m * 8, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&v2, m * 4, s));
-    TG_TRY_CUDA(cudaMallocAsync((void **)&counts, ntiles * 256 * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&k2, m * 8, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&v2, m * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&counts, ntiles * 256 * 4, s));
     TG_TRY_CUDA(cudaFuncSetAttribute(k_radix_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)RS_SMEM));
     unsigned long long *ka = keys, *kb = k2;
     uint32_t *va = vals, *vb = v2;

@@ -305,15 +305,20 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
                 }
                 rec = __shfl_sync(0xffffffffu, rec, 0);
                 k0 = __shfl_sync(0xffffffffu, k0, 0);
-                if (rec < P.reccap && k0 + nch <= P.bigcap) {
-                    P.recs[(size_t)rec * 32 + lane] = make_uint2(lo, hi);
-                    for (uint32_t c = lane; c < nch; c += 32) {
-                        const uint32_t b0 = ulo + c * CHUNK;
-                        P.bigq[k0 + c] = make_uint4(rec, b0, min(uhi, b0 + CHUNK), g);
-                    }
-                    continue;
+                // queue entries below the capacity are always written (empty ones if the
+                // record did not fit); whatever is not queued is relaxed right here
+                const bool rec_ok = rec < P.reccap;
+                if (rec_ok) P.recs[(size_t)rec * 32 + lane] = make_uint2(lo, hi);
+                uint32_t queued = 0;
+                if (k0 < P.bigcap) queued = min(nch, (uint32_t)(P.bigcap - k0));
+                for (uint32_t c = lane; c < queued; c += 32) {
+                    const uint32_t b0 = ulo + c * CHUNK;
+                    P.bigq[k0 + c] = rec_ok ? make_uint4(rec, b0, min(uhi, b0 + CHUNK), g) : make_uint4(0, 0, 0, g);
                 }
-                // capacity exceeded (not expected: both are bounds): relax in place
+                if (rec_ok) {
+                    if (queued == nch) continue;
+                    ulo = ulo + queued * CHUNK;  // the rest, in place
+                }
             }
             unit_range(P, R, g, lo, hi, ulo, uhi, ws);
         }
@@ -508,13 +513,15 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
         TG_TRY(A.alloc((void **)&Q.fr[0], Q.fcap * 8));
         TG_TRY(A.alloc((void **)&Q.fr[1], Q.fcap * 8));
     }
-    // big-union chunks: per unit at most deg/CHUNK + 1; records: one per unit with a long union
-    Q.bigcap = std::max<uint64_t>(S * (m / CHUNK + std::max<uint64_t>(n, nnodes) / BIG_T + 2) + 1024,
-                                  (uint64_t)Q.vwords * (m / CHUNK + n / BIG_T + 2) + 1024);
+    // Work queues: chunks of long unions (+ their 32-range records) and chain walks.
+    // Every producer falls back to doing the work in place when a queue is full, so
+    // the capacities only need to cover typical rounds (capped at ~1 GiB each).
+    Q.bigcap = std::min<uint64_t>(std::max<uint64_t>(S, 32) * (m / CHUNK + std::max<uint64_t>(n, nnodes) / BIG_T + 2) + 1024,
+                                  1ull << 26);
     TG_TRY(A.alloc((void **)&Q.bigq, Q.bigcap * 16));
-    Q.reccap = (uint64_t)Q.vwords * (m / BIG_T + 2) + 1024;
+    Q.reccap = std::min<uint64_t>((uint64_t)Q.vwords * (m / BIG_T + 2) + 1024, 1ull << 22);
     TG_TRY(A.alloc((void **)&Q.recs, Q.reccap * 32 * 8));
-    Q.chcap = S * (m / (INLINE_WALK + 1)) + (1u << 16);
+    Q.chcap = std::min<uint64_t>(S * (m / 2) + (1u << 16), 1ull << 26);
     TG_TRY(A.alloc((void **)&Q.chq, Q.chcap * 16));
     TG_TRY(A.alloc((void **)&Q.ctr, 64));
     TG_TRY_CUDA(cudaMemset(Q.ctr, 0, 64));

@@ -174,6 +174,10 @@ struct tg_graph {
     uint32_t last_relax_len = 0;
 };
 
+// Stream-ordered temporary allocation; on failure the block cache is returned to
+// the driver, the pool trimmed, and the allocation retried once.
+cudaError_t tg_malloc_async(void **p, size_t bytes, cudaStream_t s);
+
 // ----------------------------------------------------------------------------- primitives
 // Exclusive prefix sum of in[0..count) into out (may alias), total -> *d_total (device, may be null).
 tg_status tg_exclusive_scan_u32(const uint32_t *in, uint32_t *out, uint64_t count, uint32_t *d_total,

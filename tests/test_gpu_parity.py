@@ -215,6 +215,26 @@ def test_c2_full_sampled_rows(tg):
             np.testing.assert_array_equal(tg.as_u32(lpred[r]), S)
 
 
+@pytest.mark.slow
+def test_c3_full_sampled_rows(tg):
+    """configs[2] at full size: wiki-talk-shaped graph, all four problems, sampled rows."""
+    import torch
+    ge = tgsynth.make_graph("C3", device="cuda")
+    g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, ge.w, device=0).build()
+    srcs = tgsynth.config_sources("C3", ge)
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d, w)
+    for win in tgsynth.CONFIGS["C3"]["windows"]:
+        res = {p: g.query(p, srcs, win) for p in ("eat", "ld", "fp", "sp")}
+        torch.cuda.synchronize()
+        for r in (0, 7):
+            x = srcs[r]
+            np.testing.assert_array_equal(tg.as_u32(res["eat"][r]), oracle.eat(og, x, *win)[0])
+            np.testing.assert_array_equal(tg.as_u32(res["ld"][r]), oracle.ld(og, x, *win)[0])
+            np.testing.assert_array_equal(tg.as_u32(res["fp"][r]), oracle.fp(og, x, *win))
+            np.testing.assert_array_equal(tg.as_u32(res["sp"][r]), oracle.sp(og, x, *win))
+
+
 # --------------------------------------------------------------------------- edge cases
 def test_edge_cases(tg):
     # no edges
