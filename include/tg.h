@@ -209,6 +209,8 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *   "walk_min"   chains with at least this many edges are walked by the chain engine
  *                (default 6, min 2, before build); shorter chains are relaxed edge by
  *                edge through their own occurrences (P:L322's RemoveChain, generalised)
+ *   "relabel"    1 = internal vertex order by descending in-degree (before build; default 0:
+ *                no gain measured on R-MAT); invisible to callers
  *   "partitions" logical vertex-range partitions on this GPU (1..16, before build):
  *                runs the multi-GPU mode-1 algorithm inside one process (tests) */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);

@@ -308,7 +308,9 @@ tg_status tg_build_chains(tg_graph *g) {
         for (int p = 0; p < P; p++)
             TG_TRY(tg_build_partition(g, &g->pf[p], &g->pm[p], g->part_vb[p], g->part_vb[p + 1], 0));
     } else {
-        TG_TRY(tg_build_direction(g, &g->fwd, g->m, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, nullptr, g->max_t, 0));
+        if (g->opt_relabel) TG_TRY(tg_relabel(g, 0));
+        const uint32_t *U = g->relabeled ? g->d_ru : g->d_u, *V = g->relabeled ? g->d_rv : g->d_v;
+        TG_TRY(tg_build_direction(g, &g->fwd, g->m, U, V, g->d_t, g->d_dur, g->d_w, nullptr, g->max_t, 0));
         if (g->opt_mirror) {
             TG_TRY(tg_build_mirror(g, 0));
             g->mirror_built = true;
@@ -406,8 +408,37 @@ tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off,
     std::vector<int4> slots(m);
     TG_TRY_CUDA(cudaMemcpy(first.data(), c.chain_first, (nc + 1) * 4, cudaMemcpyDeviceToHost));
     if (m) TG_TRY_CUDA(cudaMemcpy(slots.data(), c.slots, m * 16, cudaMemcpyDeviceToHost));
-    for (uint64_t i = 0; i <= nc; i++) chain_off[i] = first[i];
-    for (uint64_t s = 0; s < m; s++) chain_edges[s] = (uint32_t)slots[s].z;
+    // chain order: when the engine relabelled vertices its chains are ordered by the
+    // internal head vertex; export them in the paper's (original head u, t, first id) order
+    std::vector<uint64_t> order(nc);
+    for (uint64_t i = 0; i < nc; i++) order[i] = i;
+    std::vector<uint32_t> hu, ht, iperm;
+    if (g->relabeled && nc) {
+        hu.resize(m);
+        ht.resize(m);
+        iperm.resize(g->n);
+        TG_TRY_CUDA(cudaMemcpy(hu.data(), mirrored ? g->d_v : g->d_u, m * 4, cudaMemcpyDeviceToHost));
+        TG_TRY_CUDA(cudaMemcpy(iperm.data(), g->iperm, (size_t)g->n * 4, cudaMemcpyDeviceToHost));
+        std::vector<uint32_t> dur(m);
+        TG_TRY_CUDA(cudaMemcpy(dur.data(), g->d_dur, m * 4, cudaMemcpyDeviceToHost));
+        for (uint64_t i = 0; i < m; i++) ht[i] = (uint32_t)slots[i].y - dur[(uint32_t)slots[i].z];  // per slot
+        std::sort(order.begin(), order.end(), [&](uint64_t a, uint64_t b) {
+            const int4 &sa = slots[first[a]], &sb = slots[first[b]];
+            const uint32_t ua = hu[(uint32_t)sa.z], ub = hu[(uint32_t)sb.z];
+            if (ua != ub) return ua < ub;
+            const uint32_t ta = ht[first[a]], tb = ht[first[b]];
+            if (ta != tb) return ta < tb;
+            return (uint32_t)sa.z < (uint32_t)sb.z;
+        });
+    }
+    {
+        uint64_t pos = 0;
+        for (uint64_t i = 0; i < nc; i++) {
+            chain_off[i] = pos;
+            for (uint32_t sl = first[order[i]]; sl < first[order[i] + 1]; sl++) chain_edges[pos++] = (uint32_t)slots[sl].z;
+        }
+        chain_off[nc] = pos;
+    }
     if (sc_tail_v || sc_arr || sc_sum_w || sc_elapsed) {
         std::vector<int4> sc(c.nlong);
         std::vector<unsigned long long> sumw(c.nlong);
@@ -424,21 +455,27 @@ tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off,
             TG_TRY_CUDA(cudaMemcpy(dur.data(), g->d_dur, m * 4, cudaMemcpyDeviceToHost));
             for (uint64_t s = 0; s < m; s++) t[s] = (uint32_t)slots[s].y - dur[(uint32_t)slots[s].z];
         }
-        uint32_t l = 0;  // long-chain index: chains with >= 2 edges numbered in chain order
-        for (uint64_t ch = 0; ch < nc; ch++) {
+        // long-chain index: chains with >= 2 edges numbered in internal chain order
+        std::vector<uint32_t> lidx(nc, 0);
+        for (uint64_t ch = 0, l = 0; ch < nc; ch++)
+            if (first[ch + 1] - first[ch] >= 2) lidx[ch] = (uint32_t)l++;
+        auto vout = [&](uint32_t v) { return g->relabeled ? iperm[v] : v; };
+        for (uint64_t oi = 0; oi < nc; oi++) {
+            const uint64_t ch = order[oi];
             uint32_t b = first[ch], e = first[ch + 1];
             int4 sl = slots[b];
+            const uint64_t ochn = oi;  // output position
             if (e - b >= 2) {
-                if (sc_tail_v) sc_tail_v[ch] = (uint32_t)sc[l].x;
-                if (sc_arr) sc_arr[ch] = (uint32_t)sc[l].y;
-                if (sc_sum_w) sc_sum_w[ch] = sumw[l];
-                if (sc_elapsed) sc_elapsed[ch] = el[l];
-                l++;
+                const uint32_t l = lidx[ch];
+                if (sc_tail_v) sc_tail_v[ochn] = vout((uint32_t)sc[l].x);
+                if (sc_arr) sc_arr[ochn] = (uint32_t)sc[l].y;
+                if (sc_sum_w) sc_sum_w[ochn] = sumw[l];
+                if (sc_elapsed) sc_elapsed[ochn] = el[l];
             } else {  // Alg. 2 line 8: a one-edge chain is its own shortcut
-                if (sc_tail_v) sc_tail_v[ch] = (uint32_t)sl.x;
-                if (sc_arr) sc_arr[ch] = (uint32_t)sl.y;
-                if (sc_sum_w) sc_sum_w[ch] = slot_w[b];
-                if (sc_elapsed) sc_elapsed[ch] = (uint32_t)sl.y - t[b];
+                if (sc_tail_v) sc_tail_v[ochn] = vout((uint32_t)sl.x);
+                if (sc_arr) sc_arr[ochn] = (uint32_t)sl.y;
+                if (sc_sum_w) sc_sum_w[ochn] = slot_w[b];
+                if (sc_elapsed) sc_elapsed[ochn] = (uint32_t)sl.y - t[b];
             }
         }
     }
@@ -461,6 +498,10 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     else if (k == "shortcuts") g->opt_shortcuts = value;
     else if (k == "round_group") g->opt_round_group = value;
     else if (k == "mirror") g->opt_mirror = value ? 1 : 0;
+    else if (k == "relabel") {
+        if (g->built) { tg_set_error("set relabel before tg_build_chains"); return TG_ERR_STATE; }
+        g->opt_relabel = value ? 1 : 0;
+    }
     else if (k == "exp") g->opt_exp = value;
     else if (k == "walk_min") {
         if (g->built) { tg_set_error("set walk_min before tg_build_chains"); return TG_ERR_STATE; }

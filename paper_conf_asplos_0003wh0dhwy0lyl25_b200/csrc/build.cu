@@ -235,6 +235,40 @@ __global__ void k_range_compact(const uint32_t *__restrict__ key, uint64_t m, ui
     }
 }
 
+// ---- internal vertex order: descending in-degree (hot relaxation targets share L2 lines)
+__global__ void k_indeg_hist(const uint32_t *__restrict__ v, uint64_t m, uint32_t *__restrict__ cnt) {
+    GRID_STRIDE(i, m) atomicAdd(&cnt[v[i]], 1u);
+}
+
+__global__ void k_degree_keys(const uint32_t *__restrict__ cnt, uint32_t n, unsigned long long *__restrict__ keys,
+                              uint32_t *__restrict__ ids) {
+    GRID_STRIDE(i, n) {
+        keys[i] = 0xFFFFFFFFull - cnt[i];
+        ids[i] = (uint32_t)i;
+    }
+}
+
+__global__ void k_perm_from_order(const uint32_t *__restrict__ order, uint32_t n, uint32_t *__restrict__ perm,
+                                  uint32_t *__restrict__ iperm) {
+    GRID_STRIDE(i, n) {
+        perm[order[i]] = (uint32_t)i;
+        iperm[i] = order[i];
+    }
+}
+
+__global__ void k_apply_perm(const uint32_t *__restrict__ u, const uint32_t *__restrict__ v, uint64_t m,
+                             const uint32_t *__restrict__ perm, uint32_t *__restrict__ ru, uint32_t *__restrict__ rv) {
+    GRID_STRIDE(i, m) {
+        ru[i] = perm[u[i]];
+        rv[i] = perm[v[i]];
+    }
+}
+
+__global__ void k_map_sources(const uint32_t *__restrict__ src, uint32_t k, const uint32_t *__restrict__ perm,
+                              uint32_t *__restrict__ out) {
+    GRID_STRIDE(i, k) out[i] = perm ? perm[src[i]] : src[i];
+}
+
 __global__ void k_mirror(const uint32_t *__restrict__ t, const uint32_t *__restrict__ dur, uint64_t m, uint32_t C,
                          uint32_t *__restrict__ mt) {
     // reading A5: e = (u,v,t,lam) -> (v,u, C - (t + lam), lam)
@@ -399,15 +433,52 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     return TG_OK;
 }
 
+tg_status tg_relabel(tg_graph *g, cudaStream_t s) {
+    const uint64_t m = g->m;
+    const uint32_t n = g->n;
+    DevArena &A = g->arena;
+    TG_TRY(A.alloc((void **)&g->perm, (uint64_t)n * 4));
+    TG_TRY(A.alloc((void **)&g->iperm, (uint64_t)n * 4));
+    TG_TRY(A.alloc((void **)&g->d_ru, std::max<uint64_t>(m, 1) * 4));
+    TG_TRY(A.alloc((void **)&g->d_rv, std::max<uint64_t>(m, 1) * 4));
+    uint32_t *cnt = nullptr, *ids = nullptr;
+    unsigned long long *keys = nullptr;
+    TG_TRY_CUDA(tg_malloc_async((void **)&cnt, (uint64_t)n * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&ids, (uint64_t)n * 4, s));
+    TG_TRY_CUDA(tg_malloc_async((void **)&keys, (uint64_t)n * 8, s));
+    TG_TRY_CUDA(cudaMemsetAsync(cnt, 0, (uint64_t)n * 4, s));
+    if (m) TG_LAUNCH(k_indeg_hist, blocks_for(m, 4), BT, 0, s, g->d_v, m, cnt);
+    TG_LAUNCH(k_degree_keys, blocks_for(n, 4), BT, 0, s, cnt, n, keys, ids);
+    unsigned long long *sk;
+    uint32_t *sv;
+    TG_TRY(tg_radix_sort_pairs(keys, ids, n, 32, &sk, &sv, s));  // stable: ties keep vertex order
+    TG_LAUNCH(k_perm_from_order, blocks_for(n, 4), BT, 0, s, ids, n, g->perm, g->iperm);
+    if (m) TG_LAUNCH(k_apply_perm, blocks_for(m, 4), BT, 0, s, g->d_u, g->d_v, m, g->perm, g->d_ru, g->d_rv);
+    TG_TRY_CUDA(cudaFreeAsync(cnt, s));
+    TG_TRY_CUDA(cudaFreeAsync(ids, s));
+    TG_TRY_CUDA(cudaFreeAsync(keys, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    g->relabeled = true;
+    return TG_OK;
+}
+
+tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cudaStream_t s) {
+    QueryScratch &Q = g->qs;
+    TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources, (uint64_t)k * 4, cudaMemcpyHostToDevice, s));
+    TG_LAUNCH(k_map_sources, 1, 64, 0, s, Q.srcs, k, g->relabeled ? g->perm : nullptr, Q.srcs_int);
+    return TG_OK;
+}
+
 tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {
+    const uint32_t *U = g->relabeled ? g->d_ru : g->d_u, *V = g->relabeled ? g->d_rv : g->d_v;
     // reading A5: G^R maps (u, v, t, lam) to (v, u, C - (t + lam), lam), C = max(t + lam)
     // mirrored departures C - (t + lam) <= C - min_t - 1
     const uint32_t mir_tmax = g->max_arr - g->min_t;
-    if (g->m == 0) return tg_build_direction(g, &g->mir, 0, g->d_v, g->d_u, g->d_t, g->d_dur, g->d_w, nullptr, 0, s);
+    if (g->m == 0) return tg_build_direction(g, &g->mir, 0, V, U, g->d_t, g->d_dur, g->d_w, nullptr, 0, s);
     uint32_t *mt = nullptr;
     TG_TRY_CUDA(tg_malloc_async((void **)&mt, g->m * 4, s));
     TG_LAUNCH(k_mirror, blocks_for(g->m, 4), BT, 0, s, g->d_t, g->d_dur, g->m, g->max_arr, mt);
-    tg_status st = tg_build_direction(g, &g->mir, g->m, g->d_v, g->d_u, mt, g->d_dur, g->d_w, nullptr, mir_tmax, s);
+    tg_status st = tg_build_direction(g, &g->mir, g->m, V, U, mt, g->d_dur, g->d_w, nullptr, mir_tmax, s);
     cudaFreeAsync(mt, s);
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     return st;

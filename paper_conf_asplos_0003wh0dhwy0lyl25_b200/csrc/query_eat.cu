@@ -399,7 +399,7 @@ __global__ void k_eat_init(unsigned long long *st, uint32_t n, uint32_t G, const
 __global__ void __launch_bounds__(256) k_eat_extract(const unsigned long long *__restrict__ st, uint32_t n, uint32_t S,
                                                      const uint32_t *__restrict__ srcs, int mode, uint32_t C,
                                                      uint32_t omega, uint32_t *__restrict__ out,
-                                                     uint32_t *__restrict__ pred) {
+                                                     uint32_t *__restrict__ pred, const uint32_t *__restrict__ perm) {
     __shared__ unsigned long long tile[32 * 65];
     const uint32_t nt = (n + 31) / 32;
     for (uint32_t tb = blockIdx.x; tb < nt; tb += gridDim.x) {
@@ -410,7 +410,8 @@ __global__ void __launch_bounds__(256) k_eat_extract(const unsigned long long *_
             for (uint32_t i = threadIdx.x; i < 32 * qs; i += blockDim.x) {
                 const uint32_t dv = i / qs, dq = i - dv * qs;
                 const uint32_t v = v0 + dv;
-                tile[dv * 65 + dq] = (v < n) ? st[(size_t)v * S + q0 + dq] : ~0ull;
+                // rows are in the engine's vertex order (perm: caller id -> internal id)
+                tile[dv * 65 + dq] = (v < n) ? st[(size_t)(perm ? perm[v] : v) * S + q0 + dq] : ~0ull;
             }
             __syncthreads();
             for (uint32_t i = threadIdx.x; i < 32 * qs; i += blockDim.x) {
@@ -533,6 +534,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     }
     TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
     TG_TRY(A.alloc((void **)&Q.srcs, S * 4));
+    TG_TRY(A.alloc((void **)&Q.srcs_int, S * 4));
     TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8 + 8));  // [S] per query + [S] = distinct slots
     TG_TRY(A.alloc((void **)&Q.touched, ((m + 31) / 32 + TG_MAXP + 1) * 4));
     if (nodes_state) {
@@ -579,7 +581,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
     }
     const bool work = any_work && g->m > 0 && alpha < omega;
-    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs, S, alpha, Q.fb[1], Q.ctl,
+    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
     uint32_t rounds = 0;
     if (work) {
@@ -646,7 +648,7 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     const int mode = ld ? 1 : (p == TG_REACH ? 2 : 0);
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
-        TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources + b0, Sb * 4, cudaMemcpyHostToDevice, s));
+        TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
         uint32_t rounds = 0;
         TG_TRY(eat_rounds(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
         g->last.rounds = std::max(g->last.rounds, rounds);
@@ -654,7 +656,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
         uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
         const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
-        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr);
+        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
+                  g->relabeled ? g->perm : (const uint32_t *)nullptr);
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (g->opt_stats) {
@@ -711,7 +714,7 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
         const uint32_t G = (Sb + 31) / 32;
-        TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources + b0, Sb * 4, cudaMemcpyHostToDevice, s));
+        TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, Sb * n * 8, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, Sb * n * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.lat, 0xFF, Sb * n * 4, s));
@@ -723,7 +726,7 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
             TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8 + 8, s));
             TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
         }
-        TG_LAUNCH(k_eat_init, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs, Sb, alpha, Q.fb[1], Q.ctl, 0);
+        TG_LAUNCH(k_eat_init, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl, 0);
         const bool work = any_work && g->m > 0 && alpha < omega;
         uint32_t rounds = 0;
         if (work) {
@@ -787,7 +790,8 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
         uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
         const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
-        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr);
+        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
+                  (const uint32_t *)nullptr);
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (g->opt_stats) {

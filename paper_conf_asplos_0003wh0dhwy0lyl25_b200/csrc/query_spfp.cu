@@ -279,12 +279,12 @@ __global__ void k_spfp_init(SpP P, const uint32_t *srcs, uint32_t S) {
 }
 
 __global__ void k_spfp_extract(const uint32_t *__restrict__ vout, uint32_t n, const uint32_t *__restrict__ srcs,
-                               uint32_t *__restrict__ out) {
+                               uint32_t *__restrict__ out, const uint32_t *__restrict__ perm) {
     const uint32_t q = blockIdx.y;
-    const uint32_t src = srcs[q];
+    const uint32_t src = srcs[q];  // caller's vertex ids
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
         const size_t i = (size_t)q * n + v;
-        out[i] = (v == src) ? 0u : vout[i];
+        out[i] = (v == src) ? 0u : vout[(size_t)q * n + (perm ? perm[v] : v)];
     }
 }
 
@@ -310,7 +310,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl);
     {
         dim3 grid(4, Sb);
-        TG_LAUNCH(k_spfp_init<FP>, grid, 256, 0, s, P, Q.srcs, Sb);
+        TG_LAUNCH(k_spfp_init<FP>, grid, 256, 0, s, P, Q.srcs_int, Sb);
     }
     TG_LAUNCH(k_spfp_ctl_start, 1, 1, 0, s, Q.ctl);
     const uint32_t grid = tg_grid_persistent(8);
@@ -343,7 +343,7 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
     const uint64_t launches0 = g_tg_launches;
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
-        TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources + b0, Sb * 4, cudaMemcpyHostToDevice, s));
+        TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
         uint32_t rounds = 0;
         if (fp) TG_TRY((spfp_rounds<true>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
         else TG_TRY((spfp_rounds<false>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
@@ -351,7 +351,7 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
         g->last.sub_batches++;
         uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
         dim3 grid((unsigned)std::min<uint64_t>((n + 255) / 256, 1024), Sb);
-        TG_LAUNCH(k_spfp_extract, grid, 256, 0, s, Q.vout, g->n, Q.srcs, o);
+        TG_LAUNCH(k_spfp_extract, grid, 256, 0, s, Q.vout, g->n, Q.srcs, o, g->relabeled ? g->perm : (const uint32_t *)nullptr);
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));

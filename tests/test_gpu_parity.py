@@ -89,6 +89,23 @@ def test_tiny_random_all_problems(tg, seed):
             _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
 
 
+def test_relabel_option(tg):
+    """Internal vertex relabelling (descending in-degree) is invisible to callers:
+    values, preds and exported chains equal the oracle."""
+    n, u, v, t, lam, w = tgsynth.tiny_random(4242, n_max=50, m_max=700, t_max=30, lam_max=4)
+    g = _gpu_graph(tg, n, u, v, t, lam, w, relabel=1, stats=1)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    for p in ("eat", "ld", "reach", "sp", "fp"):
+        _check_rows(tg, g, og, p, list(range(min(n, 20))), (2, 10**6), stats=(p == "eat"))
+    off, ce = oracle.chains(og)
+    sc = oracle.shortcuts(og, off, ce)
+    ch = g.export_chains()
+    np.testing.assert_array_equal(ch["chain_off"], off)
+    np.testing.assert_array_equal(ch["chain_edges"], ce)
+    for k in ("tail_v", "arr", "elapsed", "sum_w"):
+        np.testing.assert_array_equal(ch[k], sc[k], err_msg=k)
+
+
 @pytest.mark.parametrize("walk_min", [2, 6])
 def test_walk_threshold(tg, walk_min):
     """Every chain walked (walk_min = 2) and the default threshold give identical,

@@ -23,12 +23,14 @@ ap.add_argument("--sub-batch", type=int, default=0)
 ap.add_argument("--shortcuts", type=int, default=1)
 ap.add_argument("--exp", type=int, default=0)
 ap.add_argument("--walk-min", type=int, default=0)
+ap.add_argument("--relabel", type=int, default=1)
 a = ap.parse_args()
 
 ge = tgsynth.make_graph(a.config, device="cuda")
 cfg = tgsynth.CONFIGS[a.config]
 w = ge.w if cfg["kind"] == "wikitalk" else None
 g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, w, device=0)
+g.set_option("relabel", a.relabel)
 if a.walk_min:
     g.set_option("walk_min", a.walk_min)
 g.build()
