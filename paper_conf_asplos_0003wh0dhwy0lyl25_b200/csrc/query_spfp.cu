@@ -35,7 +35,7 @@ namespace {
 constexpr int QT = 256;
 constexpr uint32_t BIG_T = 256;
 constexpr uint32_t CHUNK = 1024;
-constexpr uint32_t WAIT_MAX = 2048;  // wait-propagation steps per item per round
+constexpr uint32_t WAIT_INLINE = 32;  // wait-propagation steps a lane does inline; longer walks go to k_spfp_wait
 
 struct SpP {
     const uint32_t *vnode_off, *node_t, *node_u, *node_eoff, *occ_slot, *occ_node;
@@ -53,6 +53,8 @@ struct SpP {
     unsigned long long *fr0, *fr1;
     uint4 *bigq;
     uint64_t bigcap;
+    uint4 *waitq;  // long wait-propagation walks {q, next node, vertex end, value}
+    uint64_t waitcap;
 };
 
 struct RoundV {
@@ -60,7 +62,7 @@ struct RoundV {
     const unsigned long long *fin;
     uint32_t fin_n;
     unsigned long long *fout;
-    uint32_t *fout_cnt, *big_cnt;
+    uint32_t *fout_cnt, *big_cnt, *wait_cnt;
 };
 
 __device__ __forceinline__ RoundV round_view(const SpP &P) {
@@ -72,6 +74,7 @@ __device__ __forceinline__ RoundV round_view(const SpP &P) {
     R.fin_n = *(volatile uint32_t *)&P.ctl->cnt[r & 3][0];
     R.fout_cnt = &P.ctl->cnt[(r + 1) & 3][0];
     R.big_cnt = &P.ctl->cnt[r & 3][1];
+    R.wait_cnt = &P.ctl->cnt[r & 3][2];
     return R;
 }
 
@@ -187,13 +190,21 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             const uint32_t d = __ldcg(dn + j);
             const uint32_t u = __ldg(P.node_u + j);
             const uint32_t vend = __ldg(P.vnode_off + u + 1);
-            // wait edges: later departure nodes of u inherit d (reading A11)
+            // wait edges: later departure nodes of u inherit d (reading A11);
+            // the first WAIT_INLINE nodes here, the rest by a warp in k_spfp_wait
             uint32_t jend = j + 1;
-            for (uint32_t steps = 0; jend < vend; jend++, steps++) {
+            bool more = false;
+            for (uint32_t steps = 0; jend < vend;) {
                 if (__ldg(P.node_t + jend) >= P.omega) break;  // no valid out-edge departs at >= omega
                 const uint32_t old = atomicMin(dn + jend, d);
                 if (old <= d) break;
-                if (steps == WAIT_MAX) { push_node(P, R, q, jend); break; }  // continue next round
+                jend++;
+                if (++steps == WAIT_INLINE) { more = jend < vend; break; }
+            }
+            if (more) {
+                const uint32_t k = atomicAdd(R.wait_cnt, 1u);
+                if (k < P.waitcap) P.waitq[k] = make_uint4(q, jend, vend, d);
+                else push_node(P, R, q, jend - 1);  // queue full: the walk continues next round
             }
             e0 = __ldg(P.node_eoff + j);
             cnt = __ldg(P.node_eoff + jend) - e0;
@@ -229,6 +240,54 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
             const uint32_t oq = __shfl_sync(0xffffffffu, q, own);
             if (g < total) spfp_edge<FP>(P, R, oq, oe0 + (g - oex));
+        }
+    }
+}
+
+// Long wait-propagation walks: warp per walk, 32 later departure nodes of the
+// vertex per step (atomicMin with the walk's value); the improved prefix's
+// out-edges are queued as chunks for k_spfp_big of the same round.  Nodes past the
+// first non-improving one that still improved (legal: waiting is transitive) are
+// pushed to the next frontier.
+template <bool FP>
+__global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
+    const RoundV R = round_view(P);
+    const uint32_t NW = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.wait_cnt, P.waitcap);
+    const int lane = threadIdx.x & 31;
+    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t it = gw; it < NW; it += nw) {
+        const uint4 c = P.waitq[it];
+        const uint32_t q = c.x, vend = c.z, d = c.w;
+        uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
+        const uint32_t jstart = c.y;
+        uint32_t j = jstart;
+        for (;;) {
+            const uint32_t jj = j + lane;
+            bool stop = true, improved = false;
+            if (jj < vend && __ldg(P.node_t + jj) < P.omega) {
+                const uint32_t old = atomicMin(dn + jj, d);
+                improved = old > d;
+                stop = !improved;
+            }
+            const uint32_t sm = __ballot_sync(0xffffffffu, stop);
+            const uint32_t first = sm ? (uint32_t)(__ffs(sm) - 1) : 32u;
+            if (improved && (uint32_t)lane > first) push_node(P, R, q, jj);
+            j += first;
+            if (first < 32) break;
+        }
+        // out-edges of the improved nodes [jstart, j)
+        if (j > jstart) {
+            const uint32_t e0 = __ldg(P.node_eoff + jstart), e1 = __ldg(P.node_eoff + j);
+            const uint32_t nch = (e1 - e0 + CHUNK - 1) / CHUNK;
+            uint32_t k = 0;
+            if (lane == 0) k = atomicAdd(R.big_cnt, nch);
+            k = __shfl_sync(0xffffffffu, k, 0);
+            for (uint32_t cc = lane; cc < nch; cc += 32) {
+                const uint32_t b0 = e0 + cc * CHUNK, b1 = min(e1, b0 + CHUNK);
+                if (k + cc < P.bigcap) P.bigq[k + cc] = make_uint4(q, b0, b1, 0);
+                else for (uint32_t pp = b0; pp < b1; pp++) spfp_edge<FP>(P, R, q, pp);
+            }
         }
     }
 }
@@ -307,6 +366,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     P.alpha = alpha; P.omega = omega; P.use_sc = (int)g->opt_shortcuts;
     P.ctl = Q.ctl; P.fr0 = Q.fr[0]; P.fr1 = Q.fr[1];
     P.bigq = Q.bigq; P.bigcap = Q.bigcap;
+    P.waitq = Q.chq; P.waitcap = Q.chcap;
     TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl);
     {
         dim3 grid(4, Sb);
@@ -319,6 +379,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     for (;;) {
         for (int k = 0; k < group; k++) {
             TG_LAUNCH(k_spfp_activate<FP>, grid, QT, 0, s, P);
+            TG_LAUNCH(k_spfp_wait<FP>, grid, QT, 0, s, P);
             TG_LAUNCH(k_spfp_big<FP>, grid, QT, 0, s, P);
         }
         TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
