@@ -369,7 +369,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     P.waitq = Q.chq; P.waitcap = Q.chcap;
     TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl);
     {
-        dim3 grid(4, Sb);
+        dim3 grid(64, Sb);  // a hub source has many departure nodes
         TG_LAUNCH(k_spfp_init<FP>, grid, 256, 0, s, P, Q.srcs_int, Sb);
     }
     TG_LAUNCH(k_spfp_ctl_start, 1, 1, 0, s, Q.ctl);
