@@ -171,6 +171,8 @@ def run_ours(a, rank, world, local_rank):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     ge, mine, problems, win, weighted, cfg = workload(a.config, a.k, rank, world, dev, a.mode)
+    torch.cuda.synchronize()
+    torch.cuda.empty_cache()  # generator temporaries: give them back before the library allocates
     k = len(mine)
     n, m = ge.n, ge.m
     w_arg = ge.w if weighted else None
@@ -339,10 +341,14 @@ def run_ours(a, rank, world, local_rank):
         "data": "synthetic",
         "config": {
             "workload": describe(a.config, ge, k, problems, win),
-            "parallelism": (f"source-sharded x{world} (replicated graph, no data-path collective)"
-                            if a.mode == "replicate" else
-                            f"vertex-range x{world} (one batch; per-round ncclAllReduce(min) of packed states)"),
-            "step": "create+validate, build_chains (fwd+mirror), " + " + ".join(f"{p} x{k}" for p in problems),
+            "parallelism": ((f"source-sharded x{world} (replicated graph, no data-path collective)"
+                             if a.mode == "replicate" else
+                             f"vertex-range x{world} (one batch; per-round ncclAllReduce(min) of packed states)")
+                            + (f"; {a.partitions} logical vertex-range partitions per GPU (shared state)"
+                               if a.partitions > 1 else "")),
+            "step": (("" if a.query_only else
+                      "create+validate, build_chains (" + ("fwd+mirror" if "ld" in problems else "fwd") + "), ")
+                     + " + ".join(f"{p} x{k}" for p in problems)),
             "query_only": a.query_only,
             "l2": "inputs larger than L2 (edge list %.0f MB, chain structure %.0f MB > 126 MB)" % (
                 m * (20 if weighted else 16) / 1e6, info["device_bytes"] / 1e6),

@@ -108,7 +108,11 @@ tg_status DevArena::alloc(void **p, size_t bytes) {
         cudaError_t e = cudaMalloc(&q, bytes);
         if (e != cudaSuccess) {
             cudaGetLastError();
-            cache_release_all(dev);  // return cached blocks to the driver and retry once
+            // return cached blocks and the stream-ordered pool's free memory to the driver, retry once
+            cudaDeviceSynchronize();
+            cache_release_all(dev);
+            cudaMemPool_t pool;
+            if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
             e = cudaMalloc(&q, bytes);
         }
         if (e != cudaSuccess) {
@@ -299,14 +303,16 @@ tg_status tg_build_chains(tg_graph *g) {
         g->nparts = 1;
         g->part_vb[0] = (uint32_t)((uint64_t)g->n * r / P);
         g->part_vb[1] = (uint32_t)((uint64_t)g->n * (r + 1) / P);
-        TG_TRY(tg_build_partition(g, &g->pf[0], &g->pm[0], g->part_vb[0], g->part_vb[1], 0));
+        TG_TRY(tg_build_partition(g, &g->pf[0], &g->pm[0], g->part_vb[0], g->part_vb[1], 0, g->opt_mirror ? 3 : 1));
+        g->mirror_built = g->opt_mirror != 0;
     } else if (g->opt_partitions > 1) {
         // logical vertex-range partitions on one GPU (same algorithm, shared state)
         const int P = g->opt_partitions;
         g->nparts = P;
         for (int p = 0; p <= P; p++) g->part_vb[p] = (uint32_t)((uint64_t)g->n * p / P);
         for (int p = 0; p < P; p++)
-            TG_TRY(tg_build_partition(g, &g->pf[p], &g->pm[p], g->part_vb[p], g->part_vb[p + 1], 0));
+            TG_TRY(tg_build_partition(g, &g->pf[p], &g->pm[p], g->part_vb[p], g->part_vb[p + 1], 0, g->opt_mirror ? 3 : 1));
+        g->mirror_built = g->opt_mirror != 0;
     } else {
         if (g->opt_relabel) TG_TRY(tg_relabel(g, 0));
         const uint32_t *U = g->relabeled ? g->d_ru : g->d_u, *V = g->relabeled ? g->d_rv : g->d_v;
@@ -345,16 +351,21 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
     cudaStream_t s = (cudaStream_t)cuda_stream;
     const bool out_dev = is_device_ptr(out);
     const bool pred_dev = is_device_ptr(pred);
+    if (p == TG_LD && !g->mirror_built) {  // lazily built mirror (option "mirror" = 0)
+        if (g->nparts > 0) {
+            for (int pi = 0; pi < g->nparts; pi++)
+                TG_TRY(tg_build_partition(g, &g->pf[pi], &g->pm[pi], g->part_vb[pi], g->part_vb[pi + 1], 0, 2));
+        } else {
+            TG_TRY(tg_build_mirror(g, 0));
+        }
+        g->mirror_built = true;
+    }
     if (g->nparts > 0) {
         if (!(p == TG_EAT || p == TG_LD || p == TG_REACH)) {
             tg_set_error("vertex-range partitioned graphs answer TG_EAT / TG_LD / TG_REACH only");
             return TG_ERR_STATE;
         }
         return tg_run_eat_partitioned(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
-    }
-    if (p == TG_LD && !g->mirror_built) {  // lazily built mirror (option "mirror" = 0)
-        TG_TRY(tg_build_mirror(g, 0));
-        g->mirror_built = true;
     }
     if (p == TG_EAT || p == TG_LD || p == TG_REACH)
         return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);

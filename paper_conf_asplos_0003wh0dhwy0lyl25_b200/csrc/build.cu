@@ -487,14 +487,18 @@ tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {
 // One vertex-range partition [vb, ve): forward chains over the edges leaving the
 // range, mirror chains over the edges entering it (the mirror's sources).
 // Slots keep the original edge ids (id map).
-tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s) {
+tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,
+                             int dirs) {
     const uint64_t m = g->m;
     uint32_t *mt = nullptr, *flag = nullptr, *cnt = nullptr;
-    TG_TRY_CUDA(tg_malloc_async((void **)&mt, std::max<uint64_t>(m, 1) * 4, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&flag, std::max<uint64_t>(m, 1) * 4, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&cnt, 4, s));
-    if (m) TG_LAUNCH(k_mirror, blocks_for(m, 4), BT, 0, s, g->d_t, g->d_dur, m, g->max_arr, mt);
+    if (dirs & 2) {
+        TG_TRY_CUDA(tg_malloc_async((void **)&mt, std::max<uint64_t>(m, 1) * 4, s));
+        if (m) TG_LAUNCH(k_mirror, blocks_for(m, 4), BT, 0, s, g->d_t, g->d_dur, m, g->max_arr, mt);
+    }
     for (int dir = 0; dir < 2; dir++) {
+        if (!((dirs >> dir) & 1)) continue;  // bit 0 forward, bit 1 mirror
         // forward: (u, v, t); mirror: (v, u, C - t - dur)
         const uint32_t *key = dir == 0 ? g->d_u : g->d_v;
         const uint32_t *uu = dir == 0 ? g->d_u : g->d_v;
@@ -520,7 +524,7 @@ tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint
         cudaFreeAsync(sub, s);
         if (r != TG_OK) return r;
     }
-    cudaFreeAsync(mt, s);
+    if (mt) cudaFreeAsync(mt, s);
     cudaFreeAsync(flag, s);
     cudaFreeAsync(cnt, s);
     TG_TRY_CUDA(cudaStreamSynchronize(s));

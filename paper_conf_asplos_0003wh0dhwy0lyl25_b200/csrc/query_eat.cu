@@ -448,6 +448,24 @@ __global__ void k_part_frontier(const unsigned long long *__restrict__ st, uint3
     uint32_t mine = 0;
     const uint64_t u0 = (uint64_t)vb * G, u1 = (uint64_t)ve * G;  // frontier units of the range
     const uint32_t lane = threadIdx.x & 31;
+    if (S < 16) {
+        // few queries: thread per unit word, looping over its queries
+        for (uint64_t unit = u0 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; unit < u1;
+             unit += (uint64_t)gridDim.x * blockDim.x) {
+            const uint32_t v = (uint32_t)(unit / G);
+            uint32_t w = 0;
+            for (uint32_t q = 0; q < S; q++) {
+                const size_t si = (size_t)v * S + q;
+                const uint32_t now = (uint32_t)(st[si] >> 32);
+                if (now < lat[si]) { lat[si] = now; w |= 1u << q; }
+            }
+            fnext[unit] = w;
+            mine += __popc(w);
+        }
+        for (int o = 16; o; o >>= 1) mine += __shfl_xor_sync(0xffffffffu, mine, o);
+        if (lane == 0 && mine) atomicAdd(count, mine);
+        return;
+    }
     const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t unit = u0 + gw; unit < u1; unit += nw) {  // warp per unit: lane = query bit

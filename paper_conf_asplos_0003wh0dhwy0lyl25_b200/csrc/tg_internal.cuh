@@ -199,7 +199,8 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
 tg_status tg_relabel(tg_graph *g, cudaStream_t s);
 // sources of a sub-batch: copy (host) and map to the internal vertex order
 tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cudaStream_t s);
-tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s);
+tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,
+                             int dirs);  // dirs: bit 0 forward, bit 1 mirror
 
 tg_status tg_run_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                        uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);

@@ -348,7 +348,7 @@ def test_logical_partitions_random(tg, parts):
 def test_logical_partitions_c1(tg):
     ge = tgsynth.make_graph("C1")
     n, u, v, t, d, w = ge.numpy()
-    g = _gpu_graph(tg, n, u, v, t, d, w, partitions=4)
+    g = _gpu_graph(tg, n, u, v, t, d, w, partitions=4, mirror=0)  # LD mirror built on first use
     og = oracle.Graph(n, u, v, t, d, w)
     for win in tgsynth.CONFIGS["C1"]["windows"]:
         _check_rows(tg, g, og, "eat", [0, 5, 99], win)

@@ -140,11 +140,15 @@ def chung_lu_endpoints(n: int, m: int, seed: int, exponent=2.0, device="cpu", ch
     return u, v
 
 
-def uniform_times(m, seed, t_hi, dur_lo, dur_hi, w_lo=1, w_hi=101, device="cpu"):
-    idx = torch.arange(m, dtype=torch.int64, device=device)
-    t = uniform_int(seed, 3000, idx, 0, t_hi).int()
-    dur = uniform_int(seed, 3001, idx, dur_lo, dur_hi + 1).int()
-    w = uniform_int(seed, 3002, idx, w_lo, w_hi).int()
+def uniform_times(m, seed, t_hi, dur_lo, dur_hi, w_lo=1, w_hi=101, device="cpu", chunk=1 << 24):
+    t = torch.empty(m, dtype=torch.int32, device=device)
+    dur = torch.empty(m, dtype=torch.int32, device=device)
+    w = torch.empty(m, dtype=torch.int32, device=device)
+    for s, e in _chunks(m, chunk):
+        idx = torch.arange(s, e, dtype=torch.int64, device=device)
+        t[s:e] = uniform_int(seed, 3000, idx, 0, t_hi).int()
+        dur[s:e] = uniform_int(seed, 3001, idx, dur_lo, dur_hi + 1).int()
+        w[s:e] = uniform_int(seed, 3002, idx, w_lo, w_hi).int()
     return t, dur, w
 
 
