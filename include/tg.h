@@ -188,8 +188,8 @@ TG_API tg_status tg_last_query_stats(const tg_graph *g, tg_query_stats *st, uint
  *   mode 1 (vertex range): ONE query batch is partitioned: rank r owns vertices
  *     [n*r/N, n*(r+1)/N) and the chains of the edges leaving them (and, for LD,
  *     of the mirror edges leaving them).  After every GAC round the packed
- *     (arrival << 32 | pred) states are combined with ncclAllReduce(min) over
- *     NVLink; `out`/`pred` are complete on every rank.  EAT / LD / REACH only.
+ *     (arrival << 32 | pred) states -- u32 arrivals when pred == NULL -- are combined
+ *     with ncclAllReduce(min) over NVLink; `out`/`pred` are complete on every rank.  EAT / LD / REACH only.
  * NCCL is loaded at run time (dlopen "libnccl.so.2"), sharing the process's copy. */
 
 /* 128-byte ncclUniqueId for tg_comm_create (rank 0 creates it, the caller broadcasts it). */
@@ -212,7 +212,14 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *   "relabel"    1 = internal vertex order by descending in-degree (before build; default 0:
  *                no gain measured on R-MAT); invisible to callers
  *   "partitions" logical vertex-range partitions on this GPU (1..16, before build):
- *                runs the multi-GPU mode-1 algorithm inside one process (tests) */
+ *                runs the multi-GPU mode-1 algorithm inside one process (tests)
+ *   "engine"     EAT/LD/REACH schedule: 0 = automatic (GAC), 1 = GAC rounds over chains
+ *                (Alg. 3), 2 = time-partitioned sweep (experimental; needs "sweep_struct")
+ *   "sweep_struct" 1 = also build the time-ordered edge list in tg_build_chains (default 0)
+ *   "sweep_part" sweep: edges per time partition (0 = automatic)
+ *   "packed_state" 1 = EAT/LD/REACH keep the packed u64 (arrival << 32 | pred) state even
+ *                when pred == NULL (default 0: without pred the state is the u32 arrival
+ *                alone -- half the state bytes; values are identical) */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
 
 /* Total kernels this library has launched in this process (all handles). */

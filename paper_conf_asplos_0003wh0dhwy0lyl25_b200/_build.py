@@ -32,16 +32,19 @@ def needs_build() -> bool:
     return any(os.path.getmtime(p) > t for p in sources() + headers())
 
 
-def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, jobs: int | None = None,
+          extra_flags: tuple = (), out: str | None = None) -> str:
+    """Compile csrc/*.cu into LIB (or `out`, with `extra_flags` -D... for tuning variants)."""
+    lib = out or LIB
+    if not force and out is None and not needs_build():
         return LIB
-    objdir = os.path.join(HERE, "build")
+    objdir = os.path.join(HERE, "build", os.path.basename(lib).replace(".so", ""))
     os.makedirs(objdir, exist_ok=True)
     procs, objs = [], []
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
         objs.append(obj)
-        cmd = [NVCC, *FLAGS, "-I", INCLUDE, "-c", src, "-o", obj]
+        cmd = [NVCC, *FLAGS, *extra_flags, "-I", INCLUDE, "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd))
         procs.append((subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT), src))
@@ -54,12 +57,12 @@ def build(force: bool = False, verbose: bool = False, jobs: int | None = None) -
             print(out.decode(errors="replace"))
     if err:
         raise RuntimeError("nvcc failed:\n" + "\n".join(err))
-    tmp = LIB + ".tmp"
+    tmp = lib + ".tmp"
     cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-cudart", "static",
            "-Xcompiler", "-fPIC", "-o", tmp, *objs, "-lpthread", "-ldl", "-lrt"]
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":

@@ -76,6 +76,12 @@ tg_status tg_comm_allreduce_min_u64(tg_comm *c, unsigned long long *buf, uint64_
     return TG_OK;
 }
 
+tg_status tg_comm_allreduce_min_u32(tg_comm *c, uint32_t *buf, uint64_t count, cudaStream_t s) {
+    if (!c->comm) return TG_OK;
+    TG_TRY_NCCL(nccl().AllReduce(buf, buf, count, kNcclUint32, kNcclMin, c->comm, s));
+    return TG_OK;
+}
+
 tg_status tg_comm_allreduce_sum_u32(tg_comm *c, uint32_t *buf, uint64_t count, cudaStream_t s) {
     if (!c->comm) return TG_OK;
     TG_TRY_NCCL(nccl().AllReduce(buf, buf, count, kNcclUint32, kNcclSum, c->comm, s));

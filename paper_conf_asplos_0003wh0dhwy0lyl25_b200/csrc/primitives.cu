@@ -215,6 +215,17 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const unsigned lon
 
 tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
                               unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s) {
+    return tg_radix_sort_pairs_snap(keys, vals, m, key_bits, sorted_keys, sorted_vals, s, 0, nullptr);
+}
+
+// As above; additionally, after the first `snap_bits` key bits have been sorted
+// (snap_bits a multiple of 8), the payload order of that intermediate state (stable
+// by the low snap_bits bits) is copied to snap_vals.
+tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
+                                   unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s,
+                                   int snap_bits, uint32_t *snap_vals) {
+    if (snap_vals && m >= 1 && (snap_bits <= 0 || m == 1 || key_bits <= 0))
+        TG_TRY_CUDA(cudaMemcpyAsync(snap_vals, vals, m * 4, cudaMemcpyDeviceToDevice, s));
     *sorted_keys = keys;
     *sorted_vals = vals;
     if (m <= 1 || key_bits <= 0) return TG_OK;
@@ -238,6 +249,8 @@ tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t
                   (uint32_t)ntiles);
         std::swap(ka, kb);
         std::swap(va, vb);
+        if (snap_vals && snap_bits > 0 && shift + 8 == snap_bits)
+            TG_TRY_CUDA(cudaMemcpyAsync(snap_vals, va, m * 4, cudaMemcpyDeviceToDevice, s));
     }
     TG_TRY_CUDA(cudaFreeAsync(counts, s));
     if (ka != keys) {

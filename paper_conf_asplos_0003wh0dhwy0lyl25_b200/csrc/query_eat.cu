@@ -47,13 +47,19 @@ constexpr int QT = 256;                 // threads per block
 constexpr uint32_t BIG_T = 128;         // unions longer than this are split into chunks
 constexpr uint32_t CHUNK = 128;         // edges per chunk (one warp)
 constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in the activating thread
+#ifndef TG_MLP
+#define TG_MLP 4                        // state reads in flight per lane in the pair loop
+#endif
+#ifndef TG_ACT_MINB
+#define TG_ACT_MINB 8                   // resident blocks per SM requested for the relax kernels
+#endif
 
 struct EatP {
     const uint32_t *vnode_off, *node_t, *node_eoff, *occ_slot;
     const int4 *slots;
     const uint2 *lc;
     const int4 *sc;
-    unsigned long long *st;
+    void *st;  // [v * S + q]: packed u64 (arrival << 32 | pred) when PK, else u32 arrival
     uint32_t *act, *bits;
     uint32_t *touched;  // stats: slots relaxed by any query of the sub-batch
     uint64_t bit_words;
@@ -71,6 +77,8 @@ struct EatP {
     uint4 *chq;
     uint64_t chcap;
     unsigned long long *relax_cnt;
+    unsigned long long *diag;  // stats: [0] union edges scanned [1] unit ranges [2] (edge, query) pairs
+                               //        [3] (vertex, query) activations with a non-empty range [4] frontier bits
 };
 
 // per-round view derived from the device-side round control
@@ -116,23 +124,53 @@ __device__ __forceinline__ void round_advance(RoundCtl *ctl) {
 // Layouts interleave the S queries of a sub-batch (query index fastest):
 //   st / act [v * S + q], frontier masks [v * G + q / 32] (bit q % 32), claim words [(slot >> 5) * S + q],
 // so the queries of a sub-batch that touch the same vertex or slot touch adjacent words.
-__device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t slot, uint32_t v,
-                                          uint32_t arr, uint32_t id) {
-    const size_t i = (size_t)v * P.S + q;
-    const unsigned long long pk = ((unsigned long long)arr << 32) | id;
+//
+// State word: PK = packed (arrival << 32 | pred edge id), u64 -- the pred of reading A9
+// rides in the low half of the min.  !PK (the caller passed pred = NULL): the arrival
+// alone, u32 -- half the bytes per state read / atomic, same arithmetic on the time.
+template <bool PK> struct StW;
+template <> struct StW<true> {
+    using T = unsigned long long;
+    static __device__ __forceinline__ T make(uint32_t arr, uint32_t id) { return ((T)arr << 32) | id; }
+    static __device__ __forceinline__ uint32_t time(T w) { return (uint32_t)(w >> 32); }
+};
+template <> struct StW<false> {
+    using T = uint32_t;
+    static __device__ __forceinline__ T make(uint32_t arr, uint32_t) { return arr; }
+    static __device__ __forceinline__ uint32_t time(T w) { return w; }
+};
+
+template <bool PK>
+__device__ __forceinline__ typename StW<PK>::T st_load(const EatP &P, size_t i) {
+    return ((const typename StW<PK>::T *)P.st)[i];
+}
+
+// Relax (v, q) with (arr, id) given a value `cur` read earlier from the state (any
+// earlier read: states only decrease, so a stale value is an upper bound and when it
+// is already <= the candidate the atomic cannot change anything -- most relaxations).
+template <bool PK>
+__device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, uint32_t q, uint32_t slot, uint32_t v,
+                                              uint32_t arr, uint32_t id, typename StW<PK>::T cur) {
+    using W = StW<PK>;
     if (P.stats) {  // work counters: relaxations per query, distinct slots of the sub-batch
         atomicAdd(P.relax_cnt + q, 1ull);
         atomicOr(P.touched + (slot >> 5), 1u << (slot & 31));
     }
-    // States only decrease: a stale cached read is an upper bound, so when it is
-    // already <= pk the atomic cannot change anything (most relaxations, W >> n).
-    if (P.st[i] <= pk) return;
-    const unsigned long long old = atomicMin(P.st + i, pk);
-    if (arr < (uint32_t)(old >> 32)) {
+    const typename W::T pk = W::make(arr, id);
+    if (cur <= pk) return;
+    const size_t i = (size_t)v * P.S + q;
+    const typename W::T old = atomicMin((typename W::T *)P.st + i, pk);
+    if (arr < W::time(old)) {
         // arrival improved: v joins the next round's frontier (bitmap: duplicates merge;
         // no shared counter -- the next activation counts the non-empty words it finds)
         atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
     }
+}
+
+template <bool PK>
+__device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t slot, uint32_t v,
+                                          uint32_t arr, uint32_t id) {
+    eat_relax_cur<PK>(P, R, q, slot, v, arr, id, st_load<PK>(P, (size_t)v * P.S + q));
 }
 
 // test-and-set of slot s's claim bit for query q; true if this caller claimed it
@@ -143,28 +181,30 @@ __device__ __forceinline__ bool claim(const EatP &P, uint32_t q, uint32_t s) {
 
 // sequential walk over slots [s, s_end): claim, relax, continue; stop at a slot
 // somebody else claimed (they continue) or past omega.
+template <bool PK>
 __device__ __forceinline__ void eat_walk(const EatP &P, const RoundV &R, uint32_t q, uint32_t s, uint32_t s_end) {
     for (; s < s_end; s++) {
         const int4 sl = tg_ld_slot(P.slots + s);
         if ((uint32_t)sl.y > P.omega) return;  // arrivals increase strictly along a chain
         if (!claim(P, q, s)) return;
-        eat_relax(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+        eat_relax<PK>(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     }
 }
 
 // A newly usable occurrence at slot s (already loaded) of a long chain.
+template <bool PK>
 __device__ __forceinline__ void eat_long(const EatP &P, const RoundV &R, uint32_t q, uint32_t s, int4 sl) {
     const uint32_t l = (uint32_t)sl.w;
     const uint2 info = __ldg(P.lc + l);  // {first slot, length}
     if (s != info.x && !claim(P, q, s)) return;  // a walker from an earlier entry got here first
-    eat_relax(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+    eat_relax<PK>(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     uint32_t s_end = info.x + info.y;
     if (s + 1 >= s_end) return;
     if (P.use_sc) {
         // skeleton: Propagate along the shortcut head -> tail (Alg. 2 / Alg. 3 line 6)
         const int4 scv = __ldg(P.sc + l);
         if ((uint32_t)scv.y <= P.omega && claim(P, q, s_end - 1)) {
-            eat_relax(P, R, q, s_end - 1, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
+            eat_relax<PK>(P, R, q, s_end - 1, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
             s_end -= 1;
         }
     }
@@ -175,7 +215,7 @@ __device__ __forceinline__ void eat_long(const EatP &P, const RoundV &R, uint32_
             return;
         }
     }
-    eat_walk(P, R, q, s + 1, s_end);
+    eat_walk<PK>(P, R, q, s + 1, s_end);
 }
 
 // Per-warp shared-memory staging of one 32-edge block: the (edge, query) pairs
@@ -186,9 +226,14 @@ struct WarpStage {
     uint32_t sidx[32];
 };
 
+template <bool PK>
 __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint32_t g, uint32_t lo, uint32_t hi,
                                            uint32_t pbeg, uint32_t pend, WarpStage &ws) {
     const int lane = threadIdx.x & 31;
+    if (P.stats && lane == 0) {
+        atomicAdd(P.diag + 0, (unsigned long long)(pend - pbeg));
+        atomicAdd(P.diag + 1, 1ull);
+    }
     for (uint32_t pb = pbeg; pb < pend; pb += 32) {
         const uint32_t p = pb + lane;
         uint32_t s = 0;
@@ -215,6 +260,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         }
         const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
         if (total == 0) continue;
+        if (P.stats && lane == 0) atomicAdd(P.diag + 2, (unsigned long long)total);
         // expand: edge lane k writes its pairs at [incl - cnt, incl) in edge-major order
         ws.slot[lane] = sl;
         ws.sidx[lane] = s;
@@ -225,15 +271,36 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
             ws.pairs[pos++] = (uint16_t)((lane << 5) | bq);
         }
         __syncwarp();
-        for (uint32_t t = lane; t < total; t += 32) {
-            const uint32_t e = ws.pairs[t];
-            const uint32_t k = e >> 5;
-            const uint32_t q = g * 32 + (e & 31);
-            const int4 osl = ws.slot[k];
-            if ((uint32_t)osl.w == TG_SINGLE)
-                eat_relax(P, R, q, ws.sidx[k], (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z);
-            else
-                eat_long(P, R, q, ws.sidx[k], osl);
+        // Lanes take the pairs 4 at a time: the 4 state reads of one-edge chains are
+        // issued before any is used (memory-level parallelism: the filter read is the
+        // latency the relax phase waits on), then each is filtered / relaxed.
+        for (uint32_t t0 = 0; t0 < total; t0 += 32 * TG_MLP) {
+            typename StW<PK>::T cur[TG_MLP];
+#pragma unroll
+            for (int j = 0; j < TG_MLP; j++) {
+                const uint32_t t = t0 + j * 32 + lane;
+                if (t < total) {
+                    const uint32_t e = ws.pairs[t];
+                    const int4 osl = ws.slot[e >> 5];
+                    if ((uint32_t)osl.w == TG_SINGLE)
+                        cur[j] = st_load<PK>(P, (size_t)(uint32_t)osl.x * P.S + g * 32 + (e & 31));
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < TG_MLP; j++) {
+                const uint32_t t = t0 + j * 32 + lane;
+                if (t < total) {
+                    const uint32_t e = ws.pairs[t];
+                    const uint32_t k = e >> 5;
+                    const uint32_t q = g * 32 + (e & 31);
+                    const int4 osl = ws.slot[k];
+                    if ((uint32_t)osl.w == TG_SINGLE)
+                        eat_relax_cur<PK>(P, R, q, ws.sidx[k], (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z,
+                                          cur[j]);
+                    else
+                        eat_long<PK>(P, R, q, ws.sidx[k], osl);
+                }
+            }
         }
         __syncwarp();
     }
@@ -246,7 +313,8 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
 // an edge index (atomicMin makes concurrent activations disjoint).  The union of
 // the lanes' ranges is relaxed edge-major (unit_range); long unions are split into
 // chunks for k_eat_big.
-__global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
+template <bool PK>
+__global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
     __shared__ WarpStage stage[QT / 32];
     WarpStage &ws = stage[threadIdx.x >> 5];
@@ -275,7 +343,7 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
             uint32_t lo = 0, hi = 0;
             if ((qm >> lane) & 1u) {
                 const size_t si = (size_t)v * P.S + q;
-                const uint32_t now = (uint32_t)(__ldcg(P.st + si) >> 32);
+                const uint32_t now = StW<PK>::time(__ldcg((const typename StW<PK>::T *)P.st + si));
                 const uint32_t a = __ldg(P.vnode_off + v), b = __ldg(P.vnode_off + v + 1);
                 const uint32_t j0 = tg_lower_bound(P.node_t, a, b, max(now, P.alpha));
                 const uint32_t elo = __ldg(P.node_eoff + j0);
@@ -287,6 +355,12 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
                     if (prev == TG_NONE) ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, j0, b, P.omega));
                     if (elo < ehi) { lo = elo; hi = ehi; }
                 }
+            }
+            if (P.stats && lane == 0) {
+                atomicAdd(P.diag + 3, (unsigned long long)__popc(__ballot_sync(0xffffffffu, lo < hi)));
+                atomicAdd(P.diag + 4, (unsigned long long)__popc(qm));
+            } else if (P.stats) {
+                __ballot_sync(0xffffffffu, lo < hi);
             }
             uint32_t ulo = (lo < hi) ? lo : 0xFFFFFFFFu, uhi = hi;
 #pragma unroll
@@ -320,7 +394,7 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
                     ulo = ulo + queued * CHUNK;  // the rest, in place
                 }
             }
-            unit_range(P, R, g, lo, hi, ulo, uhi, ws);
+            unit_range<PK>(P, R, g, lo, hi, ulo, uhi, ws);
         }
     }
     if (lane == 0 && my_units) atomicAdd(&s_units, my_units);
@@ -329,7 +403,8 @@ __global__ void __launch_bounds__(QT, 8) k_eat_activate(EatP P) {
 }
 
 // Chunks of long unions: one warp per chunk, the unit's 32 query ranges from its record.
-__global__ void __launch_bounds__(QT, 8) k_eat_big(EatP P) {
+template <bool PK>
+__global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_big(EatP P) {
     const RoundV R = round_view(P);
     __shared__ WarpStage stage[QT / 32];
     WarpStage &ws = stage[threadIdx.x >> 5];
@@ -340,13 +415,14 @@ __global__ void __launch_bounds__(QT, 8) k_eat_big(EatP P) {
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
         const uint2 r = P.recs[(size_t)c.x * 32 + lane];
-        unit_range(P, R, c.w, r.x, r.y, c.y, c.z, ws);
+        unit_range<PK>(P, R, c.w, r.x, r.y, c.y, c.z, ws);
     }
 }
 
 // ChainEngine: warp per queued walk, lanes over consecutive slots; the warp
 // continues iff its last lane claimed its slot (otherwise that slot's claimer
 // continues the chain).  Advances the round when the last block finishes.
+template <bool PK>
 __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
     const RoundV R = round_view(P);
     const uint32_t C = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.ch_cnt, P.chcap);
@@ -363,7 +439,7 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
                 if ((uint32_t)sl.y > P.omega) {
                     past = true;
                 } else if (claim(P, c.x, s)) {
-                    eat_relax(P, R, c.x, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+                    eat_relax<PK>(P, R, c.x, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
                     cont = true;
                 }
             }
@@ -377,11 +453,12 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
 
 // VInitial (Table 1): every state INF (memset), the source = (alpha, no pred),
 // frontier = the sources; round control reset for a new loop.
-__global__ void k_eat_init(unsigned long long *st, uint32_t n, uint32_t G, const uint32_t *srcs, uint32_t S,
+template <bool PK>
+__global__ void k_eat_init(void *st, uint32_t n, uint32_t G, const uint32_t *srcs, uint32_t S,
                            uint32_t alpha, uint32_t *fb1, RoundCtl *ctl, int push) {
     for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < S; q += gridDim.x * blockDim.x) {
         const uint32_t x = srcs[q];
-        st[(size_t)x * S + q] = ((unsigned long long)alpha << 32) | TG_NONE;
+        ((typename StW<PK>::T *)st)[(size_t)x * S + q] = StW<PK>::make(alpha, TG_NONE);
         if (push) atomicOr(fb1 + (size_t)x * G + (q >> 5), 1u << (q & 31));
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -396,11 +473,14 @@ __global__ void k_eat_init(unsigned long long *st, uint32_t n, uint32_t G, const
 // mode 0 = EAT, 1 = LD (mirror: value = C - time; target = omega), 2 = REACH.
 // st is [v][q]; out rows are [q][v]: a block transposes a tile of 32 vertices x S
 // queries through shared memory so both the read and the writes are coalesced.
-__global__ void __launch_bounds__(256) k_eat_extract(const unsigned long long *__restrict__ st, uint32_t n, uint32_t S,
+template <bool PK>
+__global__ void __launch_bounds__(256) k_eat_extract(const void *__restrict__ st_, uint32_t n, uint32_t S,
                                                      const uint32_t *__restrict__ srcs, int mode, uint32_t C,
                                                      uint32_t omega, uint32_t *__restrict__ out,
                                                      uint32_t *__restrict__ pred, const uint32_t *__restrict__ perm) {
     __shared__ unsigned long long tile[32 * 65];
+    const typename StW<PK>::T *st = (const typename StW<PK>::T *)st_;
+    const typename StW<PK>::T INF = (typename StW<PK>::T)~0ull;
     const uint32_t nt = (n + 31) / 32;
     for (uint32_t tb = blockIdx.x; tb < nt; tb += gridDim.x) {
         const uint32_t v0 = tb * 32;
@@ -411,16 +491,16 @@ __global__ void __launch_bounds__(256) k_eat_extract(const unsigned long long *_
                 const uint32_t dv = i / qs, dq = i - dv * qs;
                 const uint32_t v = v0 + dv;
                 // rows are in the engine's vertex order (perm: caller id -> internal id)
-                tile[dv * 65 + dq] = (v < n) ? st[(size_t)(perm ? perm[v] : v) * S + q0 + dq] : ~0ull;
+                tile[dv * 65 + dq] = (v < n) ? st[(size_t)(perm ? perm[v] : v) * S + q0 + dq] : INF;
             }
             __syncthreads();
             for (uint32_t i = threadIdx.x; i < 32 * qs; i += blockDim.x) {
                 const uint32_t dq = i / 32, dv = i - dq * 32;
                 const uint32_t v = v0 + dv, q = q0 + dq;
                 if (v >= n) continue;
-                const unsigned long long pk = tile[dv * 65 + dq];
-                const bool reached = pk != ~0ull;
-                const uint32_t t = (uint32_t)(pk >> 32), id = (uint32_t)pk;
+                const typename StW<PK>::T pk = (typename StW<PK>::T)tile[dv * 65 + dq];
+                const bool reached = pk != INF;
+                const uint32_t t = StW<PK>::time(pk), id = PK ? (uint32_t)pk : TG_NONE;
                 uint32_t val, pr = reached ? id : TG_NONE;
                 const uint32_t src = srcs[q];
                 if (mode == 0) {
@@ -442,9 +522,11 @@ __global__ void __launch_bounds__(256) k_eat_extract(const unsigned long long *_
 // next frontier of ITS vertices from the state itself (bits set by relaxations are
 // discarded): (v, q) is active iff its arrival dropped below the last activated one.
 // One thread per unit bit, so a warp assembles one frontier word with a ballot.
-__global__ void k_part_frontier(const unsigned long long *__restrict__ st, uint32_t *__restrict__ lat,
+template <bool PK>
+__global__ void k_part_frontier(const void *__restrict__ st_, uint32_t *__restrict__ lat,
                                 uint32_t *__restrict__ fnext, uint32_t S, uint32_t G, uint32_t vb, uint32_t ve,
                                 uint32_t *__restrict__ count) {
+    const typename StW<PK>::T *st = (const typename StW<PK>::T *)st_;
     uint32_t mine = 0;
     const uint64_t u0 = (uint64_t)vb * G, u1 = (uint64_t)ve * G;  // frontier units of the range
     const uint32_t lane = threadIdx.x & 31;
@@ -456,7 +538,7 @@ __global__ void k_part_frontier(const unsigned long long *__restrict__ st, uint3
             uint32_t w = 0;
             for (uint32_t q = 0; q < S; q++) {
                 const size_t si = (size_t)v * S + q;
-                const uint32_t now = (uint32_t)(st[si] >> 32);
+                const uint32_t now = StW<PK>::time(st[si]);
                 if (now < lat[si]) { lat[si] = now; w |= 1u << q; }
             }
             fnext[unit] = w;
@@ -474,7 +556,7 @@ __global__ void k_part_frontier(const unsigned long long *__restrict__ st, uint3
         bool on = false;
         if (q < S) {
             const size_t si = (size_t)v * S + q;
-            const uint32_t now = (uint32_t)(st[si] >> 32);
+            const uint32_t now = StW<PK>::time(st[si]);
             if (now < lat[si]) { lat[si] = now; on = true; }
         }
         const uint32_t w = __ballot_sync(0xffffffffu, on);
@@ -504,7 +586,7 @@ __global__ void k_ctl_reset(RoundCtl *ctl) {
 static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     QueryScratch &Q = g->qs;
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
-    if (Q.S >= S && Q.n == g->n && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat)) return TG_OK;
+    if (Q.S >= S && Q.n == g->n && Q.st && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat)) return TG_OK;
     TG_TRY_CUDA(cudaDeviceSynchronize());  // blocks go back to the cache for immediate reuse
     Q.arena.free_all();
     if (Q.h_ctr) { cudaFreeHost(Q.h_ctr); Q.h_ctr = nullptr; }
@@ -553,7 +635,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
     TG_TRY(A.alloc((void **)&Q.srcs, S * 4));
     TG_TRY(A.alloc((void **)&Q.srcs_int, S * 4));
-    TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8 + 8));  // [S] per query + [S] = distinct slots
+    TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8 + 8 + 64));  // [S] per query, [S] distinct slots, [S+1..] diag
     TG_TRY(A.alloc((void **)&Q.touched, ((m + 31) / 32 + TG_MAXP + 1) * 4));
     if (nodes_state) {
         TG_TRY(A.alloc((void **)&Q.dnode, std::max<uint64_t>(S * nnodes, 1) * 4));
@@ -583,23 +665,41 @@ uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
 
 tg_status tg_ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) { return ensure_scratch(g, S, nodes_state); }
 
+// Sources and host staging only (engines with their own state, e.g. the sweep).
+tg_status tg_ensure_scratch_srcs(tg_graph *g, uint32_t S) {
+    QueryScratch &Q = g->qs;
+    if (Q.S >= S && Q.n == g->n && Q.srcs) return TG_OK;
+    if (Q.st) return ensure_scratch(g, std::max(S, Q.S), Q.nodes_state);  // full scratch keeps working
+    TG_TRY_CUDA(cudaDeviceSynchronize());
+    Q.arena.free_all();
+    if (Q.h_ctr) { cudaFreeHost(Q.h_ctr); Q.h_ctr = nullptr; }
+    Q = QueryScratch{};
+    Q.S = S;
+    Q.n = g->n;
+    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
+    TG_TRY(Q.arena.alloc((void **)&Q.srcs, S * 4));
+    TG_TRY(Q.arena.alloc((void **)&Q.srcs_int, S * 4));
+    return TG_OK;
+}
+
 // Run the GAC rounds of one sub-batch on direction cg; returns rounds used.
+template <bool PK>
 static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
                             bool any_work, cudaStream_t s, uint32_t *rounds_out) {
     QueryScratch &Q = g->qs;
     const uint64_t n = g->n;
-    TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, S * n * 8, s));
+    TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, S * n * (PK ? 8 : 4), s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, S * n * 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, S * Q.bit_words * 4, s));
     const uint32_t G = (S + 31) / 32;
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
     if (g->opt_stats) {
-        TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8 + 8, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8 + 8 + 64, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
     }
     const bool work = any_work && g->m > 0 && alpha < omega;
-    TG_LAUNCH(k_eat_init, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
+    TG_LAUNCH(k_eat_init<PK>, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
     uint32_t rounds = 0;
     if (work) {
@@ -613,14 +713,15 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         P.touched = Q.touched;
-        const uint32_t grid = tg_grid_persistent(8);
+        P.diag = Q.relax_cnt + S + 1;
+        const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;
         const int group = trace ? 1 : (int)std::max<int64_t>(1, g->opt_round_group);
         for (;;) {
             for (int k = 0; k < group; k++) {
-                TG_LAUNCH(k_eat_activate, grid, QT, 0, s, P);
-                TG_LAUNCH(k_eat_big, grid, QT, 0, s, P);
-                TG_LAUNCH(k_eat_chain, grid, QT, 0, s, P);
+                TG_LAUNCH(k_eat_activate<PK>, grid, QT, 0, s, P);
+                TG_LAUNCH(k_eat_big<PK>, grid, QT, 0, s, P);
+                TG_LAUNCH(k_eat_chain<PK>, grid, QT, 0, s, P);
             }
             TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
@@ -664,29 +765,40 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     }
     const uint64_t launches0 = g_tg_launches;
     const int mode = ld ? 1 : (p == TG_REACH ? 2 : 0);
+    // packed (arrival | pred) states only when the caller asked for preds (or forced)
+    const bool pk = pred != nullptr || g->opt_packed_state;
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
         TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
         uint32_t rounds = 0;
-        TG_TRY(eat_rounds(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
+        if (pk) TG_TRY(eat_rounds<true>(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
+        else TG_TRY(eat_rounds<false>(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
         g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;
         uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
         uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
         const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
-        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
-                  g->relabeled ? g->perm : (const uint32_t *)nullptr);
+        if (pk)
+            TG_LAUNCH(k_eat_extract<true>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
+                      g->relabeled ? g->perm : (const uint32_t *)nullptr);
+        else
+            TG_LAUNCH(k_eat_extract<false>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
+                      g->relabeled ? g->perm : (const uint32_t *)nullptr);
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (g->opt_stats) {
             const uint64_t tw = (g->m + 31) / 32 + TG_MAXP + 1;
             TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, Q.touched, tw,
                       Q.relax_cnt + Sb);
-            std::vector<unsigned long long> h(Sb + 1);
-            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, (Sb + 1) * 8, cudaMemcpyDeviceToHost, s));
+            std::vector<unsigned long long> h(Sb + 1 + 8);
+            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, (Sb + 1 + 8) * 8, cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
             for (uint32_t q = 0; q < Sb; q++) { g->last_relax[b0 + q] = h[q]; g->last.slots_relaxed += h[q]; }
             g->last.slots_union += h[Sb];
+            static const bool trace = getenv("TG_TRACE") != nullptr;
+            if (trace)
+                fprintf(stderr, "[tg] diag S=%u: union edges %llu, unit ranges %llu, pairs %llu, activations %llu, "
+                        "frontier bits %llu\n", Sb, h[Sb + 1], h[Sb + 2], h[Sb + 3], h[Sb + 4], h[Sb + 5]);
         }
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
@@ -697,6 +809,7 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
 // ============================================================================ vertex-range partitions
 tg_status tg_comm_allreduce_min_u64(tg_comm *c, unsigned long long *buf, uint64_t count, cudaStream_t s);
 tg_status tg_comm_allreduce_sum_u32(tg_comm *c, uint32_t *buf, uint64_t count, cudaStream_t s);
+tg_status tg_comm_allreduce_min_u32(tg_comm *c, uint32_t *buf, uint64_t count, cudaStream_t s);
 
 // Single query batch partitioned by vertex range (SURVEY §8(e) mode 2).  Every
 // partition p (one per rank with NCCL, or g->nparts logical partitions on one GPU)
@@ -704,7 +817,8 @@ tg_status tg_comm_allreduce_sum_u32(tg_comm *c, uint32_t *buf, uint64_t count, c
 // packed states are combined with a min-allreduce (NCCL) -- on one GPU the logical
 // partitions share one state array -- and each partition derives its next
 // frontier from the combined state (k_part_frontier).
-tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
+template <bool PK>
+static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                                  uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s) {
     const bool ld = (p == TG_LD);
     uint32_t alpha = w.t_alpha, omega = w.t_omega;
@@ -733,7 +847,7 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         const uint32_t Sb = std::min(S, k - b0);
         const uint32_t G = (Sb + 31) / 32;
         TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
-        TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, Sb * n * 8, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, Sb * n * (PK ? 8 : 4), s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, Sb * n * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.lat, 0xFF, Sb * n * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, Sb * Q.bit_words * 4, s));
@@ -741,10 +855,10 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
         if (g->opt_stats) {
-            TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8 + 8, s));
+            TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8 + 8 + 64, s));
             TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
         }
-        TG_LAUNCH(k_eat_init, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl, 0);
+        TG_LAUNCH(k_eat_init<PK>, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl, 0);
         const bool work = any_work && g->m > 0 && alpha < omega;
         uint32_t rounds = 0;
         if (work) {
@@ -755,6 +869,7 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
             base.fb0 = Q.fb[0]; base.fb1 = Q.fb[1]; base.recs = Q.recs; base.reccap = Q.reccap;
             base.bigq = Q.bigq; base.bigcap = Q.bigcap; base.chq = Q.chq; base.chcap = Q.chcap;
             base.relax_cnt = Q.relax_cnt;
+            base.diag = Q.relax_cnt + Sb + 1;
             EatP parts[TG_MAXP];
             uint64_t bit_off = 0;  // claim bits: each partition numbers its own slots from 0
             for (int pi = 0; pi < g->nparts; pi++) {
@@ -771,7 +886,7 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 parts[pi] = P;
                 TG_LAUNCH(k_ctl_reset, 1, 1, 0, s, Q.ctl + pi);
                 // round 1's frontier: the sources, derived from the state like every later one
-                TG_LAUNCH(k_part_frontier, grid, 256, 0, s, Q.st, Q.lat, Q.fb[1], Sb, G, g->part_vb[pi],
+                TG_LAUNCH(k_part_frontier<PK>, grid, 256, 0, s, Q.st, Q.lat, Q.fb[1], Sb, G, g->part_vb[pi],
                           g->part_vb[pi + 1], Q.pcount);
             }
             if (g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
@@ -785,18 +900,21 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 for (int pi = 0; pi < g->nparts; pi++) {
                     if (parts[pi].ub0 == parts[pi].ub1) {
                         // an empty range still has to advance its round counter in lockstep
-                        TG_LAUNCH(k_eat_chain, grid, QT, 0, s, parts[pi]);
+                        TG_LAUNCH(k_eat_chain<PK>, grid, QT, 0, s, parts[pi]);
                         continue;
                     }
-                    TG_LAUNCH(k_eat_activate, grid, QT, 0, s, parts[pi]);
-                    TG_LAUNCH(k_eat_big, grid, QT, 0, s, parts[pi]);
-                    TG_LAUNCH(k_eat_chain, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH(k_eat_activate<PK>, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH(k_eat_big<PK>, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH(k_eat_chain<PK>, grid, QT, 0, s, parts[pi]);
                 }
                 // exchange: every rank ends the round with the elementwise min of all ranks' states
-                if (g->comm) TG_TRY(tg_comm_allreduce_min_u64(g->comm, Q.st, (uint64_t)Sb * n, s));
+                if (g->comm) {
+                    if (PK) TG_TRY(tg_comm_allreduce_min_u64(g->comm, (unsigned long long *)Q.st, (uint64_t)Sb * n, s));
+                    else TG_TRY(tg_comm_allreduce_min_u32(g->comm, (uint32_t *)Q.st, (uint64_t)Sb * n, s));
+                }
                 uint32_t *fnext = ((r + 1) & 1) ? Q.fb[1] : Q.fb[0];
                 for (int pi = 0; pi < g->nparts; pi++)
-                    TG_LAUNCH(k_part_frontier, grid, 256, 0, s, Q.st, Q.lat, fnext, Sb, G, g->part_vb[pi],
+                    TG_LAUNCH(k_part_frontier<PK>, grid, 256, 0, s, Q.st, Q.lat, fnext, Sb, G, g->part_vb[pi],
                               g->part_vb[pi + 1], Q.pcount);
                 if (g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
                 r++;
@@ -808,7 +926,7 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
         uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
         const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
-        TG_LAUNCH(k_eat_extract, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
+        TG_LAUNCH(k_eat_extract<PK>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
                   (const uint32_t *)nullptr);
         if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
         if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
@@ -826,4 +944,12 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     g->last.kernel_launches = g_tg_launches - launches0;
     return TG_OK;
+}
+
+tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
+                                 uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s) {
+    // packed (arrival | pred) states only when the caller asked for preds (or forced)
+    if (pred != nullptr || g->opt_packed_state)
+        return eat_partitioned<true>(g, p, sources, k, w, out, pred, out_dev, pred_dev, s);
+    return eat_partitioned<false>(g, p, sources, k, w, out, pred, out_dev, pred_dev, s);
 }

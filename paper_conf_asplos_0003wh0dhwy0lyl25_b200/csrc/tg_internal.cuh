@@ -84,6 +84,10 @@ struct ChainGraph {
     unsigned long long *sc_sumw = nullptr;
     uint32_t *sc_elapsed = nullptr;
     uint32_t *chain_first = nullptr;
+    // time-ordered edge list (the sweep schedule's topological order of the expanded DAG):
+    // te int4[m] = {u, v, t, arrival} sorted by (t, input order), te_id[m] = edge id
+    int4 *te = nullptr;
+    uint32_t *te_id = nullptr;
 };
 
 // Device-side round control of one GAC loop (no host round trip per round):
@@ -105,7 +109,7 @@ struct QueryScratch {
     uint64_t nlong = 0;
     uint64_t nnodes = 0;
     bool nodes_state = false;  // SP/FP node-state arrays present
-    unsigned long long *st = nullptr;  // [S][n] packed (time << 32 | pred)
+    void *st = nullptr;  // [n][S] packed u64 (time << 32 | pred), or u32 time when no pred is requested
     uint32_t *act = nullptr;           // [S][n] last activated time
     uint32_t *mark = nullptr;          // [S][n] (EAT) or [S][nnodes] (SP/FP) frontier dedupe stamp
     uint32_t *bits = nullptr;          // [S][ceil(m/32)] "slot relaxed" bits (interior slots of long chains)
@@ -165,6 +169,7 @@ struct tg_graph {
     int comm_mode = 0;              // 0 replicated (source sharding), 1 vertex range
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
+    void *sweep = nullptr;  // query_sweep.cu scratch (SweepScratch)
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
     // options
     int64_t opt_sub_batch = 0;
@@ -173,6 +178,10 @@ struct tg_graph {
     int64_t opt_round_group = 4;
     int opt_mirror = 1;
     int64_t opt_exp = 0;
+    int64_t opt_packed_state = 0;
+    int64_t opt_sweep_struct = 0;  // build the time-ordered edge list (sweep schedule) in tg_build_chains
+    int64_t opt_engine = 0;        // EAT/LD/REACH schedule: 0 = automatic (GAC), 1 = GAC rounds, 2 = time sweep
+    int64_t opt_sweep_part = 0;    // sweep: edges per time partition (0 = automatic)  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
     int64_t opt_walk_min = 6;  // chains with fewer edges are not walked (RemoveChain threshold, build time)       // diagnostic kernel variants (timing experiments only)        // build the LD mirror in tg_build_chains (else on the first LD query)
     bool mirror_built = false;
     // last query statistics
@@ -192,6 +201,10 @@ tg_status tg_exclusive_scan_u32(const uint32_t *in, uint32_t *out, uint64_t coun
 // Stable LSD radix sort of (key, val) pairs on the low `key_bits` bits.
 tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
                               unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s);
+// ... and after the first snap_bits (multiple of 8) bits, a copy of the payload order to snap_vals.
+tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
+                                   unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s,
+                                   int snap_bits, uint32_t *snap_vals);
 
 tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
                              const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
@@ -202,6 +215,7 @@ tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cuda
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,
                              int dirs);  // dirs: bit 0 forward, bit 1 mirror
 
+tg_status tg_ensure_scratch_srcs(tg_graph *g, uint32_t S);  // sources + staging only
 tg_status tg_run_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                        uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
 

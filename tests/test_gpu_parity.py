@@ -375,3 +375,68 @@ def test_nccl_comm_world1_vertex_range(tg):
     _check_rows(tg, g, og, "ld", srcs, (0, 10**9))
     g.close()
     tg.tg_comm_destroy(comm)
+
+
+# --------------------------------------------------------------------------- state width / schedules
+def _check_values(tg, g, og, problem, sources, win):
+    """Values only (pred = NULL: the engines keep u32 arrival states, not packed words)."""
+    out = tg.as_u32(g.query(problem, sources, win))
+    for r, x in enumerate(sources):
+        if problem == "eat":
+            exp = oracle.eat(og, x, *win)[0]
+        elif problem == "ld":
+            exp = oracle.ld(og, x, *win)[0]
+        else:
+            exp = oracle.reach(og, x, *win)
+        np.testing.assert_array_equal(out[r], exp, err_msg=f"{problem} (no pred) x={x} win={win}")
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_unpacked_state_values(tg, seed):
+    """Without pred the EAT family runs on u32 arrival states; values equal the oracle
+    (the packed path is covered by every test that asks for preds)."""
+    n, u, v, t, lam, w = tgsynth.tiny_random(seed + 3100, n_max=80, m_max=1500, t_max=60, lam_max=6)
+    g = _gpu_graph(tg, n, u, v, t, lam, w, sub_batch=5)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    srcs = list(range(min(n, 17)))
+    for win in [(0, 10**6), (5, 40)]:
+        for p in ("eat", "ld", "reach"):
+            _check_values(tg, g, og, p, srcs, win)
+
+
+def test_unpacked_state_c2_small(tg):
+    ge = tgsynth.make_graph("C2", scale_shift=-4)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, w)
+    og = oracle.Graph(n, u, v, t, d, w)
+    srcs = tgsynth.config_sources("C2", ge)
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        _check_values(tg, g, og, "eat", srcs, win)
+        _check_values(tg, g, og, "ld", srcs[:16], win)
+
+
+@pytest.mark.parametrize("part", [3, 64, 0])
+def test_sweep_engine_random(tg, part):
+    """Time-partitioned sweep schedule (engine 2): values, preds (packed words) and the
+    post-hoc work count W equal the oracle; tiny partitions force many fixup rounds."""
+    for seed in range(6):
+        n, u, v, t, lam, w = tgsynth.tiny_random(seed + 4200, n_max=70, m_max=1200, t_max=50, lam_max=5)
+        g = _gpu_graph(tg, n, u, v, t, lam, w, sweep_struct=1, engine=2, sweep_part=part, stats=1)
+        og = oracle.Graph(n, u, v, t, lam, w)
+        srcs = list(range(min(n, 40)))
+        for win in [(0, 10**6), (4, 30), (7, 7)]:
+            for p in ("eat", "ld", "reach"):
+                _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
+                _check_values(tg, g, og, p, srcs, win)
+
+
+def test_sweep_engine_c2_small(tg):
+    ge = tgsynth.make_graph("C2", scale_shift=-4)
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d, w)
+    srcs = tgsynth.config_sources("C2", ge)
+    for part in (4096, 0):
+        g = _gpu_graph(tg, n, u, v, t, d, w, sweep_struct=1, engine=2, sweep_part=part)
+        for win in tgsynth.CONFIGS["C2"]["windows"]:
+            _check_values(tg, g, og, "eat", srcs, win)
+            _check_rows(tg, g, og, "ld", srcs[:8], win)

@@ -1,0 +1,9 @@
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+L=paper_conf_asplos_0003wh0dhwy0lyl25_b200/libtempgraph.so
+timeout 300 python tools/variant_bench.py $L C1 1 --check 2>&1 | grep -v Warn
+timeout 300 python tools/variant_bench.py $L C2 64 --opt=engine:1 2>&1 | grep -v Warn
+for part in 262144 1048576 4194304; do
+timeout 300 python tools/variant_bench.py $L C2 64 --check --opt=sweep_part:$part 2>&1 | grep -v Warn
+done
+timeout 300 python tools/variant_bench.py $L C2 64 --pred --opt=sweep_part:1048576 2>&1 | grep -v Warn
+TG_TRACE=1 timeout 300 python tools/prof_query.py --config C2 --problem eat --k 64 --reps 2 --relabel 0 --stats 1 2>&1 | grep -v Warn | tail -4

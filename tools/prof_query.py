@@ -24,6 +24,9 @@ ap.add_argument("--shortcuts", type=int, default=1)
 ap.add_argument("--exp", type=int, default=0)
 ap.add_argument("--walk-min", type=int, default=0)
 ap.add_argument("--relabel", type=int, default=1)
+ap.add_argument("--stats", type=int, default=0)
+ap.add_argument("--sweep-part", type=int, default=0)
+ap.add_argument("--engine", type=int, default=0)
 a = ap.parse_args()
 
 ge = tgsynth.make_graph(a.config, device="cuda")
@@ -38,6 +41,9 @@ if a.sub_batch:
     g.set_option("sub_batch", a.sub_batch)
 g.set_option("shortcuts", a.shortcuts)
 g.set_option("exp", a.exp)
+g.set_option("stats", a.stats)
+g.set_option("sweep_part", a.sweep_part)
+g.set_option("engine", a.engine)
 src = tgsynth.config_sources(a.config, ge, k=a.k)
 win = cfg["windows"][0]
 out = torch.empty((len(src), ge.n), dtype=torch.int32, device="cuda")
