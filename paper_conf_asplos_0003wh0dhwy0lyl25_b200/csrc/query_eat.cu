@@ -242,14 +242,9 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
             s = __ldg(P.occ_slot + p);
             sl = tg_ld_slot(P.slots + s);
         }
-        // mask of queries for which edge pb+k is newly usable (lane k keeps its own)
-        uint32_t mask = 0;
-#pragma unroll 8
-        for (int k = 0; k < 32; k++) {
-            const uint32_t pk = pb + k;
-            const uint32_t m = __ballot_sync(0xffffffffu, lo <= pk && pk < hi);
-            if (lane == k) mask = m;
-        }
+        // mask of queries for which edge pb+k is newly usable (lane k keeps its own):
+        // each query lane's range as a row of block bits, transposed across the warp
+        uint32_t mask = tg_warp_transpose32(lo < hi ? tg_block_bits(lo, hi, pb) : 0u);
         if (p >= pend || (uint32_t)sl.y > P.omega) mask = 0;  // past the window end: never usable
         const uint32_t cnt = __popc(mask);
         uint32_t incl = cnt;

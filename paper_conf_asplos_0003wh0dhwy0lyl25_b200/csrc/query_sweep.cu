@@ -280,12 +280,7 @@ __device__ __forceinline__ void fix_chunk(const SwP &P, uint32_t g, uint32_t lo,
         const uint32_t p = pb + lane;
         int4 sl = make_int4(0, -1, 0, 0);
         if (p < pend) sl = __ldg(P.slots + __ldg(P.occ_slot + p));
-        uint32_t mask = 0;
-#pragma unroll 8
-        for (int k = 0; k < 32; k++) {
-            const uint32_t m = __ballot_sync(0xffffffffu, lo <= pb + k && pb + k < hi);
-            if (lane == k) mask = m;
-        }
+        uint32_t mask = tg_warp_transpose32(lo < hi ? tg_block_bits(lo, hi, pb) : 0u);
         if (p >= pend || (uint32_t)sl.y > P.omega) mask = 0;
         const uint32_t cnt = __popc(mask);
         uint32_t incl = cnt;

@@ -236,6 +236,28 @@ __device__ __forceinline__ int4 tg_ld_slot(const int4 *p) {
     return r;
 }
 
+// Bits [a, b) of the 32-edge block starting at pb covered by the edge range [lo, hi).
+__device__ __forceinline__ uint32_t tg_block_bits(uint32_t lo, uint32_t hi, uint32_t pb) {
+    const uint32_t a = lo <= pb ? 0u : min(lo - pb, 32u);
+    const uint32_t b = hi <= pb ? 0u : min(hi - pb, 32u);
+    return (uint32_t)(((1ull << b) - 1ull) & ~((1ull << a) - 1ull));
+}
+
+// 32 x 32 bit-matrix transpose across a warp: on entry lane L holds row L (bit k =
+// element (L, k)); on exit lane L holds column L (bit q = element (q, L)).  Five
+// butterfly stages swap the off-diagonal j x j blocks (j = 16, 8, 4, 2, 1).
+__device__ __forceinline__ uint32_t tg_warp_transpose32(uint32_t x) {
+    const uint32_t lane = threadIdx.x & 31;
+#pragma unroll
+    for (int j = 16, i = 0; j; j >>= 1, i++) {
+        constexpr uint32_t M[5] = {0x0000FFFFu, 0x00FF00FFu, 0x0F0F0F0Fu, 0x33333333u, 0x55555555u};
+        const uint32_t m = M[i];
+        const uint32_t y = __shfl_xor_sync(0xffffffffu, x, j);
+        x = (lane & j) ? ((x & ~m) | ((y & ~m) >> j)) : ((x & m) | ((y & m) << j));
+    }
+    return x;
+}
+
 static inline uint32_t tg_grid_persistent(int blocks_per_sm = 8) {
     return 148u * (uint32_t)blocks_per_sm;
 }

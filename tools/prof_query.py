@@ -27,6 +27,7 @@ ap.add_argument("--relabel", type=int, default=1)
 ap.add_argument("--stats", type=int, default=0)
 ap.add_argument("--sweep-part", type=int, default=0)
 ap.add_argument("--engine", type=int, default=0)
+ap.add_argument("--sweep-struct", type=int, default=0)
 a = ap.parse_args()
 
 ge = tgsynth.make_graph(a.config, device="cuda")
@@ -34,6 +35,7 @@ cfg = tgsynth.CONFIGS[a.config]
 w = ge.w if cfg["kind"] == "wikitalk" else None
 g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, w, device=0)
 g.set_option("relabel", a.relabel)
+g.set_option("sweep_struct", a.sweep_struct or int(a.engine == 2))
 if a.walk_min:
     g.set_option("walk_min", a.walk_min)
 g.build()
