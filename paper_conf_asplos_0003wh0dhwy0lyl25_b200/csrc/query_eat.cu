@@ -50,6 +50,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_MLP
 #define TG_MLP 4                        // state reads in flight per lane in the pair loop
 #endif
+#ifndef TG_COOP_SEARCH
+#define TG_COOP_SEARCH 1                // warp-cooperative departure-time search in the activation
+#endif
 #ifndef TG_ACT_MINB
 #define TG_ACT_MINB 8                   // resident blocks per SM requested for the relax kernels
 #endif
@@ -159,12 +162,14 @@ __device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, ui
     const typename W::T pk = W::make(arr, id);
     if (cur <= pk) return;
     const size_t i = (size_t)v * P.S + q;
-    const typename W::T old = atomicMin((typename W::T *)P.st + i, pk);
-    if (arr < W::time(old)) {
-        // arrival improved: v joins the next round's frontier (bitmap: duplicates merge;
-        // no shared counter -- the next activation counts the non-empty words it finds)
-        atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
-    }
+    // fire-and-forget min (RED): nobody waits on the old value.  The frontier bit is set
+    // whenever the (possibly stale) read says the arrival improves: if a concurrent
+    // relaxation of this round got there first, that relaxation improved the arrival in
+    // this round too and sets the same bit, so the frontier is exactly the set of
+    // vertices whose arrival dropped this round (bitmap: duplicates merge; no shared
+    // counter -- the next activation counts the non-empty words it finds).
+    atomicMin((typename W::T *)P.st + i, pk);
+    if (arr < W::time(cur)) atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
 }
 
 template <bool PK>
@@ -313,9 +318,6 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
     __shared__ WarpStage stage[QT / 32];
     WarpStage &ws = stage[threadIdx.x >> 5];
-    __shared__ uint32_t s_units;
-    if (threadIdx.x == 0) s_units = 0;
-    __syncthreads();
     uint32_t my_units = 0;
     const uint32_t NU = P.ub1;
     const int lane = threadIdx.x & 31;
@@ -336,21 +338,39 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
             const uint32_t g = unit - v * P.G;
             const uint32_t q = g * 32 + lane;
             uint32_t lo = 0, hi = 0;
-            if ((qm >> lane) & 1u) {
-                const size_t si = (size_t)v * P.S + q;
-                const uint32_t now = StW<PK>::time(__ldcg((const typename StW<PK>::T *)P.st + si));
-                const uint32_t a = __ldg(P.vnode_off + v), b = __ldg(P.vnode_off + v + 1);
-                const uint32_t j0 = tg_lower_bound(P.node_t, a, b, max(now, P.alpha));
-                const uint32_t elo = __ldg(P.node_eoff + j0);
-                // edges at index >= the boundary were activated before; the first
-                // activation starts from the window end (t + duration <= omega needs t < omega)
-                const uint32_t prev = atomicMin(P.act + si, elo);
-                if (elo < prev) {
-                    uint32_t ehi = prev;
-                    if (prev == TG_NONE) ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, j0, b, P.omega));
-                    if (elo < ehi) { lo = elo; hi = ehi; }
-                }
+            const bool on = (qm >> lane) & 1u;
+            const size_t si = (size_t)v * P.S + q;
+            // (v, q) is activated by this warp alone in this round (its frontier word is
+            // consumed once), so the boundary needs no atomic: plain load, issued with the
+            // state load, and a plain store
+            uint32_t prev = 0, now = 0;
+            if (on) {
+                prev = __ldcg(P.act + si);
+                now = StW<PK>::time(__ldcg((const typename StW<PK>::T *)P.st + si));
             }
+            const uint32_t a = __ldg(P.vnode_off + v), b = __ldg(P.vnode_off + v + 1);
+#if TG_COOP_SEARCH
+            // all lanes search the same vertex's departure times: warp-cooperative
+            const uint32_t j0 = tg_warp_lower_bound(P.node_t, a, b, max(now, P.alpha));
+#else
+            const uint32_t j0 = on ? tg_lower_bound(P.node_t, a, b, max(now, P.alpha)) : a;
+#endif
+            uint32_t elo = 0;
+            if (on) {
+                elo = __ldg(P.node_eoff + j0);
+                // edges at index >= the boundary were activated before
+                if (elo < prev) { P.act[si] = elo; lo = elo; hi = prev; }
+            }
+            // a first activation starts from the window end (t + duration <= omega needs t < omega)
+            if (__any_sync(0xffffffffu, hi == TG_NONE)) {
+#if TG_COOP_SEARCH
+                const uint32_t ehi = __ldg(P.node_eoff + tg_warp_lower_bound(P.node_t, a, b, P.omega));
+#else
+                const uint32_t ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, a, b, P.omega));
+#endif
+                if (hi == TG_NONE) hi = ehi;
+            }
+            if (lo >= hi) { lo = 0; hi = 0; }
             if (P.stats && lane == 0) {
                 atomicAdd(P.diag + 3, (unsigned long long)__popc(__ballot_sync(0xffffffffu, lo < hi)));
                 atomicAdd(P.diag + 4, (unsigned long long)__popc(qm));
@@ -392,9 +412,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
             unit_range<PK>(P, R, g, lo, hi, ulo, uhi, ws);
         }
     }
-    if (lane == 0 && my_units) atomicAdd(&s_units, my_units);
-    __syncthreads();
-    if (threadIdx.x == 0 && s_units) atomicAdd(R.words_cnt, s_units);
+    if (lane == 0 && my_units) atomicAdd(R.words_cnt, my_units);  // per warp: no block barrier
 }
 
 // Chunks of long unions: one warp per chunk, the unit's 32 query ranges from its record.

@@ -236,6 +236,31 @@ __device__ __forceinline__ int4 tg_ld_slot(const int4 *p) {
     return r;
 }
 
+// Lower bound of `key` (first index with a[i] >= key) in the sorted a[lo, hi), for
+// every lane of a warp searching the SAME range with its own key (all lanes call).
+// Up to 32 elements: one coalesced load, then a branchless search over registers by
+// shuffles.  Longer ranges: 32 evenly spaced samples locate a bucket of < stride
+// elements, searched per lane (its lines are shared by the warp, so mostly L1 hits).
+__device__ __forceinline__ uint32_t tg_warp_lower_bound(const uint32_t *__restrict__ a, uint32_t lo, uint32_t hi,
+                                                        uint32_t key) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t n = hi - lo;
+    const uint32_t stride = n <= 32 ? 1u : (n + 31) / 32;
+    const uint32_t idx = lane * stride;
+    const uint32_t x = idx < n ? __ldg(a + lo + idx) : 0xFFFFFFFFu;
+    uint32_t c = 0;  // samples < key (the samples are sorted; padding is above every key)
+#pragma unroll
+    for (uint32_t st = 16; st; st >>= 1) {
+        const uint32_t y = __shfl_sync(0xffffffffu, x, c + st - 1);
+        if (y < key) c += st;
+    }
+    if (__shfl_sync(0xffffffffu, x, c & 31) < key && c == 31) c = 32;
+    if (stride == 1) return lo + min(c, n);
+    const uint32_t blo = c == 0 ? lo : lo + (c - 1) * stride + 1;
+    const uint32_t bhi = min(hi, lo + c * stride);
+    return tg_lower_bound(a, blo, bhi, key);
+}
+
 // Bits [a, b) of the 32-edge block starting at pb covered by the edge range [lo, hi).
 __device__ __forceinline__ uint32_t tg_block_bits(uint32_t lo, uint32_t hi, uint32_t pb) {
     const uint32_t a = lo <= pb ? 0u : min(lo - pb, 32u);
