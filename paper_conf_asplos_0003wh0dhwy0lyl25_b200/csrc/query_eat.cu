@@ -54,7 +54,7 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #define TG_COOP_SEARCH 1                // warp-cooperative departure-time search in the activation
 #endif
 #ifndef TG_ACT_MINB
-#define TG_ACT_MINB 8                   // resident blocks per SM requested for the relax kernels
+#define TG_ACT_MINB 6                   // resident blocks per SM requested for the relax kernels (8, 7, 5, 4 measured slower)
 #endif
 
 struct EatP {
