@@ -35,6 +35,7 @@ cudaEvent_t tg_prof_begin(cudaStream_t s) {
 void tg_prof_end(const char *name, cudaStream_t s, cudaEvent_t ev0) {
     cudaEvent_t e = ev_get();
     cudaEventRecord(e, s);
+    if (name[0] == '(') name++;  // TG_LAUNCH((k<A, B>), ...): parenthesised template launches
     g_prof.push_back({name, ev0, e});
 }
 
@@ -219,8 +220,10 @@ int tg_profile_report(char *buf, uint64_t buf_len) {
         cudaEventSynchronize(r.e1);
         float ms = 0;
         cudaEventElapsedTime(&ms, r.e0, r.e1);
-        auto it = std::find_if(acc.begin(), acc.end(), [&](const Acc &p) { return p.name == r.name; });
-        if (it == acc.end()) { acc.push_back(Acc{r.name}); it = acc.end() - 1; }
+        std::string nm(r.name);
+        if (!nm.empty() && nm.back() == ')') nm.pop_back();  // "(k<A, B>)" launches
+        auto it = std::find_if(acc.begin(), acc.end(), [&](const Acc &p) { return p.name == nm; });
+        if (it == acc.end()) { acc.push_back(Acc{nm}); it = acc.end() - 1; }
         it->n++;
         it->ms += ms;
         g_ev_pool.push_back(r.e0);
