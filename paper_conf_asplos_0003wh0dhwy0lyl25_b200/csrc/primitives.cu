@@ -9,6 +9,10 @@
 
 namespace {
 
+#ifndef TG_RS_V2
+#define TG_RS_V2 1  // radix scatter with warp-private ranking
+#endif
+
 constexpr int SCAN_THREADS = 256;
 constexpr int SCAN_ITEMS = 8;
 constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
@@ -211,6 +215,108 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const unsigned lon
     }
 }
 
+#if TG_RS_V2
+// Stable scatter of one tile with warp-private ranking: warp w owns the contiguous
+// keys [w * 512, w * 512 + 512) of the tile (16 rounds of 32 coalesced keys); a key's
+// rank among equal digits of its warp is its peers below it in the round
+// (__match_any_sync) plus the warp's running count of that digit, which only warp w
+// touches -- no block barrier inside the ranking.  Then one block-level pass turns the
+// per-warp digit counts into tile positions ((warp, round, lane) = index order, so
+// the scatter is stable), the tile is staged in shared memory grouped by digit and
+// written out so that consecutive threads write consecutive global positions.
+constexpr size_t RS2_SMEM = (size_t)RS_TILE * (8 + 4) + RS_WARPS * 256 * 4 + 256 * 4 * 2 + 32 * 4;
+
+__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter2(const unsigned long long *__restrict__ kin,
+                                                               const uint32_t *__restrict__ vin,
+                                                               unsigned long long *__restrict__ kout,
+                                                               uint32_t *__restrict__ vout, uint64_t m, int shift,
+                                                               const uint32_t *__restrict__ offs, uint32_t ntiles) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    unsigned long long *skey = (unsigned long long *)smem;
+    uint32_t *sval = (uint32_t *)(skey + RS_TILE);
+    uint32_t *wcnt = sval + RS_TILE;                 // [RS_WARPS][256]
+    uint32_t *tstart = wcnt + RS_WARPS * 256;        // [256]
+    uint32_t *gofs = tstart + 256;                   // [256]
+    uint32_t *wsum = gofs + 256;                     // [32]
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t lt_mask = (1u << lane) - 1u;
+    const uint64_t base = (uint64_t)blockIdx.x * RS_TILE;
+    constexpr int PER_WARP = RS_TILE / RS_WARPS;
+
+    gofs[tid] = offs[(uint64_t)tid * ntiles + blockIdx.x];
+#pragma unroll
+    for (int w = 0; w < RS_WARPS; w++) wcnt[w * 256 + tid] = 0;
+    __syncthreads();
+
+    uint32_t *mycnt = wcnt + warp * 256;
+    unsigned long long kk[RS_ITEMS];
+    uint32_t vv[RS_ITEMS], lr[RS_ITEMS];
+    const uint64_t wbase = base + (uint64_t)warp * PER_WARP;
+#pragma unroll
+    for (int r = 0; r < RS_ITEMS; r++) {
+        const uint64_t idx = wbase + (uint64_t)r * 32 + lane;
+        const bool valid = idx < m;
+        kk[r] = valid ? kin[idx] : ~0ull;
+        vv[r] = valid ? vin[idx] : 0u;
+    }
+#pragma unroll
+    for (int r = 0; r < RS_ITEMS; r++) {
+        const uint64_t idx = wbase + (uint64_t)r * 32 + lane;
+        const bool valid = idx < m;
+        const uint32_t d = valid ? ((uint32_t)(kk[r] >> shift) & 255u) : 0x100u;
+        const uint32_t peers = __match_any_sync(0xffffffffu, d);
+        const uint32_t below = __popc(peers & lt_mask);
+        const uint32_t c = valid ? mycnt[d] : 0u;
+        __syncwarp();
+        if (valid && below == 0) mycnt[d] = c + __popc(peers);
+        __syncwarp();
+        lr[r] = c + below;
+    }
+    __syncthreads();
+    // thread tid owns digit tid: per-warp exclusive prefixes and the tile total
+    uint32_t tot = 0;
+#pragma unroll
+    for (int w = 0; w < RS_WARPS; w++) {
+        const uint32_t c = wcnt[w * 256 + tid];
+        wcnt[w * 256 + tid] = tot;
+        tot += c;
+    }
+    // exclusive scan of the digit totals -> tile-local digit starts
+    uint32_t x = tot;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[warp] = x;
+    __syncthreads();
+    uint32_t wp = 0;
+#pragma unroll
+    for (int w = 0; w < RS_WARPS; w++) wp += (w < warp) ? wsum[w] : 0u;
+    tstart[tid] = wp + x - tot;
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < RS_ITEMS; r++) {
+        const uint64_t idx = wbase + (uint64_t)r * 32 + lane;
+        if (idx < m) {
+            const uint32_t d = (uint32_t)(kk[r] >> shift) & 255u;
+            const uint32_t p = tstart[d] + mycnt[d] + lr[r];
+            skey[p] = kk[r];
+            sval[p] = vv[r];
+        }
+    }
+    __syncthreads();
+    const uint32_t nvalid = (uint32_t)min((uint64_t)RS_TILE, m - base);
+    for (uint32_t i = tid; i < nvalid; i += RS_THREADS) {
+        const unsigned long long k = skey[i];
+        const uint32_t d = (uint32_t)(k >> shift) & 255u;
+        const uint32_t pos = gofs[d] + (i - tstart[d]);
+        kout[pos] = k;
+        vout[pos] = sval[i];
+    }
+}
+#endif
+
 }  // namespace
 
 tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
@@ -239,14 +345,23 @@ tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uin
     TG_TRY_CUDA(tg_malloc_async((void **)&k2, m * 8, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&v2, m * 4, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&counts, ntiles * 256 * 4, s));
+#if TG_RS_V2
+    TG_TRY_CUDA(cudaFuncSetAttribute(k_radix_scatter2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)RS2_SMEM));
+#else
     TG_TRY_CUDA(cudaFuncSetAttribute(k_radix_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)RS_SMEM));
+#endif
     unsigned long long *ka = keys, *kb = k2;
     uint32_t *va = vals, *vb = v2;
     for (int shift = 0; shift < key_bits; shift += 8) {
         TG_LAUNCH(k_radix_hist, (unsigned)ntiles, RS_THREADS, 0, s, ka, m, shift, counts, (uint32_t)ntiles);
         TG_TRY(tg_exclusive_scan_u32(counts, counts, ntiles * 256, nullptr, s, nullptr));
+#if TG_RS_V2
+        TG_LAUNCH(k_radix_scatter2, (unsigned)ntiles, RS_THREADS, RS2_SMEM, s, ka, va, kb, vb, m, shift, counts,
+                  (uint32_t)ntiles);
+#else
         TG_LAUNCH(k_radix_scatter, (unsigned)ntiles, RS_THREADS, RS_SMEM, s, ka, va, kb, vb, m, shift, counts,
                   (uint32_t)ntiles);
+#endif
         std::swap(ka, kb);
         std::swap(va, vb);
         if (snap_vals && snap_bits > 0 && shift + 8 == snap_bits)
