@@ -72,6 +72,7 @@ struct EatP {
     int use_sc, stats, exp;
   // exp: diagnostic variants for timing only (results invalid when != 0)
     RoundCtl *ctl;
+    uint32_t round;       // GAC round of this launch (host loop counter; parity picks the bitmaps)
     uint32_t *fb0, *fb1;  // frontier masks [n][G] (bit = query within the group), by round parity
     uint2 *recs;          // big-unit records: 32 per-query ranges each
     uint64_t reccap;
@@ -94,7 +95,7 @@ struct RoundV {
 
 __device__ __forceinline__ RoundV round_view(const EatP &P) {
     RoundV R;
-    const uint32_t r = *(volatile uint32_t *)&P.ctl->round;
+    const uint32_t r = P.round;
     R.fin = (r & 1) ? P.fb1 : P.fb0;
     R.fout = (r & 1) ? P.fb0 : P.fb1;
     R.fin_n = 0;
@@ -105,23 +106,11 @@ __device__ __forceinline__ RoundV round_view(const EatP &P) {
     return R;
 }
 
-// The last block to finish the round's last kernel advances the round.
-__device__ __forceinline__ void round_advance(RoundCtl *ctl) {
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        const uint32_t d = atomicAdd(&ctl->done_blocks, 1u);
-        if (d == gridDim.x - 1) {
-            const uint32_t r = ctl->round;
-            for (int i = 0; i < 4; i++) ctl->cnt[(r + 2) & 3][i] = 0;
-            ctl->cnt[(r + 1) & 3][1] = 0;
-            ctl->cnt[(r + 1) & 3][2] = 0;
-            ctl->done_blocks = 0;
-            ctl->stamp = ctl->stamp + 1;
-            ctl->round = r + 1;
-            __threadfence();
-        }
-    }
+// Round r's counters were cleared during round r - 1: the first kernel of a round
+// clears the next round's (nobody touches them before that round; the host reads
+// only the last round of a group, which is cleared again three rounds later).
+__device__ __forceinline__ void clear_next_round(const EatP &P) {
+    if (blockIdx.x == 0 && threadIdx.x < 4) P.ctl->cnt[(P.round + 1) & 3][threadIdx.x] = 0;
 }
 
 // Layouts interleave the S queries of a sub-batch (query index fastest):
@@ -316,6 +305,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
 template <bool PK>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
+    clear_next_round(P);
     __shared__ WarpStage stage[QT / 32];
     WarpStage &ws = stage[threadIdx.x >> 5];
     uint32_t my_units = 0;
@@ -434,7 +424,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_big(EatP P) {
 
 // ChainEngine: warp per queued walk, lanes over consecutive slots; the warp
 // continues iff its last lane claimed its slot (otherwise that slot's claimer
-// continues the chain).  Advances the round when the last block finishes.
+// continues the chain).
 template <bool PK>
 __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
     const RoundV R = round_view(P);
@@ -461,7 +451,6 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
             if (__any_sync(0xffffffffu, past) || !go_on) break;
         }
     }
-    round_advance(P.ctl);
 }
 
 // VInitial (Table 1): every state INF (memset), the source = (alpha, no pred),
@@ -730,23 +719,38 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;
         const int group = trace ? 1 : (int)std::max<int64_t>(1, g->opt_round_group);
+        cudaEvent_t tev[4] = {};
+        if (trace)
+            for (auto &e : tev) cudaEventCreate(&e);
+        uint32_t r = 1;  // round 1's frontier: the sources (k_eat_init)
         for (;;) {
-            for (int k = 0; k < group; k++) {
+            for (int k = 0; k < group; k++, r++) {
+                P.round = r;
+                if (trace) cudaEventRecord(tev[0], s);
                 TG_LAUNCH(k_eat_activate<PK>, grid, QT, 0, s, P);
+                if (trace) cudaEventRecord(tev[1], s);
                 TG_LAUNCH(k_eat_big<PK>, grid, QT, 0, s, P);
-                TG_LAUNCH(k_eat_chain<PK>, grid, QT, 0, s, P);
+                if (trace) cudaEventRecord(tev[2], s);
+                TG_LAUNCH(k_eat_chain<PK>, 148, QT, 0, s, P);  // at most a few hundred walks per round
+                if (trace) cudaEventRecord(tev[3], s);
             }
             TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
             const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
-            const uint32_t last = h->round - 1;  // the round just finished
-            if (trace)
-                fprintf(stderr, "[tg] S=%u round %u: frontier words %u big-chunks %u chain-walks %u\n", S, last,
-                        h->cnt[last & 3][3], h->cnt[last & 3][1], h->cnt[last & 3][2]);
+            const uint32_t last = r - 1;  // the round just finished
+            if (trace) {
+                float ms[3] = {0, 0, 0};
+                for (int i = 0; i < 3; i++) cudaEventElapsedTime(&ms[i], tev[i], tev[i + 1]);
+                fprintf(stderr, "[tg] S=%u round %u: frontier words %u big-chunks %u chain-walks %u | activate %.3f "
+                        "big %.3f chain %.3f ms\n", S, last, h->cnt[last & 3][3], h->cnt[last & 3][1],
+                        h->cnt[last & 3][2], ms[0], ms[1], ms[2]);
+            }
             // a round whose frontier bitmap was empty ends the loop (it did no work)
             if (h->cnt[last & 3][3] == 0) { rounds = last - 1; break; }
-            if (h->round > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
+            if (r > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
         }
+        if (trace)
+            for (auto &e : tev) cudaEventDestroy(e);
     }
     *rounds_out = rounds;
     return TG_OK;
@@ -911,14 +915,11 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 if (r > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
                 TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
                 for (int pi = 0; pi < g->nparts; pi++) {
-                    if (parts[pi].ub0 == parts[pi].ub1) {
-                        // an empty range still has to advance its round counter in lockstep
-                        TG_LAUNCH(k_eat_chain<PK>, grid, QT, 0, s, parts[pi]);
-                        continue;
-                    }
+                    if (parts[pi].ub0 == parts[pi].ub1) continue;  // no vertices: never any work
+                    parts[pi].round = r;
                     TG_LAUNCH(k_eat_activate<PK>, grid, QT, 0, s, parts[pi]);
                     TG_LAUNCH(k_eat_big<PK>, grid, QT, 0, s, parts[pi]);
-                    TG_LAUNCH(k_eat_chain<PK>, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH(k_eat_chain<PK>, 148, QT, 0, s, parts[pi]);
                 }
                 // exchange: every rank ends the round with the elementwise min of all ranks' states
                 if (g->comm) {
