@@ -520,6 +520,49 @@ __global__ void __launch_bounds__(256) k_eat_extract(const void *__restrict__ st
     }
 }
 
+// Fast path of the extract for the bench configuration (u32 states, 64 queries, no
+// relabelling): a tile of 64 vertices x 64 queries is one contiguous 16 KB run of the
+// state, read with 16-byte loads, transposed in shared memory and written as 256-byte
+// row segments.
+__global__ void __launch_bounds__(256) k_eat_extract64(const uint32_t *__restrict__ st, uint32_t n,
+                                                       const uint32_t *__restrict__ srcs, int mode, uint32_t C,
+                                                       uint32_t omega, uint32_t *__restrict__ out) {
+    __shared__ uint32_t tile[64][65];
+    const uint32_t nt = (n + 63) / 64;
+    for (uint32_t tb = blockIdx.x; tb < nt; tb += gridDim.x) {
+        const uint32_t v0 = tb * 64;
+        const uint32_t nv = min(64u, n - v0);
+        __syncthreads();
+        const uint4 *src = (const uint4 *)(st + (size_t)v0 * 64);
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint32_t j = threadIdx.x + k * 256;  // uint4 index in the tile
+            const uint32_t dv = j >> 4, dq = (j & 15) * 4;
+            if (dv < nv) {
+                const uint4 x = __ldcs(src + j);
+                tile[dq][dv] = x.x;
+                tile[dq + 1][dv] = x.y;
+                tile[dq + 2][dv] = x.z;
+                tile[dq + 3][dv] = x.w;
+            }
+        }
+        __syncthreads();
+#pragma unroll 4
+        for (uint32_t i = threadIdx.x; i < 64 * 64; i += 256) {
+            const uint32_t dq = i >> 6, dv = i & 63;
+            if (dv >= nv) continue;
+            const uint32_t v = v0 + dv;
+            const uint32_t t = tile[dq][dv];
+            const bool reached = t != 0xFFFFFFFFu;
+            uint32_t val;
+            if (mode == 0) val = t;  // INF is TG_UNREACHED
+            else if (mode == 1) val = (v == __ldg(srcs + dq)) ? omega : (reached ? C - t : TG_UNREACHED);
+            else val = reached ? 1u : 0u;
+            __stcs(out + (size_t)dq * n + v, val);
+        }
+    }
+}
+
 // Vertex-range partitions: after the state exchange, each partition derives the
 // next frontier of ITS vertices from the state itself (bits set by relaxations are
 // discarded): (v, q) is active iff its arrival dropped below the last activated one.
@@ -798,6 +841,9 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         if (pk)
             TG_LAUNCH(k_eat_extract<true>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
                       g->relabeled ? g->perm : (const uint32_t *)nullptr);
+        else if (Sb == 64 && !g->relabeled)
+            TG_LAUNCH(k_eat_extract64, (unsigned)std::min<uint64_t>((n + 63) / 64, 148ull * 8), 256, 0, s,
+                      (const uint32_t *)Q.st, g->n, Q.srcs, mode, C, w.t_omega, o);
         else
             TG_LAUNCH(k_eat_extract<false>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
                       g->relabeled ? g->perm : (const uint32_t *)nullptr);
