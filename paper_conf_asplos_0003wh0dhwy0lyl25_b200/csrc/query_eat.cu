@@ -150,6 +150,7 @@ __device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, ui
     }
     const typename W::T pk = W::make(arr, id);
     if (cur <= pk) return;
+    if (P.stats) atomicAdd(P.diag + 5, 1ull);  // relaxations past the filter read
     const size_t i = (size_t)v * P.S + q;
     // fire-and-forget min (RED): nobody waits on the old value.  The frontier bit is set
     // whenever the (possibly stale) read says the arrival improves: if a concurrent
@@ -861,7 +862,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
             static const bool trace = getenv("TG_TRACE") != nullptr;
             if (trace)
                 fprintf(stderr, "[tg] diag S=%u: union edges %llu, unit ranges %llu, pairs %llu, activations %llu, "
-                        "frontier bits %llu\n", Sb, h[Sb + 1], h[Sb + 2], h[Sb + 3], h[Sb + 4], h[Sb + 5]);
+                        "frontier bits %llu, past filter %llu\n", Sb, h[Sb + 1], h[Sb + 2], h[Sb + 3], h[Sb + 4],
+                        h[Sb + 5], h[Sb + 6]);
         }
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
