@@ -50,6 +50,7 @@ struct SpP {
     uint32_t alpha, omega;
     int use_sc;
     RoundCtl *ctl;
+    uint32_t round, stamp;  // round of this launch and its dedupe stamp (host counters)
     unsigned long long *fr0, *fr1;
     uint4 *bigq;
     uint64_t bigcap;
@@ -67,8 +68,8 @@ struct RoundV {
 
 __device__ __forceinline__ RoundV round_view(const SpP &P) {
     RoundV R;
-    const uint32_t r = *(volatile uint32_t *)&P.ctl->round;
-    R.stamp = *(volatile uint32_t *)&P.ctl->stamp;
+    const uint32_t r = P.round;
+    R.stamp = P.stamp;
     R.fin = (r & 1) ? P.fr1 : P.fr0;
     R.fout = (r & 1) ? P.fr0 : P.fr1;
     R.fin_n = *(volatile uint32_t *)&P.ctl->cnt[r & 3][0];
@@ -78,22 +79,15 @@ __device__ __forceinline__ RoundV round_view(const SpP &P) {
     return R;
 }
 
-__device__ __forceinline__ void round_advance(RoundCtl *ctl) {
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        const uint32_t d = atomicAdd(&ctl->done_blocks, 1u);
-        if (d == gridDim.x - 1) {
-            const uint32_t r = ctl->round;
-            for (int i = 0; i < 4; i++) ctl->cnt[(r + 2) & 3][i] = 0;
-            ctl->cnt[(r + 1) & 3][1] = 0;
-            ctl->cnt[(r + 1) & 3][2] = 0;
-            ctl->done_blocks = 0;
-            ctl->stamp = ctl->stamp + 1;
-            ctl->round = r + 1;
-            __threadfence();
-        }
-    }
+// Counters of later rounds, cleared by the first kernel of round r: round r+2's
+// (its input count is written during round r+1) and round r+1's work-queue counts.
+// The host reads round r+1's input count after round r; it is cleared again only in
+// round r+3.
+__device__ __forceinline__ void clear_later_rounds(const SpP &P) {
+    if (blockIdx.x != 0) return;
+    const uint32_t r = P.round;
+    if (threadIdx.x < 4) P.ctl->cnt[(r + 2) & 3][threadIdx.x] = 0;
+    else if (threadIdx.x < 6) P.ctl->cnt[(r + 1) & 3][threadIdx.x - 3] = 0;
 }
 
 __device__ __forceinline__ void push_node(const SpP &P, const RoundV &R, uint32_t q, uint32_t j) {
@@ -175,6 +169,7 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_
 template <bool FP>
 __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
     const RoundV R = round_view(P);
+    clear_later_rounds(P);
     const uint32_t F = R.fin_n;
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -303,7 +298,6 @@ __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
         const uint4 c = P.bigq[it];
         for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<FP>(P, R, c.x, p);
     }
-    round_advance(P.ctl);
 }
 
 // VInitial: the source's departure nodes tau >= alpha get 0 (SP) / LS = tau (FP).
@@ -311,14 +305,6 @@ __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
 __global__ void k_spfp_ctl_init(RoundCtl *ctl) {
     for (int i = 0; i < 4; i++)
         for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
-    ctl->round = 0;  // k_spfp_init pushes with round 0's view: output buffer 1, count cnt[1][0]
-    ctl->done_blocks = 0;
-    ctl->stamp = ctl->stamp + 1;
-}
-
-__global__ void k_spfp_ctl_start(RoundCtl *ctl) {
-    ctl->round = 1;
-    ctl->stamp = ctl->stamp + 1;
 }
 
 template <bool FP>
@@ -368,16 +354,22 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     P.bigq = Q.bigq; P.bigcap = Q.bigcap;
     P.waitq = Q.chq; P.waitcap = Q.chcap;
     TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl);
+    // rounds and dedupe stamps are host counters passed with each launch; stamps only
+    // grow (marks of earlier rounds and loops never match)
     {
+        P.round = 0;  // k_spfp_init pushes with round 0's view: output buffer 1, count cnt[1][0]
+        P.stamp = ++Q.stamp;
         dim3 grid(64, Sb);  // a hub source has many departure nodes
         TG_LAUNCH(k_spfp_init<FP>, grid, 256, 0, s, P, Q.srcs_int, Sb);
     }
-    TG_LAUNCH(k_spfp_ctl_start, 1, 1, 0, s, Q.ctl);
     const uint32_t grid = tg_grid_persistent(8);
     const int group = (int)std::max<int64_t>(1, g->opt_round_group);
     uint32_t rounds = 0;
+    uint32_t r = 1;
     for (;;) {
-        for (int k = 0; k < group; k++) {
+        for (int k = 0; k < group; k++, r++) {
+            P.round = r;
+            P.stamp = ++Q.stamp;
             TG_LAUNCH(k_spfp_activate<FP>, grid, QT, 0, s, P);
             TG_LAUNCH(k_spfp_wait<FP>, grid, QT, 0, s, P);
             TG_LAUNCH(k_spfp_big<FP>, grid, QT, 0, s, P);
@@ -385,8 +377,9 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
         TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
         TG_TRY_CUDA(cudaStreamSynchronize(s));
         const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
-        if (h->cnt[h->round & 3][0] == 0) { rounds = h->round - 1; break; }
-        if (h->round > 10000000) { tg_set_error("SP/FP rounds did not converge"); return TG_ERR_CUDA; }
+        // r is the next round: its input count was written by the round just finished
+        if (h->cnt[r & 3][0] == 0) { rounds = r - 1; break; }
+        if (r > 10000000) { tg_set_error("SP/FP rounds did not converge"); return TG_ERR_CUDA; }
     }
     *rounds_out = rounds;
     return TG_OK;

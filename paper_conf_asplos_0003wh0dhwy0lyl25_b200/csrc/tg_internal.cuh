@@ -111,6 +111,7 @@ struct QueryScratch {
     bool nodes_state = false;  // SP/FP node-state arrays present
     void *st = nullptr;  // [n][S] packed u64 (time << 32 | pred), or u32 time when no pred is requested
     uint32_t *act = nullptr;           // [S][n] last activated time
+    uint32_t stamp = 0;                // SP/FP frontier dedupe stamps handed out (host counter; marks start at 0)
     uint32_t *mark = nullptr;          // [S][n] (EAT) or [S][nnodes] (SP/FP) frontier dedupe stamp
     uint32_t *bits = nullptr;          // [S][ceil(m/32)] "slot relaxed" bits (interior slots of long chains)
     uint64_t bit_words = 0;            // words per query
