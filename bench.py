@@ -171,6 +171,8 @@ def run_ours(a, rank, world, local_rank):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     ge, mine, problems, win, weighted, cfg = workload(a.config, a.k, rank, world, dev, a.mode)
+    if not weighted:
+        ge.w = None  # weights are not part of this workload (w = duration, reading A7)
     torch.cuda.synchronize()
     torch.cuda.empty_cache()  # generator temporaries: give them back before the library allocates
     k = len(mine)
@@ -319,6 +321,10 @@ def run_ours(a, rank, world, local_rank):
         }
 
     e2e = None
+    if persistent is not None:
+        persistent.close()  # the e2e leg builds its own graph (two C5 graphs do not fit one GPU)
+        persistent = None
+        torch.cuda.synchronize()
     if not a.no_e2e and comm is None:
         e2e = run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev)
 

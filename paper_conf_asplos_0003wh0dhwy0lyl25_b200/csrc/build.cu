@@ -108,7 +108,7 @@ __global__ void k_snap(const uint32_t *__restrict__ sid, uint64_t m, const uint4
             lo[j] = hi[j] = 0;
             arr[j] = r[j].y;
             if (p < m) {
-                srec[p] = r[j];
+                if (srec) srec[p] = r[j];
                 lo[j] = vnode_off[r[j].x];
                 hi[j] = vnode_off[r[j].x + 1];
             }
@@ -183,7 +183,7 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
                                 const uint32_t *__restrict__ succ, uint64_t m,
                                 const uint32_t *__restrict__ chain_first, const uint32_t *__restrict__ chain_len,
                                 const uint32_t *__restrict__ lidx, const uint32_t *__restrict__ sid,
-                                const uint4 *__restrict__ srec,
+                                const uint4 *__restrict__ srec, const uint4 *__restrict__ rec,
                                 const uint32_t *__restrict__ tn, const uint32_t *__restrict__ node_of,
                                 int4 *__restrict__ slots, uint32_t *__restrict__ slot_w,
                                 uint32_t *__restrict__ slot_tn, uint32_t *__restrict__ occ_slot,
@@ -207,7 +207,7 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
         uint32_t e = 0;
         while (q != TG_NONE) {
             e = sid[q];
-            r = srec[q];  // the edge's record in sorted order (written by k_snap)
+            r = srec ? srec[q] : rec[e];  // the edge's record (in sorted order when k_snap wrote it)
             if (q == p) r0 = r;
             slots[s] = make_int4((int)r.x, (int)r.y, (int)(id_map ? id_map[e] : e), (int)cw);
             slot_w[s] = r.z;
@@ -448,11 +448,22 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_TRY_CUDA(tg_malloc_async((void **)&indeg, nn * 4, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&hub, nn, s));
     TG_TRY_CUDA(cudaMemsetAsync(indeg, 0, nn * 4, s));
+    // sorted copy of the records for the chain scatter, when the device has room for it
+    // (a 1.47 B-edge partitioned build does not): otherwise the scatter gathers again
     uint4 *srec = nullptr;
-    TG_TRY_CUDA(tg_malloc_async((void **)&srec, m * 16, s));
+    {
+        size_t fr = 0, tot = 0;
+        cudaMemGetInfo(&fr, &tot);
+        if (fr > m * 16 + (4ull << 30) && tg_malloc_async((void **)&srec, m * 16, s) != cudaSuccess) {
+            cudaGetLastError();
+            srec = nullptr;
+        }
+    }
     TG_LAUNCH(k_snap, blocks_for(m, 4 * TG_SNAP_ILP), BT, 0, s, sid, m, rec, cg->vnode_off, cg->node_t, tn, indeg, srec);
-    TG_TRY_CUDA(cudaFreeAsync(rec, s));
-    rec = nullptr;
+    if (srec) {
+        TG_TRY_CUDA(cudaFreeAsync(rec, s));
+        rec = nullptr;
+    }
     TG_LAUNCH(k_hubs, blocks_for(nn, 4), BT, 0, s, indeg, cg->node_eoff, nn, hub);
     TG_TRY_CUDA(cudaFreeAsync(indeg, s));
 
@@ -494,12 +505,12 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_TRY(A.alloc((void **)&cg->sc_sumw, std::max<uint64_t>(L, 1) * 8));
     TG_TRY(A.alloc((void **)&cg->sc_elapsed, std::max<uint64_t>(L, 1) * 4));
     TG_LAUNCH(k_chain_scatter, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, cg->chain_first, chain_len, lidx, sid,
-              srec, tn, node_of, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
+              srec, rec, tn, node_of, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
               cg->sc_sumw, cg->sc_elapsed, id_map, (uint32_t)std::max<int64_t>(2, g->opt_walk_min));
 
-    for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)srec, (void *)hub,
+    for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)srec, (void *)rec, (void *)hub,
                     (void *)head, (void *)succ, (void *)cidx, (void *)chain_len, (void *)lidx})
-        TG_TRY_CUDA(cudaFreeAsync(p, s));
+        if (p) TG_TRY_CUDA(cudaFreeAsync(p, s));
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     return TG_OK;
 }

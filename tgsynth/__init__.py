@@ -80,7 +80,7 @@ class TemporalEdges:
                              self.dur.to(device), self.w.to(device), dict(self.meta))
 
     def numpy(self):
-        f = lambda a: a.cpu().numpy().astype(np.uint32)
+        f = lambda a: None if a is None else a.cpu().numpy().astype(np.uint32)
         return self.n, f(self.u), f(self.v), f(self.t), f(self.dur), f(self.w)
 
 
