@@ -45,35 +45,58 @@ __device__ __forceinline__ T block_excl_scan(T v, T *sh, T &total) {
     return wp + x - v;
 }
 
+// Each thread owns SCAN_ITEMS consecutive elements (two 16-byte loads when the tile is
+// full), so a tile needs one block-wide scan of the thread totals.
+__device__ __forceinline__ void scan_load8(const uint32_t *in, uint64_t idx, uint64_t count, uint32_t (&x)[SCAN_ITEMS]) {
+    if (idx + SCAN_ITEMS <= count) {
+        const uint4 a = *(const uint4 *)(in + idx), b = *(const uint4 *)(in + idx + 4);
+        x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
+    } else {
+#pragma unroll
+        for (int i = 0; i < SCAN_ITEMS; i++) x[i] = (idx + i < count) ? in[idx + i] : 0u;
+    }
+}
+
 __global__ void k_scan_reduce(const uint32_t *__restrict__ in, uint64_t count, uint32_t *__restrict__ sums) {
     __shared__ uint32_t sh[32];
-    uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE;
+    const uint64_t idx = (uint64_t)blockIdx.x * SCAN_TILE + (uint64_t)threadIdx.x * SCAN_ITEMS;
+    uint32_t x[SCAN_ITEMS];
+    scan_load8(in, idx, count, x);
     uint32_t acc = 0;
 #pragma unroll
-    for (int i = 0; i < SCAN_ITEMS; i++) {
-        uint64_t idx = base + (uint64_t)i * SCAN_THREADS + threadIdx.x;
-        if (idx < count) acc += in[idx];
-    }
+    for (int i = 0; i < SCAN_ITEMS; i++) acc += x[i];
     uint32_t total;
     block_excl_scan<uint32_t>(acc, sh, total);
     if (threadIdx.x == 0) sums[blockIdx.x] = total;
 }
 
+// in == out is allowed: every thread reads its own elements before writing them.
 __global__ void k_scan_apply(const uint32_t *in, uint32_t *out, uint64_t count,
                              const uint32_t *__restrict__ tile_off, uint32_t *d_total) {
     __shared__ uint32_t sh[32];
-    uint64_t base = (uint64_t)blockIdx.x * SCAN_TILE;
-    uint32_t carry = tile_off ? tile_off[blockIdx.x] : 0u;
+    const uint64_t idx = (uint64_t)blockIdx.x * SCAN_TILE + (uint64_t)threadIdx.x * SCAN_ITEMS;
+    uint32_t x[SCAN_ITEMS];
+    scan_load8(in, idx, count, x);
+    uint32_t acc = 0;
+#pragma unroll
+    for (int i = 0; i < SCAN_ITEMS; i++) acc += x[i];
+    uint32_t total;
+    uint32_t run = block_excl_scan<uint32_t>(acc, sh, total) + (tile_off ? tile_off[blockIdx.x] : 0u);
 #pragma unroll
     for (int i = 0; i < SCAN_ITEMS; i++) {
-        uint64_t idx = base + (uint64_t)i * SCAN_THREADS + threadIdx.x;
-        uint32_t v = (idx < count) ? in[idx] : 0u;
-        uint32_t row_total;
-        uint32_t ex = block_excl_scan<uint32_t>(v, sh, row_total);
-        if (idx < count) out[idx] = carry + ex;
-        carry += row_total;
+        const uint32_t v = x[i];
+        x[i] = run;
+        run += v;
     }
-    if (d_total && blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) *d_total = carry;
+    if (idx + SCAN_ITEMS <= count) {
+        *(uint4 *)(out + idx) = make_uint4(x[0], x[1], x[2], x[3]);
+        *(uint4 *)(out + idx + 4) = make_uint4(x[4], x[5], x[6], x[7]);
+    } else {
+#pragma unroll
+        for (int i = 0; i < SCAN_ITEMS; i++)
+            if (idx + i < count) out[idx + i] = x[i];
+    }
+    if (d_total && blockIdx.x == gridDim.x - 1 && threadIdx.x == SCAN_THREADS - 1) *d_total = run;
 }
 
 }  // namespace
