@@ -404,7 +404,8 @@ def run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev):
             tg.tg_query(g.h, tg.PROBLEMS[p], mine, win, houts[p])
         g.close()
 
-    step()
+    for _ in range(max(1, a.warmup)):  # same warm-up as the device-resident timing
+        step()
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()

@@ -2,6 +2,9 @@
 # step, one full capture of the round-4 activate/big kernels, then the bench lines.
 set -x
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+mkdir -p gpurun_out/prof
+timeout 600 python bench.py > gpurun_out/prof/bench_C2.json 2> gpurun_out/prof/bench_C2.err
+timeout 600 python bench.py --config C3 > gpurun_out/prof/bench_C3.json 2> gpurun_out/prof/bench_C3.err
 O=gpurun_out/prof
 mkdir -p $O
 M=dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum
@@ -12,5 +15,3 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 python tools/launches.py $O/launches_bench_step.csv 1000 > $O/launches_bench_step_summary.txt
 timeout 900 ncu --set full --import-source on --clock-control none --kernel-name regex:"k_eat_(activate|big)" --launch-skip 6 --launch-count 2 -o $O/eat_round4_activate_big_full -f python tools/prof_query.py --config C2 --problem eat --k 64 --reps 1 > /dev/null 2>&1
 cp $O/relax_traffic_C2.json profiles/round1/relax_traffic_C2.json
-timeout 600 python bench.py > $O/bench_C2.json 2> $O/bench_C2.err
-timeout 600 python bench.py --config C3 > $O/bench_C3.json 2> $O/bench_C3.err
