@@ -9,10 +9,6 @@
 
 namespace {
 
-#ifndef TG_RS_V2
-#define TG_RS_V2 1  // radix scatter with warp-private ranking
-#endif
-
 constexpr int SCAN_THREADS = 256;
 constexpr int SCAN_ITEMS = 8;
 constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
@@ -129,116 +125,32 @@ constexpr int RS_THREADS = 256;
 constexpr int RS_ITEMS = 16;
 constexpr int RS_TILE = RS_THREADS * RS_ITEMS;  // 4096 keys per tile
 constexpr int RS_WARPS = RS_THREADS / 32;
-constexpr size_t RS_SMEM = (size_t)RS_TILE * (8 + 4) + 2 * RS_WARPS * 256 * 4 + 256 * 4 * 2;
 
+// Digit width DB (8..10 bits): 2^DB buckets, DPT = 2^DB / 256 consecutive digits per
+// thread in the block-level passes.
+template <int DB>
 __global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const unsigned long long *__restrict__ keys, uint64_t m,
                                                            int shift, uint32_t *__restrict__ counts,
                                                            uint32_t ntiles) {
-    __shared__ uint32_t hist[256];
-    hist[threadIdx.x] = 0;
+    constexpr int ND = 1 << DB, DPT = ND / RS_THREADS;
+    __shared__ uint32_t hist[ND];
+#pragma unroll
+    for (int k = 0; k < DPT; k++) hist[threadIdx.x * DPT + k] = 0;
     __syncthreads();
-    uint64_t base = (uint64_t)blockIdx.x * RS_TILE;
+    const uint64_t base = (uint64_t)blockIdx.x * RS_TILE;
 #pragma unroll 4
     for (int i = 0; i < RS_ITEMS; i++) {
-        uint64_t idx = base + (uint64_t)i * RS_THREADS + threadIdx.x;
-        if (idx < m) atomicAdd(&hist[(uint32_t)(keys[idx] >> shift) & 255u], 1u);
-    }
-    __syncthreads();
-    counts[(uint64_t)threadIdx.x * ntiles + blockIdx.x] = hist[threadIdx.x];
-}
-
-// Stable scatter of one tile: ranks are computed in element order (round, warp,
-// lane), the tile is staged in shared memory grouped by digit, then written out
-// so that consecutive threads write consecutive global positions.
-__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const unsigned long long *__restrict__ kin,
-                                                              const uint32_t *__restrict__ vin,
-                                                              unsigned long long *__restrict__ kout,
-                                                              uint32_t *__restrict__ vout, uint64_t m, int shift,
-                                                              const uint32_t *__restrict__ offs, uint32_t ntiles) {
-    extern __shared__ __align__(16) unsigned char smem[];
-    unsigned long long *skey = (unsigned long long *)smem;
-    uint32_t *sval = (uint32_t *)(skey + RS_TILE);
-    uint32_t *wcnt = sval + RS_TILE;                 // [2][RS_WARPS][256]
-    uint32_t *tstart = wcnt + 2 * RS_WARPS * 256;    // [256]
-    uint32_t *gofs = tstart + 256;                   // [256]
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t lt_mask = (1u << lane) - 1u;
-    const uint64_t base = (uint64_t)blockIdx.x * RS_TILE;
-
-    gofs[tid] = offs[(uint64_t)tid * ntiles + blockIdx.x];
-    for (int w = 0; w < 2 * RS_WARPS; w++) wcnt[w * 256 + tid] = 0;
-    __syncthreads();
-
-    uint32_t lr[RS_ITEMS];
-    unsigned long long kk[RS_ITEMS];
-    uint32_t vv[RS_ITEMS];
-    uint32_t running = 0;  // thread tid owns digit tid
-#pragma unroll
-    for (int r = 0; r < RS_ITEMS; r++) {
-        uint32_t *A = wcnt + (r & 1) * RS_WARPS * 256;
-        uint32_t *B = wcnt + ((r + 1) & 1) * RS_WARPS * 256;
-        uint64_t idx = base + (uint64_t)r * RS_THREADS + tid;
-        bool valid = idx < m;
-        kk[r] = valid ? kin[idx] : 0ull;
-        vv[r] = valid ? vin[idx] : 0u;
-        uint32_t d = valid ? ((uint32_t)(kk[r] >> shift) & 255u) : 0x100u;
-        uint32_t peers = __match_any_sync(0xffffffffu, d);
-        uint32_t rank = __popc(peers & lt_mask);
-        if (valid && rank == 0) A[warp * 256 + d] = __popc(peers);
-        __syncthreads();
-        {
-            uint32_t run = running;
-#pragma unroll
-            for (int w = 0; w < RS_WARPS; w++) {
-                uint32_t c = A[w * 256 + tid];
-                A[w * 256 + tid] = run;
-                run += c;
-            }
-            running = run;
-#pragma unroll
-            for (int w = 0; w < RS_WARPS; w++) B[w * 256 + tid] = 0;
-        }
-        __syncthreads();
-        lr[r] = valid ? (A[warp * 256 + d] + rank) : 0u;
-    }
-    // exclusive scan of the tile's digit totals -> tile-local digit starts
-    {
-        uint32_t x = running;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= o) x += y;
-        }
-        __syncthreads();
-        if (lane == 31) wcnt[warp] = x;
-        __syncthreads();
-        uint32_t wp = 0;
-        for (int w = 0; w < warp; w++) wp += wcnt[w];
-        tstart[tid] = wp + x - running;
+        const uint64_t idx = base + (uint64_t)i * RS_THREADS + threadIdx.x;
+        if (idx < m) atomicAdd(&hist[(uint32_t)(keys[idx] >> shift) & (ND - 1)], 1u);
     }
     __syncthreads();
 #pragma unroll
-    for (int r = 0; r < RS_ITEMS; r++) {
-        uint64_t idx = base + (uint64_t)r * RS_THREADS + tid;
-        if (idx < m) {
-            uint32_t d = (uint32_t)(kk[r] >> shift) & 255u;
-            uint32_t p = tstart[d] + lr[r];
-            skey[p] = kk[r];
-            sval[p] = vv[r];
-        }
-    }
-    __syncthreads();
-    uint32_t nvalid = (uint32_t)min((uint64_t)RS_TILE, m - base);
-    for (uint32_t i = tid; i < nvalid; i += RS_THREADS) {
-        unsigned long long k = skey[i];
-        uint32_t d = (uint32_t)(k >> shift) & 255u;
-        uint32_t pos = gofs[d] + (i - tstart[d]);
-        kout[pos] = k;
-        vout[pos] = sval[i];
+    for (int k = 0; k < DPT; k++) {
+        const uint32_t d = threadIdx.x * DPT + k;
+        counts[(uint64_t)d * ntiles + blockIdx.x] = hist[d];
     }
 }
 
-#if TG_RS_V2
 // Stable scatter of one tile with warp-private ranking: warp w owns the contiguous
 // keys [w * 512, w * 512 + 512) of the tile (16 rounds of 32 coalesced keys); a key's
 // rank among equal digits of its warp is its peers below it in the round
@@ -247,31 +159,37 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const unsigned lon
 // per-warp digit counts into tile positions ((warp, round, lane) = index order, so
 // the scatter is stable), the tile is staged in shared memory grouped by digit and
 // written out so that consecutive threads write consecutive global positions.
-constexpr size_t RS2_SMEM = (size_t)RS_TILE * (8 + 4) + RS_WARPS * 256 * 4 + 256 * 4 * 2 + 32 * 4;
+template <int DB>
+constexpr size_t rs_smem() {
+    return (size_t)RS_TILE * (8 + 4) + (size_t)RS_WARPS * (1 << DB) * 4 + (size_t)(1 << DB) * 4 * 2 + 32 * 4;
+}
 
-__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter2(const unsigned long long *__restrict__ kin,
-                                                               const uint32_t *__restrict__ vin,
-                                                               unsigned long long *__restrict__ kout,
-                                                               uint32_t *__restrict__ vout, uint64_t m, int shift,
-                                                               const uint32_t *__restrict__ offs, uint32_t ntiles) {
+template <int DB>
+__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const unsigned long long *__restrict__ kin,
+                                                              const uint32_t *__restrict__ vin,
+                                                              unsigned long long *__restrict__ kout,
+                                                              uint32_t *__restrict__ vout, uint64_t m, int shift,
+                                                              const uint32_t *__restrict__ offs, uint32_t ntiles) {
+    constexpr int ND = 1 << DB, DPT = ND / RS_THREADS;
     extern __shared__ __align__(16) unsigned char smem[];
     unsigned long long *skey = (unsigned long long *)smem;
     uint32_t *sval = (uint32_t *)(skey + RS_TILE);
-    uint32_t *wcnt = sval + RS_TILE;                 // [RS_WARPS][256]
-    uint32_t *tstart = wcnt + RS_WARPS * 256;        // [256]
-    uint32_t *gofs = tstart + 256;                   // [256]
-    uint32_t *wsum = gofs + 256;                     // [32]
+    uint32_t *wcnt = sval + RS_TILE;                 // [RS_WARPS][ND]
+    uint32_t *tstart = wcnt + RS_WARPS * ND;         // [ND]
+    uint32_t *gofs = tstart + ND;                    // [ND]
+    uint32_t *wsum = gofs + ND;                      // [32]
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
     const uint64_t base = (uint64_t)blockIdx.x * RS_TILE;
     constexpr int PER_WARP = RS_TILE / RS_WARPS;
+    const uint32_t d0 = tid * DPT;  // this thread's digits in the block-level passes
 
-    gofs[tid] = offs[(uint64_t)tid * ntiles + blockIdx.x];
 #pragma unroll
-    for (int w = 0; w < RS_WARPS; w++) wcnt[w * 256 + tid] = 0;
+    for (int k = 0; k < DPT; k++) gofs[d0 + k] = offs[(uint64_t)(d0 + k) * ntiles + blockIdx.x];
+    for (int i = tid; i < RS_WARPS * ND; i += RS_THREADS) wcnt[i] = 0;
     __syncthreads();
 
-    uint32_t *mycnt = wcnt + warp * 256;
+    uint32_t *mycnt = wcnt + warp * ND;
     unsigned long long kk[RS_ITEMS];
     uint32_t vv[RS_ITEMS], lr[RS_ITEMS];
     const uint64_t wbase = base + (uint64_t)warp * PER_WARP;
@@ -286,7 +204,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter2(const unsigned lo
     for (int r = 0; r < RS_ITEMS; r++) {
         const uint64_t idx = wbase + (uint64_t)r * 32 + lane;
         const bool valid = idx < m;
-        const uint32_t d = valid ? ((uint32_t)(kk[r] >> shift) & 255u) : 0x100u;
+        const uint32_t d = valid ? ((uint32_t)(kk[r] >> shift) & (ND - 1)) : (uint32_t)ND;
         const uint32_t peers = __match_any_sync(0xffffffffu, d);
         const uint32_t below = __popc(peers & lt_mask);
         const uint32_t c = valid ? mycnt[d] : 0u;
@@ -296,16 +214,22 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter2(const unsigned lo
         lr[r] = c + below;
     }
     __syncthreads();
-    // thread tid owns digit tid: per-warp exclusive prefixes and the tile total
-    uint32_t tot = 0;
+    // per-warp exclusive prefixes of this thread's digits, and their tile totals
+    uint32_t tot[DPT], tsum = 0;
 #pragma unroll
-    for (int w = 0; w < RS_WARPS; w++) {
-        const uint32_t c = wcnt[w * 256 + tid];
-        wcnt[w * 256 + tid] = tot;
-        tot += c;
+    for (int k = 0; k < DPT; k++) {
+        uint32_t t = 0;
+#pragma unroll
+        for (int w = 0; w < RS_WARPS; w++) {
+            const uint32_t c = wcnt[w * ND + d0 + k];
+            wcnt[w * ND + d0 + k] = t;
+            t += c;
+        }
+        tot[k] = t;
+        tsum += t;
     }
-    // exclusive scan of the digit totals -> tile-local digit starts
-    uint32_t x = tot;
+    // exclusive scan of the digit totals (thread order = digit order) -> tile-local digit starts
+    uint32_t x = tsum;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
         const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
@@ -313,16 +237,20 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter2(const unsigned lo
     }
     if (lane == 31) wsum[warp] = x;
     __syncthreads();
-    uint32_t wp = 0;
+    uint32_t run = x - tsum;
 #pragma unroll
-    for (int w = 0; w < RS_WARPS; w++) wp += (w < warp) ? wsum[w] : 0u;
-    tstart[tid] = wp + x - tot;
+    for (int w = 0; w < RS_WARPS; w++) run += (w < warp) ? wsum[w] : 0u;
+#pragma unroll
+    for (int k = 0; k < DPT; k++) {
+        tstart[d0 + k] = run;
+        run += tot[k];
+    }
     __syncthreads();
 #pragma unroll
     for (int r = 0; r < RS_ITEMS; r++) {
         const uint64_t idx = wbase + (uint64_t)r * 32 + lane;
         if (idx < m) {
-            const uint32_t d = (uint32_t)(kk[r] >> shift) & 255u;
+            const uint32_t d = (uint32_t)(kk[r] >> shift) & (ND - 1);
             const uint32_t p = tstart[d] + mycnt[d] + lr[r];
             skey[p] = kk[r];
             sval[p] = vv[r];
@@ -332,13 +260,31 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter2(const unsigned lo
     const uint32_t nvalid = (uint32_t)min((uint64_t)RS_TILE, m - base);
     for (uint32_t i = tid; i < nvalid; i += RS_THREADS) {
         const unsigned long long k = skey[i];
-        const uint32_t d = (uint32_t)(k >> shift) & 255u;
+        const uint32_t d = (uint32_t)(k >> shift) & (ND - 1);
         const uint32_t pos = gofs[d] + (i - tstart[d]);
         kout[pos] = k;
         vout[pos] = sval[i];
     }
 }
-#endif
+
+template <int DB>
+tg_status radix_passes(unsigned long long *&ka, uint32_t *&va, unsigned long long *&kb, uint32_t *&vb, uint64_t m,
+                       int key_bits, uint64_t ntiles, uint32_t *counts, cudaStream_t s, int snap_bits,
+                       uint32_t *snap_vals) {
+    TG_TRY_CUDA(cudaFuncSetAttribute(k_radix_scatter<DB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)rs_smem<DB>()));
+    for (int shift = 0; shift < key_bits; shift += DB) {
+        TG_LAUNCH(k_radix_hist<DB>, (unsigned)ntiles, RS_THREADS, 0, s, ka, m, shift, counts, (uint32_t)ntiles);
+        TG_TRY(tg_exclusive_scan_u32(counts, counts, ntiles << DB, nullptr, s, nullptr));
+        TG_LAUNCH(k_radix_scatter<DB>, (unsigned)ntiles, RS_THREADS, rs_smem<DB>(), s, ka, va, kb, vb, m, shift,
+                  counts, (uint32_t)ntiles);
+        std::swap(ka, kb);
+        std::swap(va, vb);
+        if (snap_vals && snap_bits > 0 && shift + DB == snap_bits)
+            TG_TRY_CUDA(cudaMemcpyAsync(snap_vals, va, m * 4, cudaMemcpyDeviceToDevice, s));
+    }
+    return TG_OK;
+}
 
 }  // namespace
 
@@ -359,37 +305,30 @@ tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uin
     *sorted_vals = vals;
     if (m <= 1 || key_bits <= 0) return TG_OK;
     uint64_t ntiles = (m + RS_TILE - 1) / RS_TILE;
-    if (ntiles * 256 >= 0xFFFFFFFFull) {
+    if ((ntiles << 10) >= 0xFFFFFFFFull) {
         tg_set_error("radix sort: too many tiles");
         return TG_ERR_RANGE;
+    }
+    // digit width: the fewest passes over the key bits (ties: the narrower digit); an
+    // intermediate snapshot (sweep time order) needs whole 8-bit digits
+    int db = 8;
+    if (!(snap_vals && snap_bits > 0)) {
+        const int p8 = (key_bits + 7) / 8, p9 = (key_bits + 8) / 9, p10 = (key_bits + 9) / 10;
+        db = (p10 < p9 && p10 < p8) ? 10 : (p9 < p8 ? 9 : 8);
+#ifdef TG_RS_DB_FORCE
+        db = TG_RS_DB_FORCE;  // tuning experiments
+#endif
     }
     unsigned long long *k2 = nullptr;
     uint32_t *v2 = nullptr, *counts = nullptr;
     TG_TRY_CUDA(tg_malloc_async((void **)&k2, m * 8, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&v2, m * 4, s));
-    TG_TRY_CUDA(tg_malloc_async((void **)&counts, ntiles * 256 * 4, s));
-#if TG_RS_V2
-    TG_TRY_CUDA(cudaFuncSetAttribute(k_radix_scatter2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)RS2_SMEM));
-#else
-    TG_TRY_CUDA(cudaFuncSetAttribute(k_radix_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)RS_SMEM));
-#endif
+    TG_TRY_CUDA(tg_malloc_async((void **)&counts, (ntiles << db) * 4, s));
     unsigned long long *ka = keys, *kb = k2;
     uint32_t *va = vals, *vb = v2;
-    for (int shift = 0; shift < key_bits; shift += 8) {
-        TG_LAUNCH(k_radix_hist, (unsigned)ntiles, RS_THREADS, 0, s, ka, m, shift, counts, (uint32_t)ntiles);
-        TG_TRY(tg_exclusive_scan_u32(counts, counts, ntiles * 256, nullptr, s, nullptr));
-#if TG_RS_V2
-        TG_LAUNCH(k_radix_scatter2, (unsigned)ntiles, RS_THREADS, RS2_SMEM, s, ka, va, kb, vb, m, shift, counts,
-                  (uint32_t)ntiles);
-#else
-        TG_LAUNCH(k_radix_scatter, (unsigned)ntiles, RS_THREADS, RS_SMEM, s, ka, va, kb, vb, m, shift, counts,
-                  (uint32_t)ntiles);
-#endif
-        std::swap(ka, kb);
-        std::swap(va, vb);
-        if (snap_vals && snap_bits > 0 && shift + 8 == snap_bits)
-            TG_TRY_CUDA(cudaMemcpyAsync(snap_vals, va, m * 4, cudaMemcpyDeviceToDevice, s));
-    }
+    if (db == 10) TG_TRY((radix_passes<10>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals)));
+    else if (db == 9) TG_TRY((radix_passes<9>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals)));
+    else TG_TRY((radix_passes<8>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals)));
     TG_TRY_CUDA(cudaFreeAsync(counts, s));
     if (ka != keys) {
         // result lives in the scratch buffers: copy back so the caller's buffers hold it

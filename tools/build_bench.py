@@ -46,6 +46,7 @@ if "--check" in sys.argv:
     import hashlib
     h = hashlib.sha1()
     for mir in (False, True):
-        for a in g.export_chains(mirrored=mir):
-            h.update(np.ascontiguousarray(np.asarray(a)).tobytes())
+        ex = g.export_chains(mirrored=mir)
+        for key in sorted(ex):
+            h.update(np.ascontiguousarray(ex[key]).tobytes())
     print("  chain export digest:", h.hexdigest())
