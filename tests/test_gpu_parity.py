@@ -177,6 +177,27 @@ def test_c2_small_batch(tg):
         _check_rows(tg, g, og, "ld", srcs[:16], win)
 
 
+@pytest.mark.parametrize("k", [40, 64, 65])
+def test_two_query_groups(tg, k):
+    """Sub-batches spanning two 32-query groups (a partial second group at 40, full at
+    64, and 64 + a ragged 1-query sub-batch at 65): packed (pred) and u32-state (values
+    only, the bench path) rows against the oracle."""
+    import torch
+    ge = tgsynth.make_graph("C2", scale_shift=-5)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d)
+    og = oracle.Graph(n, u, v, t, d)
+    srcs = tgsynth.config_sources("C2", ge, k=k)
+    win = tgsynth.CONFIGS["C2"]["windows"][1]
+    for p in ("eat", "ld"):
+        _check_rows(tg, g, og, p, srcs, win)
+        vals = tg.as_u32(g.query(p, srcs, win))
+        torch.cuda.synchronize()
+        for r in (0, k // 2, k - 1):
+            ref = (oracle.eat if p == "eat" else oracle.ld)(og, srcs[r], *win)[0]
+            np.testing.assert_array_equal(vals[r], ref, err_msg=f"u32-state {p} row {r}")
+
+
 def test_union_work_count(tg):
     """W_union (distinct slots relaxed by any query of the sub-batch, the bench's
     algorithmic-bytes input) equals the union of the oracle's usable valid edges."""
