@@ -21,6 +21,8 @@
 #include <cooperative_groups.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 #include "tg_internal.cuh"
@@ -36,6 +38,10 @@ constexpr int QT = 256;
 constexpr uint32_t BIG_T = 256;
 constexpr uint32_t CHUNK = 1024;
 constexpr uint32_t WAIT_INLINE = 32;  // wait-propagation steps a lane does inline; longer walks go to k_spfp_wait
+#ifndef TG_WAIT_SEG
+#define TG_WAIT_SEG 128  // C3: FP 2.45 -> 0.89 ms, SP 2.95 -> 0.90 ms per 16 queries (1024: 1.18, 256: 0.92, 64: 0.89)
+#endif
+constexpr uint32_t WAIT_SEG = TG_WAIT_SEG;  // nodes per queued wait segment (one warp each)
 
 struct SpP {
     const uint32_t *vnode_off, *node_t, *node_u, *node_eoff, *occ_slot, *occ_node;
@@ -197,9 +203,15 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
                 if (++steps == WAIT_INLINE) { more = jend < vend; break; }
             }
             if (more) {
-                const uint32_t k = atomicAdd(R.wait_cnt, 1u);
-                if (k < P.waitcap) P.waitq[k] = make_uint4(q, jend, vend, d);
-                else push_node(P, R, q, jend - 1);  // queue full: the walk continues next round
+                // the rest of the walk as WAIT_SEG-node segments, walked by different warps in
+                // parallel: waiting from node j to ANY later node is legal, so every segment
+                // applies d on its own and stops at its first node that is already as good
+                // (that node's own value is being propagated past it)
+                const uint32_t nseg = (vend - jend + WAIT_SEG - 1) / WAIT_SEG;
+                const uint32_t k = atomicAdd(R.wait_cnt, nseg);
+                for (uint32_t c = 0; c < nseg && k + c < P.waitcap; c++)
+                    P.waitq[k + c] = make_uint4(q, jend + c * WAIT_SEG, min(vend, jend + (c + 1) * WAIT_SEG), d);
+                if (k + nseg > P.waitcap) push_node(P, R, q, jend - 1);  // queue full: continue next round
             }
             e0 = __ldg(P.node_eoff + j);
             cnt = __ldg(P.node_eoff + jend) - e0;
@@ -366,21 +378,39 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     const int group = (int)std::max<int64_t>(1, g->opt_round_group);
     uint32_t rounds = 0;
     uint32_t r = 1;
+    static const bool trace = getenv("TG_TRACE") != nullptr;
+    cudaEvent_t tev[4] = {};
+    if (trace)
+        for (auto &e : tev) cudaEventCreate(&e);
     for (;;) {
-        for (int k = 0; k < group; k++, r++) {
+        for (int k = 0; k < (trace ? 1 : group); k++, r++) {
             P.round = r;
             P.stamp = ++Q.stamp;
+            if (trace) cudaEventRecord(tev[0], s);
             TG_LAUNCH(k_spfp_activate<FP>, grid, QT, 0, s, P);
+            if (trace) cudaEventRecord(tev[1], s);
             TG_LAUNCH(k_spfp_wait<FP>, grid, QT, 0, s, P);
+            if (trace) cudaEventRecord(tev[2], s);
             TG_LAUNCH(k_spfp_big<FP>, grid, QT, 0, s, P);
+            if (trace) cudaEventRecord(tev[3], s);
         }
         TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
         TG_TRY_CUDA(cudaStreamSynchronize(s));
         const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
+        if (trace) {
+            float ms[3] = {0, 0, 0};
+            for (int i = 0; i < 3; i++) cudaEventElapsedTime(&ms[i], tev[i], tev[i + 1]);
+            const uint32_t last = r - 1;
+            fprintf(stderr, "[tg] %s S=%u round %u: frontier %u wait-walks %u big-chunks %u | activate %.3f wait %.3f "
+                    "big %.3f ms\n", FP ? "FP" : "SP", Sb, last, h->cnt[last & 3][0], h->cnt[last & 3][2],
+                    h->cnt[last & 3][1], ms[0], ms[1], ms[2]);
+        }
         // r is the next round: its input count was written by the round just finished
         if (h->cnt[r & 3][0] == 0) { rounds = r - 1; break; }
         if (r > 10000000) { tg_set_error("SP/FP rounds did not converge"); return TG_ERR_CUDA; }
     }
+    if (trace)
+        for (auto &e : tev) cudaEventDestroy(e);
     *rounds_out = rounds;
     return TG_OK;
 }
