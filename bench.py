@@ -75,6 +75,7 @@ class ClockSampler:
     }
 
     def __init__(self, device_index):
+        self.interval = float(os.environ.get("BENCH_CLOCK_INTERVAL", "0.01"))
         self.samples = []
         self.reasons = set()
         self.max_mhz = None
@@ -101,7 +102,7 @@ class ClockSampler:
                         self.reasons.add(name)
             except Exception:
                 pass
-            time.sleep(0.01)
+            time.sleep(self.interval)
 
     def start(self):
         if self.ok:
@@ -210,10 +211,29 @@ def run_ours(a, rank, world, local_rank):
         if world > 1:
             dist.barrier()
 
-    # warm-up
-    for _ in range(max(a.warmup, 0)):
+    # warm-up (with the in-library event profiling on when it will be on in the timed
+    # region: the event pool then already holds the events the timed steps record)
+    if not a.no_profile:
+        tg.tg_profile_enable(True)
+    wms = []
+    for i in range(max(a.warmup, 0) + 30):
+        # at least W warm-up steps; then up to 30 more until the last three agree within
+        # 10 % (the box settles: a process that just exited can still disturb the first
+        # few hundred ms)
+        if i >= max(a.warmup, 3) and max(wms[-3:]) <= 1.1 * min(wms[-3:]):
+            break
+        if i >= max(a.warmup, 0) and a.warmup < 3:
+            break
+        w0 = torch.cuda.Event(enable_timing=True)
+        w1 = torch.cuda.Event(enable_timing=True)
+        w0.record()
         step()
+        w1.record()
+        torch.cuda.synchronize()
+        wms.append(w0.elapsed_time(w1))
     torch.cuda.synchronize()
+    tg.tg_profile_enable(False)
+    tg.tg_profile_report()  # recycle the warm-up's events into the pool
 
     # work counts (untimed): W per query from the engine's first-touch counter (== oracle W, tested)
     gstat = persistent or make_graph()
@@ -245,31 +265,57 @@ def run_ours(a, rank, world, local_rank):
 
     # timed region (CUDA events on the stream all our kernels run on: the legacy default stream)
     prof = not a.no_profile
-    sampler = ClockSampler(local_rank)
-    if prof:
-        tg.tg_profile_report()  # clear
-        tg.tg_profile_enable(True)
-    launches0 = tg.tg_kernel_launch_count()
-    barrier()
-    torch.cuda.synchronize()
-    sampler.start()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for _ in range(a.steps):
-        step()
-    e1.record()
-    torch.cuda.synchronize()
-    barrier()
-    clocks = sampler.stop()
-    launches = tg.tg_kernel_launch_count() - launches0
-    kprof = tg.tg_profile_report() if prof else {}
-    tg.tg_profile_enable(False)
-    ms = e0.elapsed_time(e1) / a.steps
+
+    def timed():
+        """EXACTLY a.steps steps between barrier + synchronize on both sides (CUDA events on the
+        stream every kernel of ours runs on), NVML clocks sampled during the region."""
+        sampler = ClockSampler(local_rank)
+        if prof:
+            tg.tg_profile_report()  # clear
+            tg.tg_profile_enable(True)
+        launches0 = tg.tg_kernel_launch_count()
+        barrier()
+        torch.cuda.synchronize()
+        sampler.start()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        marks = []  # per-step boundaries (events on the same stream; no extra synchronisation)
+        for _ in range(a.steps):
+            step()
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record()
+            marks.append(ev)
+        e1.record()
+        torch.cuda.synchronize()
+        barrier()
+        clocks = sampler.stop()
+        step_ms = [round(e0.elapsed_time(marks[0]), 3)] + [round(marks[i - 1].elapsed_time(marks[i]), 3)
+                                                           for i in range(1, len(marks))]
+        launches = tg.tg_kernel_launch_count() - launches0
+        kprof = tg.tg_profile_report() if prof else {}
+        tg.tg_profile_enable(False)
+        ms = e0.elapsed_time(e1) / a.steps
+        if world > 1:
+            t = torch.tensor([ms], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms, step_ms, clocks, launches, kprof
+
+    ms, step_ms, clocks, launches, kprof = timed()
+    # A transient host/driver disturbance (seen right after another GPU process exits:
+    # a few consecutive steps at 3x the others) is re-measured once, like a clock event;
+    # both attempts are reported.
+    first_attempt = None
+    med = sorted(step_ms)[len(step_ms) // 2]
+    disturbed = float(max(step_ms) > 1.5 * med)
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([disturbed], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        disturbed = float(t.item())
+    if disturbed:
+        first_attempt = {"ms_per_step": ms, "step_ms": step_ms}
+        ms, step_ms, clocks, launches, kprof = timed()
 
     queries_per_step = k * len(problems) * (world if a.mode == "replicate" else 1)
     value = queries_per_step / (ms / 1e3)
@@ -373,13 +419,15 @@ def run_ours(a, rank, world, local_rank):
         "e2e": e2e,
         "gpu_launches": launches,
         "clocks": clocks,
+        "step_ms": step_ms,
+        "remeasured": first_attempt,
+        "warmup_steps_run": len(wms),
     }
-    if rank == 0:
-        print(json.dumps(res), flush=True)
     if comm is not None:
         tg.tg_comm_destroy(comm)
     if world > 1:
         dist.destroy_process_group()
+    return res if rank == 0 else None
 
 
 def run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev):
@@ -409,15 +457,26 @@ def run_e2e(a, tg, ge, mine, problems, win, weighted, world, dev):
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
     steps = max(1, min(a.steps, 3))
-    e0.record()
-    for _ in range(steps):
-        step()
-    e1.record()
-    torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / steps
+
+    def timed():
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        marks = []
+        e0.record()
+        for _ in range(steps):
+            step()
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record()
+            marks.append(ev)
+        e1.record()
+        torch.cuda.synchronize()
+        st = [e0.elapsed_time(marks[0])] + [marks[i - 1].elapsed_time(marks[i]) for i in range(1, len(marks))]
+        return e0.elapsed_time(e1) / steps, st
+
+    ms, st = timed()
+    if max(st) > 1.5 * min(st):  # transient disturbance (see the device-resident timing): re-measure once
+        ms, st = timed()
     if world > 1:
         t = torch.tensor([ms], dtype=torch.float64, device=dev)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
@@ -497,7 +556,7 @@ def run_reference(a, rank, world):
            "config": {"workload": describe(a.config, ge, k, problems, win)},
            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": 1, "kind": "oracle", "sample": sample},
            "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(res), flush=True)
+    return res
 
 
 def main():
@@ -509,10 +568,19 @@ def main():
     if world == 1 and a.gpus > 1:
         print(json.dumps({"error": "use torchrun --nproc-per-node N for --gpus N > 1"}))
         return 2
-    if a.impl == "reference":
-        run_reference(a, rank, world)
-    else:
-        run_ours(a, rank, world, local_rank)
+    # stdout carries exactly one JSON line: native libraries (NCCL's version banner, ...)
+    # print to fd 1, so fd 1 points at stderr while the benchmark runs
+    sys.stdout.flush()
+    saved = os.dup(1)
+    os.dup2(2, 1)
+    try:
+        res = run_reference(a, rank, world) if a.impl == "reference" else run_ours(a, rank, world, local_rank)
+    finally:
+        sys.stdout.flush()
+        os.dup2(saved, 1)
+        os.close(saved)
+    if res is not None:
+        print(json.dumps(res), flush=True)
     return 0
 
 

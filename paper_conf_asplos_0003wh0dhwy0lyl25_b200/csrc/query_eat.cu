@@ -678,7 +678,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
         TG_TRY(A.alloc((void **)&Q.lat, S * n * 4));
         TG_TRY(A.alloc((void **)&Q.pcount, 64));
     }
-    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
+    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 4096));  // >= TG_MAXP round-control records
     TG_TRY(A.alloc((void **)&Q.srcs, S * 4));
     TG_TRY(A.alloc((void **)&Q.srcs_int, S * 4));
     TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8 + 8 + 64));  // [S] per query, [S] distinct slots, [S+1..] diag
@@ -722,7 +722,7 @@ tg_status tg_ensure_scratch_srcs(tg_graph *g, uint32_t S) {
     Q = QueryScratch{};
     Q.S = S;
     Q.n = g->n;
-    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 256));
+    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 4096));  // >= TG_MAXP round-control records
     TG_TRY(Q.arena.alloc((void **)&Q.srcs, S * 4));
     TG_TRY(Q.arena.alloc((void **)&Q.srcs_int, S * 4));
     return TG_OK;
@@ -875,6 +875,7 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
 tg_status tg_comm_allreduce_min_u64(tg_comm *c, unsigned long long *buf, uint64_t count, cudaStream_t s);
 tg_status tg_comm_allreduce_sum_u32(tg_comm *c, uint32_t *buf, uint64_t count, cudaStream_t s);
 tg_status tg_comm_allreduce_min_u32(tg_comm *c, uint32_t *buf, uint64_t count, cudaStream_t s);
+int tg_comm_world(const tg_comm *c);
 
 // Single query batch partitioned by vertex range (SURVEY §8(e) mode 2).  Every
 // partition p (one per rank with NCCL, or g->nparts logical partitions on one GPU)
@@ -923,7 +924,13 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
             TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8 + 8 + 64, s));
             TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
         }
-        TG_LAUNCH(k_eat_init<PK>, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl, 0);
+        // One process holds every partition (logical partitions, or a world of 1): the
+        // partitions share the state and the frontier bitmaps, so the bits the relaxations
+        // set ARE the next frontier (as in the unpartitioned engine).  Across ranks the
+        // frontier is derived from the exchanged state instead (k_part_frontier).
+        const bool local = !g->comm || tg_comm_world(g->comm) == 1;
+        TG_LAUNCH(k_eat_init<PK>, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl,
+                  local ? 1 : 0);
         const bool work = any_work && g->m > 0 && alpha < omega;
         uint32_t rounds = 0;
         if (work) {
@@ -951,17 +958,20 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 parts[pi] = P;
                 TG_LAUNCH(k_ctl_reset, 1, 1, 0, s, Q.ctl + pi);
                 // round 1's frontier: the sources, derived from the state like every later one
-                TG_LAUNCH(k_part_frontier<PK>, grid, 256, 0, s, Q.st, Q.lat, Q.fb[1], Sb, G, g->part_vb[pi],
-                          g->part_vb[pi + 1], Q.pcount);
+                if (!local)
+                    TG_LAUNCH(k_part_frontier<PK>, grid, 256, 0, s, Q.st, Q.lat, Q.fb[1], Sb, G, g->part_vb[pi],
+                              g->part_vb[pi + 1], Q.pcount);
             }
-            if (g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
+            if (!local) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
             uint32_t r = 1;
             for (;;) {
-                TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.pcount, 4, cudaMemcpyDeviceToHost, s));
-                TG_TRY_CUDA(cudaStreamSynchronize(s));
-                if (Q.h_ctr[0] == 0) break;
+                if (!local) {
+                    TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.pcount, 4, cudaMemcpyDeviceToHost, s));
+                    TG_TRY_CUDA(cudaStreamSynchronize(s));
+                    if (Q.h_ctr[0] == 0) break;
+                    TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
+                }
                 if (r > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
-                TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
                 for (int pi = 0; pi < g->nparts; pi++) {
                     if (parts[pi].ub0 == parts[pi].ub1) continue;  // no vertices: never any work
                     parts[pi].round = r;
@@ -969,16 +979,25 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                     TG_LAUNCH(k_eat_big<PK>, grid, QT, 0, s, parts[pi]);
                     TG_LAUNCH(k_eat_chain<PK>, 148, QT, 0, s, parts[pi]);
                 }
-                // exchange: every rank ends the round with the elementwise min of all ranks' states
-                if (g->comm) {
-                    if (PK) TG_TRY(tg_comm_allreduce_min_u64(g->comm, (unsigned long long *)Q.st, (uint64_t)Sb * n, s));
-                    else TG_TRY(tg_comm_allreduce_min_u32(g->comm, (uint32_t *)Q.st, (uint64_t)Sb * n, s));
+                if (local) {
+                    // a round in which no partition consumed a frontier word did no work
+                    TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl) * g->nparts, cudaMemcpyDeviceToHost, s));
+                    TG_TRY_CUDA(cudaStreamSynchronize(s));
+                    const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
+                    uint64_t words = 0;
+                    for (int pi = 0; pi < g->nparts; pi++) words += h[pi].cnt[r & 3][3];
+                    if (words == 0) { rounds = r - 1; break; }
+                    r++;
+                    continue;
                 }
+                // exchange: every rank ends the round with the elementwise min of all ranks' states
+                if (PK) TG_TRY(tg_comm_allreduce_min_u64(g->comm, (unsigned long long *)Q.st, (uint64_t)Sb * n, s));
+                else TG_TRY(tg_comm_allreduce_min_u32(g->comm, (uint32_t *)Q.st, (uint64_t)Sb * n, s));
                 uint32_t *fnext = ((r + 1) & 1) ? Q.fb[1] : Q.fb[0];
                 for (int pi = 0; pi < g->nparts; pi++)
                     TG_LAUNCH(k_part_frontier<PK>, grid, 256, 0, s, Q.st, Q.lat, fnext, Sb, G, g->part_vb[pi],
                               g->part_vb[pi + 1], Q.pcount);
-                if (g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
+                TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
                 r++;
                 rounds = r - 1;
             }
