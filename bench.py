@@ -47,6 +47,8 @@ def parse_args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-profile", action="store_true", help="do not bracket kernels with CUDA events")
+    ap.add_argument("--profile-all", action="store_true",
+                    help="bracket every kernel with CUDA events (default: only the relaxation kernels)")
     ap.add_argument("--query-only", action="store_true", help="time only tg_query (graph built once)")
     ap.add_argument("--mode", choices=["replicate", "vertex"], default="replicate",
                     help="multi-GPU mode: replicate = source sharding (weak scaling); vertex = one batch "
@@ -213,8 +215,9 @@ def run_ours(a, rank, world, local_rank):
 
     # warm-up (with the in-library event profiling on when it will be on in the timed
     # region: the event pool then already holds the events the timed steps record)
-    if not a.no_profile:
-        tg.tg_profile_enable(True)
+    plevel = 0 if a.no_profile else (1 if a.profile_all else 2)
+    if plevel:
+        tg.tg_profile_enable(plevel)
     wms = []
     for i in range(max(a.warmup, 0) + 30):
         # at least W warm-up steps; then up to 30 more until the last three agree within
@@ -272,7 +275,7 @@ def run_ours(a, rank, world, local_rank):
         sampler = ClockSampler(local_rank)
         if prof:
             tg.tg_profile_report()  # clear
-            tg.tg_profile_enable(True)
+            tg.tg_profile_enable(plevel)
         launches0 = tg.tg_kernel_launch_count()
         barrier()
         torch.cuda.synchronize()
@@ -308,7 +311,8 @@ def run_ours(a, rank, world, local_rank):
     # both attempts are reported.
     first_attempt = None
     med = sorted(step_ms)[len(step_ms) // 2]
-    disturbed = float(max(step_ms) > 1.5 * med)
+    warm_ref = sorted(wms[-3:])[len(wms[-3:]) // 2] if len(wms) >= 3 else None
+    disturbed = float(max(step_ms) > 1.5 * med or (warm_ref is not None and ms > 1.25 * warm_ref))
     if world > 1:
         t = torch.tensor([disturbed], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -332,7 +336,6 @@ def run_ours(a, rank, world, local_rank):
         relax_ms = sum(kprof[x][1] for x in relax_names)
         relax_launches = sum(kprof[x][0] for x in relax_names)
         dom = max(kprof.items(), key=lambda kv: kv[1][1])
-        total_kernel_ms = sum(v[1] for v in kprof.values())
         # SURVEY 8(d), batched with source lanes: every slot relaxed by some query of a
         # sub-batch is read once (16 B slot + 4 B occurrence), every relaxation touches
         # 8 B of packed state: B = W_union * 20 + sum_q W_q * 8.  (In vertex mode the
@@ -359,9 +362,10 @@ def run_ours(a, rank, world, local_rank):
             "single_source_formula_GBps": single_source_bytes / (relax_ms / 1e3) / 1e9 if relax_ms else None,
             "relax_ms_per_step": relax_ms / a.steps,
             "relax_launches_per_step": relax_launches / a.steps,
-            "relax_share_of_kernel_time": relax_ms / total_kernel_ms if total_kernel_ms else None,
+            "relax_share_of_step": relax_ms / a.steps / ms,
             "dominant_single_kernel": dom[0],
-            "dominant_single_kernel_share": dom[1][1] / total_kernel_ms if total_kernel_ms else None,
+            "dominant_single_kernel_share_of_step": dom[1][1] / a.steps / ms,
+            "profiled_kernels": "all" if plevel == 1 else "relaxation kernels only (CUDA events per launch)",
             "kernels_ms_per_step": {x: round(v[1] / a.steps, 4) for x, v in
                                     sorted(kprof.items(), key=lambda kv: -kv[1][1])[:12]},
         }
@@ -422,6 +426,7 @@ def run_ours(a, rank, world, local_rank):
         "step_ms": step_ms,
         "remeasured": first_attempt,
         "warmup_steps_run": len(wms),
+        "warmup_settled_ms": warm_ref,
     }
     if comm is not None:
         tg.tg_comm_destroy(comm)

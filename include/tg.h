@@ -230,8 +230,10 @@ TG_API uint64_t tg_kernel_launch_count(void);
  * This returns every cached block to the CUDA driver. */
 TG_API void tg_release_cached_memory(void);
 
-/* Per-kernel timing for measurement: when enabled, every launch is bracketed by
- * a CUDA event pair recorded on the launching stream.  tg_profile_report
+/* Per-kernel timing for measurement: on = 1 brackets every launch with a CUDA
+ * event pair recorded on the launching stream; on = 2 only the relaxation kernels
+ * of the EAT family (activation, chunked ranges, chain walks: the roofline kernels),
+ * which keeps the recording overhead out of the rest of the step; 0 = off.  tg_profile_report
  * synchronises on the recorded events and folds them into a per-kernel table;
  * with buf != NULL it writes the table as a JSON object
  * {"kernel_name": [launches, total_ms], ...} (NUL-terminated, truncated to

@@ -208,7 +208,7 @@ void tg_release_cached_memory(void) {
     cudaGetLastError();
 }
 
-void tg_profile_enable(int on) { g_tg_profile = on ? 1 : 0; }
+void tg_profile_enable(int on) { g_tg_profile = (on < 0 || on > 2) ? 1 : on; }
 
 int tg_profile_report(char *buf, uint64_t buf_len) {
     // {"kernel": [launches, total_ms], ...}.  Recorded launches are folded into a

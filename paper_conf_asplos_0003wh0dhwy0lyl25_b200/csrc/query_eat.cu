@@ -771,11 +771,11 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
             for (int k = 0; k < group; k++, r++) {
                 P.round = r;
                 if (trace) cudaEventRecord(tev[0], s);
-                TG_LAUNCH(k_eat_activate<PK>, grid, QT, 0, s, P);
+                TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, P);
                 if (trace) cudaEventRecord(tev[1], s);
-                TG_LAUNCH(k_eat_big<PK>, grid, QT, 0, s, P);
+                TG_LAUNCH_RELAX(k_eat_big<PK>, grid, QT, 0, s, P);
                 if (trace) cudaEventRecord(tev[2], s);
-                TG_LAUNCH(k_eat_chain<PK>, 148, QT, 0, s, P);  // at most a few hundred walks per round
+                TG_LAUNCH_RELAX(k_eat_chain<PK>, 148, QT, 0, s, P);  // at most a few hundred walks per round
                 if (trace) cudaEventRecord(tev[3], s);
             }
             TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
@@ -975,9 +975,9 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 for (int pi = 0; pi < g->nparts; pi++) {
                     if (parts[pi].ub0 == parts[pi].ub1) continue;  // no vertices: never any work
                     parts[pi].round = r;
-                    TG_LAUNCH(k_eat_activate<PK>, grid, QT, 0, s, parts[pi]);
-                    TG_LAUNCH(k_eat_big<PK>, grid, QT, 0, s, parts[pi]);
-                    TG_LAUNCH(k_eat_chain<PK>, 148, QT, 0, s, parts[pi]);
+                    TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH_RELAX(k_eat_big<PK>, grid, QT, 0, s, parts[pi]);
+                    TG_LAUNCH_RELAX(k_eat_chain<PK>, 148, QT, 0, s, parts[pi]);
                 }
                 if (local) {
                     // a round in which no partition consumed a frontier word did no work

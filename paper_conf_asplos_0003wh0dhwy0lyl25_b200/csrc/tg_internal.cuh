@@ -39,14 +39,20 @@ extern uint64_t g_tg_launches;  // kernels launched by this library (process-wid
 extern int g_tg_profile;
 cudaEvent_t tg_prof_begin(cudaStream_t s);
 void tg_prof_end(const char *name, cudaStream_t s, cudaEvent_t ev0);
-#define TG_LAUNCH(kernel, grid, block, smem, stream, ...)                  \
-    do {                                                                   \
-        cudaEvent_t _ev0 = g_tg_profile ? tg_prof_begin(stream) : nullptr; \
-        kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);        \
-        g_tg_launches++;                                                   \
-        if (_ev0) tg_prof_end(#kernel, stream, _ev0);                      \
-        TG_TRY_CUDA(cudaGetLastError());                                   \
+#define TG_LAUNCH_LVL(lvl, kernel, grid, block, smem, stream, ...)                    \
+    do {                                                                              \
+        cudaEvent_t _ev0 = (g_tg_profile && g_tg_profile <= (lvl)) ? tg_prof_begin(stream) \
+                                                                    : nullptr;          \
+        kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);                   \
+        g_tg_launches++;                                                              \
+        if (_ev0) tg_prof_end(#kernel, stream, _ev0);                                 \
+        TG_TRY_CUDA(cudaGetLastError());                                              \
     } while (0)
+// every kernel (profiled at level 1); the relaxation kernels (profiled at levels 1 and 2)
+#define TG_LAUNCH(kernel, grid, block, smem, stream, ...) \
+    TG_LAUNCH_LVL(1, kernel, grid, block, smem, stream, __VA_ARGS__)
+#define TG_LAUNCH_RELAX(kernel, grid, block, smem, stream, ...) \
+    TG_LAUNCH_LVL(2, kernel, grid, block, smem, stream, __VA_ARGS__)
 
 // ----------------------------------------------------------------------------- device memory
 // Simple owning device buffer list for a graph handle.

@@ -223,8 +223,9 @@ def tg_release_cached_memory():
     load_library().tg_release_cached_memory()
 
 
-def tg_profile_enable(on: bool = True):
-    load_library().tg_profile_enable(1 if on else 0)
+def tg_profile_enable(on=True):
+    """True / 1: every kernel; 2: only the EAT-family relaxation kernels; False / 0: off."""
+    load_library().tg_profile_enable(int(on) if not isinstance(on, bool) else (1 if on else 0))
 
 
 def tg_profile_report() -> dict:
