@@ -204,7 +204,7 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *   "sub_batch"  sources processed concurrently (0 = automatic)
  *   "stats"      1 = count relaxations per query (slower), 0 = off
  *   "shortcuts"  1 = relax chain tails through shortcuts on first entry (default), 0 = off
- *   "round_group" rounds launched between host convergence checks (default 4)
+ *   "round_group" rounds launched between host convergence checks (default 8)
  *   "mirror"     1 = build the LD mirror in tg_build_chains (default), 0 = on first LD query
  *   "walk_min"   chains with at least this many edges are walked by the chain engine
  *                (default 6, min 2, before build); shorter chains are relaxed edge by

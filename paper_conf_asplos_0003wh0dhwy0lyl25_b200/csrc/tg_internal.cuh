@@ -182,7 +182,7 @@ struct tg_graph {
     int64_t opt_sub_batch = 0;
     int64_t opt_stats = 0;
     int64_t opt_shortcuts = 1;
-    int64_t opt_round_group = 4;
+    int64_t opt_round_group = 8;  // GAC rounds launched per host convergence check
     int opt_mirror = 1;
     int64_t opt_exp = 0;
     int64_t opt_packed_state = 0;
