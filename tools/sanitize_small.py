@@ -18,6 +18,9 @@ for opts in ({}, {"walk_min": 2}, {"partitions": 3}):
     src = list(range(40))
     for p in ("eat", "ld", "reach") + (() if opts.get("partitions") else ("fp", "sp")):
         g.query(p, src, (10, 900))
+    if not opts:
+        g.query("eat", list(range(64)), (0, 1000))   # u32 states, 64-query extract fast path
+        g.query("ld", [5], (0, 1000))                # single-query batch
     host = torch.empty((3, ge.n), dtype=torch.int32)
     tg.tg_query(g.h, tg.TG_EAT, [0, 1, 2], (0, 1000), host)
     g.close()
