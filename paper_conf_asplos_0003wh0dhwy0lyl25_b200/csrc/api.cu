@@ -97,6 +97,29 @@ cudaError_t tg_malloc_async(void **p, size_t bytes, cudaStream_t s) {
     return e;
 }
 
+namespace {
+std::vector<void *> g_pinned;
+std::mutex g_pinned_mu;
+}  // namespace
+
+cudaError_t tg_pinned_get(void **p) {
+    {
+        std::lock_guard<std::mutex> lk(g_pinned_mu);
+        if (!g_pinned.empty()) {
+            *p = g_pinned.back();
+            g_pinned.pop_back();
+            return cudaSuccess;
+        }
+    }
+    return cudaMallocHost(p, 4096);
+}
+
+void tg_pinned_put(void *p) {
+    if (!p) return;
+    std::lock_guard<std::mutex> lk(g_pinned_mu);
+    g_pinned.push_back(p);
+}
+
 tg_status DevArena::alloc(void **p, size_t bytes) {
     *p = nullptr;
     bytes = round_bytes(bytes ? bytes : 16);
@@ -389,7 +412,7 @@ void tg_graph_destroy(tg_graph *g) {
     DeviceGuard dg(g->device);
     cudaDeviceSynchronize();
     g->qs.arena.free_all();
-    if (g->qs.h_ctr) cudaFreeHost(g->qs.h_ctr);
+    tg_pinned_put(g->qs.h_ctr);
     tg_sweep_free(g);
     g->arena.free_all();
     delete[] g->last_relax;

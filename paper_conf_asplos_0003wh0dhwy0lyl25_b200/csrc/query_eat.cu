@@ -635,7 +635,8 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     if (Q.S >= S && Q.n == g->n && Q.st && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat)) return TG_OK;
     TG_TRY_CUDA(cudaDeviceSynchronize());  // blocks go back to the cache for immediate reuse
     Q.arena.free_all();
-    if (Q.h_ctr) { cudaFreeHost(Q.h_ctr); Q.h_ctr = nullptr; }
+    tg_pinned_put(Q.h_ctr);
+    Q.h_ctr = nullptr;
     Q = QueryScratch{};
     const uint64_t n = g->n, m = g->m;
     Q.S = S;
@@ -678,7 +679,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
         TG_TRY(A.alloc((void **)&Q.lat, S * n * 4));
         TG_TRY(A.alloc((void **)&Q.pcount, 64));
     }
-    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 4096));  // >= TG_MAXP round-control records
+    TG_TRY_CUDA(tg_pinned_get((void **)&Q.h_ctr));  // >= TG_MAXP round-control records
     TG_TRY(A.alloc((void **)&Q.srcs, S * 4));
     TG_TRY(A.alloc((void **)&Q.srcs_int, S * 4));
     TG_TRY(A.alloc((void **)&Q.relax_cnt, S * 8 + 8 + 64));  // [S] per query, [S] distinct slots, [S+1..] diag
@@ -718,11 +719,12 @@ tg_status tg_ensure_scratch_srcs(tg_graph *g, uint32_t S) {
     if (Q.st) return ensure_scratch(g, std::max(S, Q.S), Q.nodes_state);  // full scratch keeps working
     TG_TRY_CUDA(cudaDeviceSynchronize());
     Q.arena.free_all();
-    if (Q.h_ctr) { cudaFreeHost(Q.h_ctr); Q.h_ctr = nullptr; }
+    tg_pinned_put(Q.h_ctr);
+    Q.h_ctr = nullptr;
     Q = QueryScratch{};
     Q.S = S;
     Q.n = g->n;
-    TG_TRY_CUDA(cudaMallocHost((void **)&Q.h_ctr, 4096));  // >= TG_MAXP round-control records
+    TG_TRY_CUDA(tg_pinned_get((void **)&Q.h_ctr));  // >= TG_MAXP round-control records
     TG_TRY(Q.arena.alloc((void **)&Q.srcs, S * 4));
     TG_TRY(Q.arena.alloc((void **)&Q.srcs_int, S * 4));
     return TG_OK;

@@ -200,6 +200,10 @@ struct tg_graph {
 // Stream-ordered temporary allocation; on failure the block cache is returned to
 // the driver, the pool trimmed, and the allocation retried once.
 cudaError_t tg_malloc_async(void **p, size_t bytes, cudaStream_t s);
+// 4 KB pinned host blocks for round-control readback, cached process-wide (a new
+// graph per step would otherwise pay cudaMallocHost / cudaFreeHost every step)
+cudaError_t tg_pinned_get(void **p);
+void tg_pinned_put(void *p);
 
 // ----------------------------------------------------------------------------- primitives
 // Exclusive prefix sum of in[0..count) into out (may alias), total -> *d_total (device, may be null).
