@@ -13,6 +13,9 @@
 //   7. shortcut per long chain (Alg. 2 fold) and the occurrence index (replaces the
 //      GPU hash table of: sorted-edge position -> slot)
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 
 #include "tg_internal.cuh"
 
@@ -364,12 +367,25 @@ static int bits_for(uint64_t x) {  // bits to represent values in [0, x]
     return std::max(b, 1);
 }
 
+// TG_TRACE_BUILD=1: synchronise at the build's section boundaries and print the host
+// time of each section to stderr (diagnostics of slow builds; off by default)
+static void bmark(cudaStream_t s, const char *label) {
+    static const bool on = getenv("TG_TRACE_BUILD") != nullptr;
+    if (!on) return;
+    static std::chrono::steady_clock::time_point last;
+    cudaStreamSynchronize(s);
+    const auto now = std::chrono::steady_clock::now();
+    if (label) fprintf(stderr, "build-trace %s %.3f\n", label, std::chrono::duration<double, std::milli>(now - last).count());
+    last = now;
+}
+
 tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
                              const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
                              uint32_t tmax, cudaStream_t s) {
     const uint32_t n = g->n;
     cg->n = n;
     cg->m = m;
+    bmark(s, nullptr);
     DevArena &A = g->arena;
     TG_TRY(A.alloc((void **)&cg->vnode_off, ((size_t)n + 1) * 4));
     if (m == 0) {
@@ -402,6 +418,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
         TG_TRY_CUDA(cudaFreeAsync(tsid, s));
     }
 
+    bmark(s, "sort");
     // ---- 2. departure nodes
     uint32_t *node_of = nullptr, *d_cnt = nullptr;
     TG_TRY(A.alloc((void **)&cg->occ_node, m * 4));
@@ -438,6 +455,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_LAUNCH(k_vnode_off, blocks_for(nn + 1, 4), BT, 0, s, cg->node_u, nn, n, cg->vnode_off);
     TG_TRY_CUDA(cudaFreeAsync(keys, s));
 
+    bmark(s, "nodes");
     // ---- 3./4. snap, in-degree, hubs
     uint32_t *tn = nullptr, *indeg = nullptr;
     uint4 *rec = nullptr;
@@ -452,13 +470,32 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     // (a 1.47 B-edge partitioned build does not): otherwise the scatter gathers again
     uint4 *srec = nullptr;
     {
+        // memory the stream-ordered pool holds but does not use serves the copy without
+        // asking the driver: cudaMemGetInfo stalls the host for 10-100 ms at times on
+        // the virtualised GPU boxes (TG_TRACE_BUILD), so it is only the fallback
         size_t fr = 0, tot = 0;
-        cudaMemGetInfo(&fr, &tot);
-        if (fr > m * 16 + (4ull << 30) && tg_malloc_async((void **)&srec, m * 16, s) != cudaSuccess) {
+        bool room = false;
+        {
+            int dev = 0;
+            cudaGetDevice(&dev);
+            cudaMemPool_t pool;
+            uint64_t reserved = 0, used = 0;
+            if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess &&
+                cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved) == cudaSuccess &&
+                cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used) == cudaSuccess)
+                room = reserved >= used && reserved - used >= m * 16 + (1ull << 20);
+            cudaGetLastError();
+        }
+        if (!room) {
+            cudaMemGetInfo(&fr, &tot);
+            room = fr > m * 16 + (4ull << 30);
+        }
+        if (room && tg_malloc_async((void **)&srec, m * 16, s) != cudaSuccess) {
             cudaGetLastError();
             srec = nullptr;
         }
     }
+    bmark(s, "memgetinfo");
     TG_LAUNCH(k_snap, blocks_for(m, 4 * TG_SNAP_ILP), BT, 0, s, sid, m, rec, cg->vnode_off, cg->node_t, tn, indeg, srec);
     if (srec) {
         TG_TRY_CUDA(cudaFreeAsync(rec, s));
@@ -467,6 +504,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_LAUNCH(k_hubs, blocks_for(nn, 4), BT, 0, s, indeg, cg->node_eoff, nn, hub);
     TG_TRY_CUDA(cudaFreeAsync(indeg, s));
 
+    bmark(s, "snap_hubs");
     // ---- 5. heads / successors; chain ids in (head u, head t, first id) order
     uint32_t *head = nullptr, *succ = nullptr, *cidx = nullptr;
     TG_TRY_CUDA(tg_malloc_async((void **)&head, m * 4, s));
@@ -479,6 +517,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     cg->nchains = nch;
 
+    bmark(s, "chains");
     // ---- 6. chain lengths, slot offsets, long-chain numbering
     uint32_t *chain_len = nullptr, *lidx = nullptr;
     TG_TRY_CUDA(tg_malloc_async((void **)&chain_len, (uint64_t)nch * 4 + 4, s));
@@ -512,6 +551,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
                     (void *)head, (void *)succ, (void *)cidx, (void *)chain_len, (void *)lidx})
         if (p) TG_TRY_CUDA(cudaFreeAsync(p, s));
     TG_TRY_CUDA(cudaStreamSynchronize(s));
+    bmark(s, "scatter");
     return TG_OK;
 }
 
