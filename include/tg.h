@@ -213,10 +213,13 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *                no gain measured on R-MAT); invisible to callers
  *   "partitions" logical vertex-range partitions on this GPU (1..16, before build):
  *                runs the multi-GPU mode-1 algorithm inside one process (tests)
- *   "engine"     EAT/LD/REACH schedule: 0 = automatic (GAC), 1 = GAC rounds over chains
- *                (Alg. 3), 2 = time-partitioned sweep (experimental; needs "sweep_struct")
- *   "sweep_struct" 1 = also build the time-ordered edge list in tg_build_chains (default 0)
- *   "sweep_part" sweep: edges per time partition (0 = automatic)
+ *   "exchange"   1 = vertex-range partitions run the cross-rank algorithm even inside one
+ *                process: logical partitions relax private state copies that are combined
+ *                by an elementwise-min kernel after every round (the stand-in for
+ *                ncclAllReduce(min)); a communicator of world 1 calls NCCL itself.  Every
+ *                partition then derives its next frontier from the combined state, as
+ *                the ranks of a multi-GPU run do (tests; default 0: one process shares
+ *                one state and frontier)
  *   "packed_state" 1 = EAT/LD/REACH keep the packed u64 (arrival << 32 | pred) state even
  *                when pred == NULL (default 0: without pred the state is the u32 arrival
  *                alone -- half the state bytes; values are identical) */

@@ -52,6 +52,8 @@ def _load():
             f = getattr(lib, name)
             f.restype = i64
             f.argtypes = [u32, u64, P, P, P, P, P, u32, u32, u32, P, P]
+        lib.oracle_time_order.restype = ctypes.c_int
+        lib.oracle_time_order.argtypes = [u64, P, P]
         lib.oracle_sp.restype = ctypes.c_int
         lib.oracle_sp.argtypes = [u32, u64, P, P, P, P, P, P, u32, u32, u32, P]
         lib.oracle_fp.restype = ctypes.c_int
@@ -76,7 +78,9 @@ class Graph:
     """Edge-list temporal graph: e = (u, v, t, t + lam[, w]).
 
     ``w`` defaults to ``lam`` (reading A7).  Sorting is done once with numpy
-    (a library primitive): ``order`` by t (stable), ``order_ut`` by (u, t, id).
+    (a library primitive) for ``order_ut`` by (u, t, id); ``order`` (by t, ties in
+    input order) is the C counting sort ``oracle_time_order`` (pinned against
+    numpy's stable argsort).
     """
 
     def __init__(self, n, u, v, t, lam, w=None):
@@ -90,7 +94,10 @@ class Graph:
     @property
     def order(self):
         if self._order is None:
-            self._order = np.ascontiguousarray(np.argsort(self.t, kind="stable"), dtype=np.int64)
+            order = np.empty(max(self.m, 1), np.int64)
+            if _load().oracle_time_order(self.m, _p(self.t), _p(order)) != 0:
+                raise MemoryError
+            self._order = order[: self.m]
         return self._order
 
     @property

@@ -24,8 +24,9 @@
  * so the order among equal t is irrelevant.
  *
  * All values are uint32.  ORACLE_NONE = 0xFFFFFFFF marks "unreached" / "no pred".
- * The caller supplies `order`: edge indices sorted by t ascending (a library sort,
- * numpy.argsort(kind="stable")).
+ * The caller supplies `order`: edge indices sorted by t ascending, ties in input
+ * order (oracle_time_order below: a textbook stable counting sort; pinned against
+ * numpy.argsort(kind="stable") in tests/test_oracle_pins.py).
  *
  * Alg. 1 (§4.1) and Alg. 2 (§4.2) are written out for the
  * chain / shortcut parity of the transformer and skeleton generator.
@@ -39,6 +40,32 @@
 static int valid_edge(uint32_t t, uint32_t lam, uint32_t alpha, uint32_t omega) {
     /* P:L110 window [start, end]: start <= start(P), end(P) <= end (reading A3). */
     return t >= alpha && (uint64_t)t + lam <= (uint64_t)omega;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Stable sort of the edge indices by departure time (the "topological order" of
+ * P:L123): two counting-sort passes (LSD) over the low and the high 16 bits of t.
+ * Counting sort is stable, so after both passes edges are ordered by t with ties
+ * in input order.  Returns -1 if the scratch allocation fails. */
+int oracle_time_order(uint64_t m, const uint32_t *t, int64_t *order) {
+    int64_t *tmp = (int64_t *)malloc((m ? m : 1) * sizeof(int64_t));
+    uint64_t *cnt = (uint64_t *)malloc(65537 * sizeof(uint64_t));
+    if (!tmp || !cnt) { free(tmp); free(cnt); return -1; }
+    for (uint64_t i = 0; i < m; i++) tmp[i] = (int64_t)i;
+    int64_t *src = tmp, *dst = order;
+    for (int pass = 0; pass < 2; pass++) {
+        const int shift = 16 * pass;
+        memset(cnt, 0, 65537 * sizeof(uint64_t));
+        for (uint64_t i = 0; i < m; i++) cnt[((t[src[i]] >> shift) & 0xFFFFu) + 1]++;
+        for (int d = 0; d < 65536; d++) cnt[d + 1] += cnt[d];
+        for (uint64_t i = 0; i < m; i++) dst[cnt[(t[src[i]] >> shift) & 0xFFFFu]++] = src[i];
+        int64_t *x = src; src = dst; dst = x;
+    }
+    /* two passes: the result is back in tmp's partner -- src now points at it */
+    if (src != order) memcpy(order, src, m * sizeof(int64_t));
+    free(tmp);
+    free(cnt);
+    return 0;
 }
 
 /* ------------------------------------------------------------------------- */

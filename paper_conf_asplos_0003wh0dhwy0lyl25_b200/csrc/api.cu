@@ -165,10 +165,6 @@ tg_status tg_validate_edges(tg_graph *g, cudaStream_t s);
 tg_status tg_build_mirror(tg_graph *g, cudaStream_t s);
 tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                             uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
-tg_status tg_run_sweep(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
-                       uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
-bool tg_sweep_available(const tg_graph *g, tg_problem p);
-void tg_sweep_free(tg_graph *g);
 tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                       bool out_dev, cudaStream_t s);
 tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
@@ -398,10 +394,6 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
         return tg_run_eat_partitioned(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     }
     if (p == TG_EAT || p == TG_LD || p == TG_REACH) {
-        // schedule: the time sweep (default when its edge list was built) or GAC rounds
-        if (g->opt_engine == 2 && tg_sweep_available(g, p))
-            return tg_run_sweep(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
-        if (g->opt_engine == 2) { tg_set_error("sweep schedule unavailable (option sweep_struct = 0 or partitioned)"); return TG_ERR_STATE; }
         return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     }
     return tg_run_spfp(g, p, sources, n_sources, w, out, out_dev, s);
@@ -411,9 +403,9 @@ void tg_graph_destroy(tg_graph *g) {
     if (!g) return;
     DeviceGuard dg(g->device);
     cudaDeviceSynchronize();
+    tg_sink_destroy(g);
     g->qs.arena.free_all();
     tg_pinned_put(g->qs.h_ctr);
-    tg_sweep_free(g);
     g->arena.free_all();
     delete[] g->last_relax;
     delete g;
@@ -549,17 +541,8 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
         if (g->built) { tg_set_error("set relabel before tg_build_chains"); return TG_ERR_STATE; }
         g->opt_relabel = value ? 1 : 0;
     }
-    else if (k == "exp") g->opt_exp = value;
+    else if (k == "exchange") g->opt_exchange = value ? 1 : 0;
     else if (k == "packed_state") g->opt_packed_state = value ? 1 : 0;
-    else if (k == "engine") {
-        if (value < 0 || value > 2) { tg_set_error("engine must be 0 (auto), 1 (gac) or 2 (sweep)"); return TG_ERR_RANGE; }
-        g->opt_engine = value;
-    }
-    else if (k == "sweep_part") g->opt_sweep_part = value < 0 ? 0 : std::min<int64_t>(value, 0x7FFFFFFF);
-    else if (k == "sweep_struct") {
-        if (g->built) { tg_set_error("set sweep_struct before tg_build_chains"); return TG_ERR_STATE; }
-        g->opt_sweep_struct = value ? 1 : 0;
-    }
     else if (k == "walk_min") {
         if (g->built) { tg_set_error("set walk_min before tg_build_chains"); return TG_ERR_STATE; }
         g->opt_walk_min = value < 2 ? 2 : value;

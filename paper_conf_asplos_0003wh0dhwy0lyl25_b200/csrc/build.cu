@@ -230,19 +230,6 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
     }
 }
 
-// time-ordered edge records for the sweep schedule: te[i] = {u, v, t, t + duration}
-__global__ void k_time_edges(const uint32_t *__restrict__ tsid, uint64_t m, const uint32_t *__restrict__ U,
-                             const uint32_t *__restrict__ V, const uint32_t *__restrict__ T,
-                             const uint32_t *__restrict__ DUR, const uint32_t *__restrict__ id_map,
-                             int4 *__restrict__ te, uint32_t *__restrict__ te_id) {
-    GRID_STRIDE(i, m) {
-        const uint32_t e = tsid[i];
-        const uint32_t t = T[e];
-        te[i] = make_int4((int)U[e], (int)V[e], (int)t, (int)(t + DUR[e]));
-        te_id[i] = id_map ? id_map[e] : e;
-    }
-}
-
 __global__ void k_validate(const uint32_t *__restrict__ u, const uint32_t *__restrict__ v,
                            const uint32_t *__restrict__ t, const uint32_t *__restrict__ dur,
                            const uint32_t *__restrict__ w, uint64_t m, uint32_t n, uint32_t *__restrict__ res) {
@@ -395,28 +382,17 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
         return TG_OK;
     }
     // ---- 1. sort by (u, t, id); tmax bounds this direction's t (known from validation).
-    // With the time-ordered edge list requested, t occupies whole radix digits, so the
-    // LSD passes over t alone leave the ids in (t, id) order: that intermediate payload
-    // is the sweep's time order (no extra sort; same pass count on the configs).
     const uint32_t maxt = tmax;
-    const bool want_te = g->nparts == 0 && g->opt_sweep_struct;
-    const int tbits = want_te ? (bits_for(maxt) + 7) / 8 * 8 : bits_for(maxt);
+    const int tbits = bits_for(maxt);
     const int ubits = bits_for(n - 1);
     unsigned long long *keys = nullptr;
-    uint32_t *sid = nullptr, *tsid = nullptr;
+    uint32_t *sid = nullptr;
     TG_TRY_CUDA(tg_malloc_async((void **)&keys, m * 8, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&sid, m * 4, s));
-    if (want_te) TG_TRY_CUDA(tg_malloc_async((void **)&tsid, m * 4, s));
     TG_LAUNCH(k_make_keys, blocks_for(m, 4), BT, 0, s, u, t, m, tbits, keys, sid);
     unsigned long long *sk;
     uint32_t *sv;
-    TG_TRY(tg_radix_sort_pairs_snap(keys, sid, m, tbits + ubits, &sk, &sv, s, want_te ? tbits : 0, tsid));
-    if (want_te) {
-        TG_TRY(A.alloc((void **)&cg->te, m * 16));
-        TG_TRY(A.alloc((void **)&cg->te_id, m * 4));
-        TG_LAUNCH(k_time_edges, blocks_for(m, 4), BT, 0, s, tsid, m, u, v, t, dur, id_map, cg->te, cg->te_id);
-        TG_TRY_CUDA(cudaFreeAsync(tsid, s));
-    }
+    TG_TRY(tg_radix_sort_pairs(keys, sid, m, tbits + ubits, &sk, &sv, s));
 
     bmark(s, "sort");
     // ---- 2. departure nodes

@@ -69,8 +69,7 @@ struct EatP {
     uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
     uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
     uint32_t alpha, omega;
-    int use_sc, stats, exp;
-  // exp: diagnostic variants for timing only (results invalid when != 0)
+    int use_sc, stats;
     RoundCtl *ctl;
     uint32_t round;       // GAC round of this launch (host loop counter; parity picks the bitmaps)
     uint32_t *fb0, *fb1;  // frontier masks [n][G] (bit = query within the group), by round parity
@@ -611,6 +610,20 @@ __global__ void k_part_frontier(const void *__restrict__ st_, uint32_t *__restri
     if (lane == 0 && mine) atomicAdd(count, mine);
 }
 
+// Exchange of logical partitions in one process (option "exchange"): partition p
+// relaxed into its private state copy st + p * len; every copy ends the round with the
+// elementwise min of all copies -- exactly what ncclAllReduce(min) leaves on every rank.
+template <bool PK>
+__global__ void k_state_min_exchange(void *__restrict__ st_, uint32_t P, uint64_t len) {
+    using T = typename StW<PK>::T;
+    T *st = (T *)st_;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < len; i += (uint64_t)gridDim.x * blockDim.x) {
+        T m = st[i];
+        for (uint32_t p = 1; p < P; p++) m = min(m, st[p * len + i]);
+        for (uint32_t p = 0; p < P; p++) st[p * len + i] = m;
+    }
+}
+
 __global__ void k_popcount(const uint32_t *__restrict__ w, uint64_t nw, unsigned long long *__restrict__ out) {
     unsigned long long c = 0;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x)
@@ -632,7 +645,10 @@ __global__ void k_ctl_reset(RoundCtl *ctl) {
 static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     QueryScratch &Q = g->qs;
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
-    if (Q.S >= S && Q.n == g->n && Q.st && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat)) return TG_OK;
+    const uint32_t copies = (g->opt_exchange && !g->comm && g->nparts > 1) ? (uint32_t)g->nparts : 1u;
+    if (Q.S >= S && Q.n == g->n && Q.st && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat) &&
+        Q.st_copies >= copies)
+        return TG_OK;
     TG_TRY_CUDA(cudaDeviceSynchronize());  // blocks go back to the cache for immediate reuse
     Q.arena.free_all();
     tg_pinned_put(Q.h_ctr);
@@ -644,7 +660,8 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     Q.nnodes = nnodes;
     Q.nodes_state = nodes_state;
     DevArena &A = Q.arena;
-    TG_TRY(A.alloc((void **)&Q.st, S * n * 8));
+    Q.st_copies = copies;
+    TG_TRY(A.alloc((void **)&Q.st, S * n * 8 * copies));
     TG_TRY(A.alloc((void **)&Q.act, S * n * 4));
     Q.vwords = (uint32_t)((S + 31) / 32);  // query groups per vertex
     TG_TRY(A.alloc((void **)&Q.fb[0], n * Q.vwords * 4));
@@ -712,24 +729,6 @@ uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
 
 tg_status tg_ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) { return ensure_scratch(g, S, nodes_state); }
 
-// Sources and host staging only (engines with their own state, e.g. the sweep).
-tg_status tg_ensure_scratch_srcs(tg_graph *g, uint32_t S) {
-    QueryScratch &Q = g->qs;
-    if (Q.S >= S && Q.n == g->n && Q.srcs) return TG_OK;
-    if (Q.st) return ensure_scratch(g, std::max(S, Q.S), Q.nodes_state);  // full scratch keeps working
-    TG_TRY_CUDA(cudaDeviceSynchronize());
-    Q.arena.free_all();
-    tg_pinned_put(Q.h_ctr);
-    Q.h_ctr = nullptr;
-    Q = QueryScratch{};
-    Q.S = S;
-    Q.n = g->n;
-    TG_TRY_CUDA(tg_pinned_get((void **)&Q.h_ctr));  // >= TG_MAXP round-control records
-    TG_TRY(Q.arena.alloc((void **)&Q.srcs, S * 4));
-    TG_TRY(Q.arena.alloc((void **)&Q.srcs_int, S * 4));
-    return TG_OK;
-}
-
 // Run the GAC rounds of one sub-batch on direction cg; returns rounds used.
 template <bool PK>
 static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
@@ -757,7 +756,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
         P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
         P.ub0 = 0; P.ub1 = g->n * G;
-        P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats; P.exp = (int)g->opt_exp;
+        P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         P.touched = Q.touched;
@@ -818,8 +817,7 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     TG_TRY(ensure_scratch(g, S, false));
     QueryScratch &Q = g->qs;
     const uint64_t n = g->n;
-    if (!out_dev && !Q.out_stage) TG_TRY(Q.arena.alloc((void **)&Q.out_stage, (uint64_t)Q.S * n * 4));
-    if (pred && !pred_dev && !Q.pred_stage) TG_TRY(Q.arena.alloc((void **)&Q.pred_stage, (uint64_t)Q.S * n * 4));
+    TG_TRY(tg_sink_begin(g, !out_dev, pred && !pred_dev));
     g->last = tg_query_stats{};
     if (g->opt_stats) {
         delete[] g->last_relax;
@@ -838,8 +836,10 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         else TG_TRY(eat_rounds<false>(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
         g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;
-        uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
-        uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
+        const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
+        uint32_t *o = out_dev ? out + (size_t)b0 * n : nullptr;
+        uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : pred) : nullptr;
+        TG_TRY(tg_sink_target(g, bi, !out_dev, pred && !pred_dev, &o, &pr, s));
         const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
         if (pk)
             TG_LAUNCH(k_eat_extract<true>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
@@ -850,8 +850,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         else
             TG_LAUNCH(k_eat_extract<false>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
                       g->relabeled ? g->perm : (const uint32_t *)nullptr);
-        if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
-        if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
+        TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n,
+                             (pred && !pred_dev) ? pred + (size_t)b0 * n : nullptr, (size_t)Sb * n * 4, s));
         if (g->opt_stats) {
             const uint64_t tw = (g->m + 31) / 32 + TG_MAXP + 1;
             TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, Q.touched, tw,
@@ -869,6 +869,7 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         }
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
+    TG_TRY(tg_sink_end(g));
     g->last.kernel_launches = g_tg_launches - launches0;
     return TG_OK;
 }
@@ -900,8 +901,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
     TG_TRY(ensure_scratch(g, S, false));
     QueryScratch &Q = g->qs;
     const uint64_t n = g->n;
-    if (!out_dev && !Q.out_stage) TG_TRY(Q.arena.alloc((void **)&Q.out_stage, (uint64_t)Q.S * n * 4));
-    if (pred && !pred_dev && !Q.pred_stage) TG_TRY(Q.arena.alloc((void **)&Q.pred_stage, (uint64_t)Q.S * n * 4));
+    TG_TRY(tg_sink_begin(g, !out_dev, pred && !pred_dev));
     g->last = tg_query_stats{};
     if (g->opt_stats) {
         delete[] g->last_relax;
@@ -915,7 +915,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         const uint32_t Sb = std::min(S, k - b0);
         const uint32_t G = (Sb + 31) / 32;
         TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
-        TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, Sb * n * (PK ? 8 : 4), s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, Sb * n * (PK ? 8 : 4) * Q.st_copies, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, Sb * n * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.lat, 0xFF, Sb * n * 4, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, Sb * Q.bit_words * 4, s));
@@ -930,9 +930,15 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         // partitions share the state and the frontier bitmaps, so the bits the relaxations
         // set ARE the next frontier (as in the unpartitioned engine).  Across ranks the
         // frontier is derived from the exchanged state instead (k_part_frontier).
-        const bool local = !g->comm || tg_comm_world(g->comm) == 1;
-        TG_LAUNCH(k_eat_init<PK>, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl,
-                  local ? 1 : 0);
+        // Option "exchange" forces the cross-rank algorithm in one process: logical
+        // partitions then relax private state copies combined by k_state_min_exchange
+        // (the stand-in for ncclAllReduce), and a world of 1 calls NCCL itself.
+        const bool local = !g->opt_exchange && (!g->comm || tg_comm_world(g->comm) == 1);
+        const uint32_t ncopy = (!local && !g->comm) ? (uint32_t)g->nparts : 1u;
+        const uint64_t slen = (uint64_t)Sb * n;  // state words of one copy
+        for (uint32_t c = 0; c < ncopy; c++)
+            TG_LAUNCH(k_eat_init<PK>, (Sb + 255) / 256, 256, 0, s, (char *)Q.st + c * slen * (PK ? 8 : 4), g->n, G,
+                      Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl, local ? 1 : 0);
         const bool work = any_work && g->m > 0 && alpha < omega;
         uint32_t rounds = 0;
         if (work) {
@@ -949,6 +955,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
             for (int pi = 0; pi < g->nparts; pi++) {
                 const ChainGraph &cg = ld ? g->pm[pi] : g->pf[pi];
                 EatP P = base;
+                if (ncopy > 1) P.st = (char *)Q.st + pi * slen * (PK ? 8 : 4);  // private copy
                 P.bits = Q.bits + bit_off * Sb;
                 P.touched = Q.touched + bit_off;
                 bit_off += (cg.m + 31) / 32;
@@ -964,7 +971,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                     TG_LAUNCH(k_part_frontier<PK>, grid, 256, 0, s, Q.st, Q.lat, Q.fb[1], Sb, G, g->part_vb[pi],
                               g->part_vb[pi + 1], Q.pcount);
             }
-            if (!local) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
+            if (!local && g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
             uint32_t r = 1;
             for (;;) {
                 if (!local) {
@@ -992,27 +999,35 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                     r++;
                     continue;
                 }
-                // exchange: every rank ends the round with the elementwise min of all ranks' states
-                if (PK) TG_TRY(tg_comm_allreduce_min_u64(g->comm, (unsigned long long *)Q.st, (uint64_t)Sb * n, s));
-                else TG_TRY(tg_comm_allreduce_min_u32(g->comm, (uint32_t *)Q.st, (uint64_t)Sb * n, s));
+                // exchange: every rank (every logical partition's copy) ends the round with the
+                // elementwise min of all ranks' states
+                if (g->comm) {
+                    if (PK) TG_TRY(tg_comm_allreduce_min_u64(g->comm, (unsigned long long *)Q.st, slen, s));
+                    else TG_TRY(tg_comm_allreduce_min_u32(g->comm, (uint32_t *)Q.st, slen, s));
+                } else if (ncopy > 1) {
+                    TG_LAUNCH(k_state_min_exchange<PK>, (unsigned)std::min<uint64_t>((slen + 255) / 256, 148ull * 16), 256,
+                              0, s, Q.st, ncopy, slen);
+                }
                 uint32_t *fnext = ((r + 1) & 1) ? Q.fb[1] : Q.fb[0];
                 for (int pi = 0; pi < g->nparts; pi++)
                     TG_LAUNCH(k_part_frontier<PK>, grid, 256, 0, s, Q.st, Q.lat, fnext, Sb, G, g->part_vb[pi],
                               g->part_vb[pi + 1], Q.pcount);
-                TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
+                if (g->comm) TG_TRY(tg_comm_allreduce_sum_u32(g->comm, Q.pcount, 1, s));
                 r++;
                 rounds = r - 1;
             }
         }
         g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;
-        uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
-        uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : Q.pred_stage) : nullptr;
+        const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
+        uint32_t *o = out_dev ? out + (size_t)b0 * n : nullptr;
+        uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : pred) : nullptr;
+        TG_TRY(tg_sink_target(g, bi, !out_dev, pred && !pred_dev, &o, &pr, s));
         const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
         TG_LAUNCH(k_eat_extract<PK>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
                   (const uint32_t *)nullptr);
-        if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
-        if (pred && !pred_dev) TG_TRY_CUDA(cudaMemcpyAsync(pred + (size_t)b0 * n, Q.pred_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
+        TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n,
+                             (pred && !pred_dev) ? pred + (size_t)b0 * n : nullptr, (size_t)Sb * n * 4, s));
         if (g->opt_stats) {
             const uint64_t tw = (g->m + 31) / 32 + TG_MAXP + 1;
             TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, Q.touched, tw,
@@ -1025,6 +1040,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         }
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
+    TG_TRY(tg_sink_end(g));
     g->last.kernel_launches = g_tg_launches - launches0;
     return TG_OK;
 }

@@ -422,7 +422,7 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
     TG_TRY(tg_ensure_scratch(g, S, true));
     QueryScratch &Q = g->qs;
     const uint64_t n = g->n;
-    if (!out_dev && !Q.out_stage) TG_TRY(Q.arena.alloc((void **)&Q.out_stage, (uint64_t)Q.S * n * 4));
+    TG_TRY(tg_sink_begin(g, !out_dev, false));
     g->last = tg_query_stats{};
     const uint64_t launches0 = g_tg_launches;
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
@@ -433,12 +433,15 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
         else TG_TRY((spfp_rounds<false>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
         g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;
-        uint32_t *o = out_dev ? out + (size_t)b0 * n : Q.out_stage;
+        const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
+        uint32_t *o = out_dev ? out + (size_t)b0 * n : nullptr, *no_pred = nullptr;
+        TG_TRY(tg_sink_target(g, bi, !out_dev, false, &o, &no_pred, s));
         dim3 grid((unsigned)std::min<uint64_t>((n + 255) / 256, 1024), Sb);
         TG_LAUNCH(k_spfp_extract, grid, 256, 0, s, Q.vout, g->n, Q.srcs, o, g->relabeled ? g->perm : (const uint32_t *)nullptr);
-        if (!out_dev) TG_TRY_CUDA(cudaMemcpyAsync(out + (size_t)b0 * n, Q.out_stage, (size_t)Sb * n * 4, cudaMemcpyDeviceToHost, s));
+        TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n, nullptr, (size_t)Sb * n * 4, s));
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
+    TG_TRY(tg_sink_end(g));
     g->last.kernel_launches = g_tg_launches - launches0;
     return TG_OK;
 }

@@ -90,10 +90,6 @@ struct ChainGraph {
     unsigned long long *sc_sumw = nullptr;
     uint32_t *sc_elapsed = nullptr;
     uint32_t *chain_first = nullptr;
-    // time-ordered edge list (the sweep schedule's topological order of the expanded DAG):
-    // te int4[m] = {u, v, t, arrival} sorted by (t, input order), te_id[m] = edge id
-    int4 *te = nullptr;
-    uint32_t *te_id = nullptr;
 };
 
 // Device-side round control of one GAC loop (no host round trip per round):
@@ -116,6 +112,7 @@ struct QueryScratch {
     uint64_t nnodes = 0;
     bool nodes_state = false;  // SP/FP node-state arrays present
     void *st = nullptr;  // [n][S] packed u64 (time << 32 | pred), or u32 time when no pred is requested
+    uint32_t st_copies = 1;  // option "exchange" with logical partitions: one private state copy each
     uint32_t *act = nullptr;           // [S][n] last activated time
     uint32_t stamp = 0;                // SP/FP frontier dedupe stamps handed out (host counter; marks start at 0)
     uint32_t *mark = nullptr;          // [S][n] (EAT) or [S][nnodes] (SP/FP) frontier dedupe stamp
@@ -142,7 +139,7 @@ struct QueryScratch {
     uint32_t *srcs_int = nullptr;  // [S] the same in the engine's internal vertex order
     unsigned long long *relax_cnt = nullptr;  // [S] + distinct-slot count
     uint32_t *touched = nullptr;              // stats: slots relaxed by any query of the sub-batch
-    uint32_t *out_stage = nullptr, *pred_stage = nullptr;  // [S][n] when out is host memory
+    uint32_t *out_stage[2] = {nullptr, nullptr}, *pred_stage[2] = {nullptr, nullptr};  // [S][n] x 2 for host outputs
     DevArena arena;
 };
 
@@ -176,7 +173,6 @@ struct tg_graph {
     int comm_mode = 0;              // 0 replicated (source sharding), 1 vertex range
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
-    void *sweep = nullptr;  // query_sweep.cu scratch (SweepScratch)
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
     // options
     int64_t opt_sub_batch = 0;
@@ -184,13 +180,13 @@ struct tg_graph {
     int64_t opt_shortcuts = 1;
     int64_t opt_round_group = 8;  // GAC rounds launched per host convergence check
     int opt_mirror = 1;
-    int64_t opt_exp = 0;
-    int64_t opt_packed_state = 0;
-    int64_t opt_sweep_struct = 0;  // build the time-ordered edge list (sweep schedule) in tg_build_chains
-    int64_t opt_engine = 0;        // EAT/LD/REACH schedule: 0 = automatic (GAC), 1 = GAC rounds, 2 = time sweep
-    int64_t opt_sweep_part = 0;    // sweep: edges per time partition (0 = automatic)  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
-    int64_t opt_walk_min = 6;  // chains with fewer edges are not walked (RemoveChain threshold, build time)       // diagnostic kernel variants (timing experiments only)        // build the LD mirror in tg_build_chains (else on the first LD query)
+    int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
+    int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
+    int64_t opt_walk_min = 6;  // chains with fewer edges are not walked (RemoveChain threshold, build time)
     bool mirror_built = false;
+    // host-memory outputs: copy stream and per-staging-buffer events (host_out.cu)
+    cudaStream_t cstream = nullptr;
+    cudaEvent_t ev_x[2] = {nullptr, nullptr}, ev_c[2] = {nullptr, nullptr};
     // last query statistics
     tg_query_stats last{};
     uint64_t *last_relax = nullptr;  // host, per query
@@ -226,7 +222,17 @@ tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cuda
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,
                              int dirs);  // dirs: bit 0 forward, bit 1 mirror
 
-tg_status tg_ensure_scratch_srcs(tg_graph *g, uint32_t S);  // sources + staging only
+// Host-memory outputs (host_out.cu).  Sub-batch b is extracted into staging buffer
+// b & 1 on the query stream and copied to the host on a copy stream, so the copy of
+// sub-batch b overlaps the rounds of sub-batch b + 1.  tg_sink_target waits (on the
+// query stream) until buffer b & 1's previous copy has finished; tg_sink_flush issues
+// the copy; tg_sink_end waits for the last copies before tg_query returns.
+tg_status tg_sink_begin(tg_graph *g, bool out_host, bool pred_host);
+tg_status tg_sink_target(tg_graph *g, uint32_t b, bool out_host, bool pred_host, uint32_t **o, uint32_t **pr,
+                         cudaStream_t s);
+tg_status tg_sink_flush(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *host_pred, size_t bytes, cudaStream_t s);
+tg_status tg_sink_end(tg_graph *g);
+void tg_sink_destroy(tg_graph *g);
 tg_status tg_run_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                        uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
 

@@ -378,9 +378,14 @@ def test_logical_partitions_c1(tg):
         g.query("sp", [0], (0, 10))  # partitioned graphs answer EAT/LD/REACH only
 
 
-def test_nccl_comm_world1_vertex_range(tg):
-    """The NCCL path of mode 1 with world = 1 (one GPU available): communicator
-    creation, attach, per-round ncclAllReduce(min) and the count reduction."""
+@pytest.mark.parametrize("exchange", [0, 1])
+def test_nccl_comm_world1_vertex_range(tg, exchange):
+    """Mode 1 through an NCCL communicator of world 1 (one GPU available).  With
+    exchange = 1 the rank runs the cross-rank round exactly as in a multi-GPU run:
+    per-round ncclAllReduce(min) of the states, k_part_frontier (next frontier derived
+    from the exchanged state) and ncclAllReduce(sum) of the frontier count.  With
+    exchange = 0 a world of 1 shares its state like logical partitions (no NCCL call
+    in the round loop)."""
     import torch
     from paper_conf_asplos_0003wh0dhwy0lyl25_b200 import distributed as tgd
     ge = tgsynth.make_graph("C2", scale_shift=-6)
@@ -388,14 +393,65 @@ def test_nccl_comm_world1_vertex_range(tg):
     comm = tgd.make_comm(0, 1, 0)
     f = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.uint32).view(np.int32)).cuda()
     g = tg.Graph(n, f(u), f(v), f(t), f(d), device=0)
+    g.set_option("exchange", exchange)
     tg.tg_graph_attach_comm(g.h, comm, 1)
     g.build()
     og = oracle.Graph(n, u, v, t, d)
     srcs = tgsynth.config_sources("C2", ge, k=8)
     _check_rows(tg, g, og, "eat", srcs, (0, 10**9))
     _check_rows(tg, g, og, "ld", srcs, (0, 10**9))
+    _check_values(tg, g, og, "reach", srcs, (1000, 40000))
     g.close()
     tg.tg_comm_destroy(comm)
+
+
+@pytest.mark.parametrize("parts", [2, 3, 8])
+def test_exchange_partitions_random(tg, parts):
+    """The multi-rank vertex-range algorithm (P:L313 rounds) inside one
+    process: every logical partition relaxes its own chains into a PRIVATE state copy,
+    the copies are combined by an elementwise min after every round (what
+    ncclAllReduce(min) leaves on every rank), and each partition derives its next
+    frontier from the combined state (k_part_frontier).  Bit-exact with preds and
+    first-touch W, packed and u32 states."""
+    for seed in range(5):
+        rng = np.random.default_rng(seed + 177)
+        n, m = 300 + 50 * seed, 4000
+        u = rng.integers(0, n, m).astype(np.uint32); v = rng.integers(0, n, m).astype(np.uint32)
+        t = rng.integers(0, 300, m).astype(np.uint32); lam = rng.integers(1, 6, m).astype(np.uint32)
+        g = _gpu_graph(tg, n, u, v, t, lam, partitions=parts, exchange=1, stats=1, sub_batch=37)
+        og = oracle.Graph(n, u, v, t, lam)
+        srcs = [int(x) for x in rng.choice(n, 40, replace=False)]
+        for win in [(0, 10**6), (30, 200)]:
+            for p in ("eat", "ld", "reach"):
+                _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
+                _check_values(tg, g, og, p, srcs, win)
+        g.close()
+
+
+def test_exchange_partitions_c1(tg):
+    ge = tgsynth.make_graph("C1")
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d, w)
+    for parts in (2, 8):
+        g = _gpu_graph(tg, n, u, v, t, d, w, partitions=parts, exchange=1)
+        for win in tgsynth.CONFIGS["C1"]["windows"]:
+            _check_rows(tg, g, og, "eat", [0, 5, 99], win)
+            _check_rows(tg, g, og, "ld", [0, 5], win)
+            _check_values(tg, g, og, "eat", [0, 7], win)
+        g.close()
+
+
+def test_exchange_partitions_c5_eighth(tg):
+    """C5-shaped (Chung-Lu, lambda ~ U[1,15]) at 1/8 scale, 8 partitions, single-source
+    EAT as in the C5 configuration: values and preds against the oracle."""
+    ge = tgsynth.make_graph("C5", device="cuda", scale_shift=-3)
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d)
+    srcs = tgsynth.config_sources("C5", ge, k=2)
+    g = _gpu_graph(tg, n, u, v, t, d, partitions=8, exchange=1, mirror=0)
+    _check_rows(tg, g, og, "eat", srcs, (0, 10**9))
+    _check_values(tg, g, og, "eat", srcs, (0, 10**9))
+    g.close()
 
 
 # --------------------------------------------------------------------------- state width / schedules
@@ -434,30 +490,3 @@ def test_unpacked_state_c2_small(tg):
     for win in tgsynth.CONFIGS["C2"]["windows"]:
         _check_values(tg, g, og, "eat", srcs, win)
         _check_values(tg, g, og, "ld", srcs[:16], win)
-
-
-@pytest.mark.parametrize("part", [3, 64, 0])
-def test_sweep_engine_random(tg, part):
-    """Time-partitioned sweep schedule (engine 2): values, preds (packed words) and the
-    post-hoc work count W equal the oracle; tiny partitions force many fixup rounds."""
-    for seed in range(6):
-        n, u, v, t, lam, w = tgsynth.tiny_random(seed + 4200, n_max=70, m_max=1200, t_max=50, lam_max=5)
-        g = _gpu_graph(tg, n, u, v, t, lam, w, sweep_struct=1, engine=2, sweep_part=part, stats=1)
-        og = oracle.Graph(n, u, v, t, lam, w)
-        srcs = list(range(min(n, 40)))
-        for win in [(0, 10**6), (4, 30), (7, 7)]:
-            for p in ("eat", "ld", "reach"):
-                _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
-                _check_values(tg, g, og, p, srcs, win)
-
-
-def test_sweep_engine_c2_small(tg):
-    ge = tgsynth.make_graph("C2", scale_shift=-4)
-    n, u, v, t, d, w = ge.numpy()
-    og = oracle.Graph(n, u, v, t, d, w)
-    srcs = tgsynth.config_sources("C2", ge)
-    for part in (4096, 0):
-        g = _gpu_graph(tg, n, u, v, t, d, w, sweep_struct=1, engine=2, sweep_part=part)
-        for win in tgsynth.CONFIGS["C2"]["windows"]:
-            _check_values(tg, g, og, "eat", srcs, win)
-            _check_rows(tg, g, og, "ld", srcs[:8], win)

@@ -348,3 +348,15 @@ def test_c1_scale_runs():
     assert (A != NONE).sum() > 1000 and W > 0.5 * len(u)
     off, ce = oracle.chains(g)
     assert off[-1] == len(u)
+
+
+def test_time_order_is_stable_sort():
+    """The oracle's counting sort (oracle_time_order) is the stable sort by t of P:L123's
+    time order: identical to numpy's stable argsort, ties (many equal t) in input order,
+    times spanning both 16-bit digits."""
+    rng = np.random.default_rng(5)
+    for m, hi in [(0, 1), (1, 5), (1000, 4), (50_000, 1 << 16), (50_000, 1 << 31), (20_000, 70_000)]:
+        t = rng.integers(0, hi, m).astype(np.uint32)
+        z = np.zeros(m, np.uint32)
+        g = oracle.Graph(4, z, z, t, z + 1)
+        np.testing.assert_array_equal(g.order, np.argsort(t, kind="stable"))

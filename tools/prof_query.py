@@ -21,13 +21,9 @@ ap.add_argument("--k", type=int, default=64)
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--sub-batch", type=int, default=0)
 ap.add_argument("--shortcuts", type=int, default=1)
-ap.add_argument("--exp", type=int, default=0)
 ap.add_argument("--walk-min", type=int, default=0)
 ap.add_argument("--relabel", type=int, default=1)
 ap.add_argument("--stats", type=int, default=0)
-ap.add_argument("--sweep-part", type=int, default=0)
-ap.add_argument("--engine", type=int, default=0)
-ap.add_argument("--sweep-struct", type=int, default=0)
 a = ap.parse_args()
 
 ge = tgsynth.make_graph(a.config, device="cuda")
@@ -35,17 +31,13 @@ cfg = tgsynth.CONFIGS[a.config]
 w = ge.w if cfg["kind"] == "wikitalk" else None
 g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, w, device=0)
 g.set_option("relabel", a.relabel)
-g.set_option("sweep_struct", a.sweep_struct or int(a.engine == 2))
 if a.walk_min:
     g.set_option("walk_min", a.walk_min)
 g.build()
 if a.sub_batch:
     g.set_option("sub_batch", a.sub_batch)
 g.set_option("shortcuts", a.shortcuts)
-g.set_option("exp", a.exp)
 g.set_option("stats", a.stats)
-g.set_option("sweep_part", a.sweep_part)
-g.set_option("engine", a.engine)
 src = tgsynth.config_sources(a.config, ge, k=a.k)
 win = cfg["windows"][0]
 out = torch.empty((len(src), ge.n), dtype=torch.int32, device="cuda")
