@@ -559,18 +559,23 @@ def run_reference(a, rank, world):
     del ge
     t_sort = _oracle_preprocess_seconds(og)
     cores = a.cpu_threads or os.cpu_count() or 1
-    srcs = [job[i % len(job)] for i in range(a.warmup + a.steps)]
-    if a.warmup:
-        oracle_allcore(og, problems, srcs[:a.warmup], win, cores)
-    wall, per = oracle_allcore(og, problems, srcs[a.warmup:], win, cores)
+    # the K timed steps are spread over the threads in whole waves (at least one query per
+    # thread, so every core works); the warm-up is one wave of min(W, cores) queries
+    n_timed = -(-max(a.steps, cores) // cores) * cores
+    n_warm = min(a.warmup, cores)
+    srcs = [job[i % len(job)] for i in range(n_warm + n_timed)]
+    if n_warm:
+        oracle_allcore(og, problems, srcs[:n_warm], win, cores)
+    wall, per = oracle_allcore(og, problems, srcs[n_warm:], win, cores)
     q = len(per) / wall
     k_job = len(job) * len(problems)
     value = k_job / (t_sort + k_job / q)
-    sample = (f"{a.steps} timed steps (+{a.warmup} warm-up), each one source x ({'+'.join(problems)}) oracle "
-              f"scans, run one per thread on {cores} threads: {wall:.2f} s = {q:.3f} q/s; time sort "
+    sample = (f"{n_timed} timed oracle queries ({a.steps} steps rounded up to whole waves of {cores} threads; "
+              f"+{n_warm} warm-up), each one source x ({'+'.join(problems)}) scans, one per thread: "
+              f"{wall:.2f} s = {q:.3f} q/s; time sort "
               f"{t_sort:.2f} s once; value = the job's {k_job} queries / (sort + queries at that rate)")
     return {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT,
-            "n_gpus": world, "steps": a.steps, "warmup": a.warmup, "ms_per_step": wall / a.steps * 1e3,
+            "n_gpus": world, "steps": a.steps, "warmup": a.warmup, "ms_per_step": wall / n_timed * 1e3,
             "higher_is_better": True, "scaling": "strong" if a.scaling == "strong" else "weak",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": wl},

@@ -111,7 +111,7 @@ cudaError_t tg_pinned_get(void **p) {
             return cudaSuccess;
         }
     }
-    return cudaMallocHost(p, 4096);
+    return cudaMallocHost(p, 8192);  // >= TG_MAXP RoundCtl records
 }
 
 void tg_pinned_put(void *p) {
@@ -165,6 +165,8 @@ tg_status tg_validate_edges(tg_graph *g, cudaStream_t s);
 tg_status tg_build_mirror(tg_graph *g, cudaStream_t s);
 tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                             uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
+tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
+                            bool out_dev, cudaStream_t s);
 tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                       bool out_dev, cudaStream_t s);
 tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
@@ -393,6 +395,7 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
         }
         return tg_run_eat_partitioned(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     }
+    if (p == TG_REACH && !pred) return tg_run_reach_bits(g, sources, n_sources, w, out, out_dev, s);
     if (p == TG_EAT || p == TG_LD || p == TG_REACH) {
         return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     }
@@ -406,6 +409,8 @@ void tg_graph_destroy(tg_graph *g) {
     tg_sink_destroy(g);
     g->qs.arena.free_all();
     tg_pinned_put(g->qs.h_ctr);
+    g->rs.arena.free_all();
+    tg_pinned_put(g->rs.h_ctr);
     g->arena.free_all();
     delete[] g->last_relax;
     delete g;

@@ -98,10 +98,10 @@ __device__ __forceinline__ RoundV round_view(const EatP &P) {
     R.fin = (r & 1) ? P.fb1 : P.fb0;
     R.fout = (r & 1) ? P.fb0 : P.fb1;
     R.fin_n = 0;
-    R.rec_cnt = &P.ctl->cnt[r & 3][0];
-    R.big_cnt = &P.ctl->cnt[r & 3][1];
-    R.ch_cnt = &P.ctl->cnt[r & 3][2];
-    R.words_cnt = &P.ctl->cnt[r & 3][3];
+    R.rec_cnt = &P.ctl->cnt[r & (TG_RING - 1)][0];
+    R.big_cnt = &P.ctl->cnt[r & (TG_RING - 1)][1];
+    R.ch_cnt = &P.ctl->cnt[r & (TG_RING - 1)][2];
+    R.words_cnt = &P.ctl->cnt[r & (TG_RING - 1)][3];
     return R;
 }
 
@@ -109,7 +109,7 @@ __device__ __forceinline__ RoundV round_view(const EatP &P) {
 // clears the next round's (nobody touches them before that round; the host reads
 // only the last round of a group, which is cleared again three rounds later).
 __device__ __forceinline__ void clear_next_round(const EatP &P) {
-    if (blockIdx.x == 0 && threadIdx.x < 4) P.ctl->cnt[(P.round + 1) & 3][threadIdx.x] = 0;
+    if (blockIdx.x == 0 && threadIdx.x < 4) P.ctl->cnt[(P.round + 1) & (TG_RING - 1)][threadIdx.x] = 0;
 }
 
 // Layouts interleave the S queries of a sub-batch (query index fastest):
@@ -464,7 +464,7 @@ __global__ void k_eat_init(void *st, uint32_t n, uint32_t G, const uint32_t *src
         if (push) atomicOr(fb1 + (size_t)x * G + (q >> 5), 1u << (q & 31));
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
-        for (int i = 0; i < 4; i++)
+        for (int i = 0; i < TG_RING; i++)
             for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
         ctl->round = 1;
         ctl->done_blocks = 0;
@@ -633,7 +633,7 @@ __global__ void k_popcount(const uint32_t *__restrict__ w, uint64_t nw, unsigned
 }
 
 __global__ void k_ctl_reset(RoundCtl *ctl) {
-    for (int i = 0; i < 4; i++)
+    for (int i = 0; i < TG_RING; i++)
         for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
     ctl->round = 1;
     ctl->done_blocks = 0;
@@ -787,11 +787,18 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
                 float ms[3] = {0, 0, 0};
                 for (int i = 0; i < 3; i++) cudaEventElapsedTime(&ms[i], tev[i], tev[i + 1]);
                 fprintf(stderr, "[tg] S=%u round %u: frontier words %u big-chunks %u chain-walks %u | activate %.3f "
-                        "big %.3f chain %.3f ms\n", S, last, h->cnt[last & 3][3], h->cnt[last & 3][1],
-                        h->cnt[last & 3][2], ms[0], ms[1], ms[2]);
+                        "big %.3f chain %.3f ms\n", S, last, h->cnt[last & (TG_RING - 1)][3], h->cnt[last & (TG_RING - 1)][1],
+                        h->cnt[last & (TG_RING - 1)][2], ms[0], ms[1], ms[2]);
             }
             // a round whose frontier bitmap was empty ends the loop (it did no work)
-            if (h->cnt[last & 3][3] == 0) { rounds = last - 1; break; }
+            if (h->cnt[last & (TG_RING - 1)][3] == 0) {
+                // the group's first round that consumed no frontier word did no work
+                uint32_t first = last;
+                for (uint32_t q = last + 1 - (uint32_t)group; q < last; q++)
+                    if (q >= 1 && h->cnt[q & (TG_RING - 1)][3] == 0) { first = q; break; }
+                rounds = first - 1;
+                break;
+            }
             if (r > 1000000) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
         }
         if (trace)
@@ -994,7 +1001,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                     TG_TRY_CUDA(cudaStreamSynchronize(s));
                     const RoundCtl *h = (const RoundCtl *)Q.h_ctr;
                     uint64_t words = 0;
-                    for (int pi = 0; pi < g->nparts; pi++) words += h[pi].cnt[r & 3][3];
+                    for (int pi = 0; pi < g->nparts; pi++) words += h[pi].cnt[r & (TG_RING - 1)][3];
                     if (words == 0) { rounds = r - 1; break; }
                     r++;
                     continue;

@@ -92,17 +92,18 @@ struct ChainGraph {
     uint32_t *chain_first = nullptr;
 };
 
-// Device-side round control of one GAC loop (no host round trip per round):
-// round r reads frontier buffer r&1 with count cnt[r&3][0], appends to buffer
-// (r+1)&1 / cnt[(r+1)&3][0]; cnt[r&3][1..2] count big chunks / chain walks.  The
-// last block of a round's last kernel advances `round`, bumps `stamp` and clears
-// the ring slots the next round will write.
+// Device-side round control of one GAC loop (no host round trip per round): a ring
+// of per-round counters, round r at cnt[r % TG_RING]; the first kernel of a round
+// clears a later round's slot.  The ring is deeper than the host's round group, so
+// after a group the host sees every round of it (the first round whose frontier was
+// empty is the round count).
+#define TG_RING 16
 struct RoundCtl {
     uint32_t round;
     uint32_t stamp;
     uint32_t done_blocks;
     uint32_t pad;
-    uint32_t cnt[4][4];
+    uint32_t cnt[TG_RING][4];
 };
 
 struct QueryScratch {
@@ -143,6 +144,23 @@ struct QueryScratch {
     DevArena arena;
 };
 
+// Bit-lane reachability scratch (query_reach.cu): one u64 word per departure node and
+// per vertex for a sub-batch of up to 64 sources.
+struct ReachScratch {
+    uint64_t nn = 0, n = 0;
+    unsigned long long *R = nullptr, *VR = nullptr;
+    uint32_t *D[2] = {nullptr, nullptr}, *dmin[2] = {nullptr, nullptr}, *dmax[2] = {nullptr, nullptr};
+    uint32_t *vf[2] = {nullptr, nullptr};
+    uint4 *bigq = nullptr;
+    uint64_t bigcap = 0;
+    struct RoundCtl *ctl = nullptr;
+    unsigned long long *cnt = nullptr;
+    uint32_t *srcs = nullptr;
+    uint32_t *stage[1] = {nullptr};
+    uint32_t *h_ctr = nullptr;
+    DevArena arena;
+};
+
 #define TG_MAXP 16  // logical vertex-range partitions per process (tests / one rank's share)
 
 struct tg_comm;  // comm.cu: NCCL communicator (loaded with dlopen)
@@ -173,6 +191,7 @@ struct tg_graph {
     int comm_mode = 0;              // 0 replicated (source sharding), 1 vertex range
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
+    ReachScratch rs;
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
     // options
     int64_t opt_sub_batch = 0;

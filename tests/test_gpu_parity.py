@@ -490,3 +490,64 @@ def test_unpacked_state_c2_small(tg):
     for win in tgsynth.CONFIGS["C2"]["windows"]:
         _check_values(tg, g, og, "eat", srcs, win)
         _check_values(tg, g, og, "ld", srcs[:16], win)
+
+
+# --------------------------------------------------------------------------- bit-lane reachability (f2)
+def _check_reach(tg, g, og, sources, win, host=False):
+    import torch
+    if host:
+        out = torch.empty((len(sources), og.n), dtype=torch.int32)
+        tg.tg_query(g.h, tg.TG_REACH, sources, win, out)
+    else:
+        out = g.query("reach", sources, win)
+    out = tg.as_u32(out)
+    for r, x in enumerate(sources):
+        np.testing.assert_array_equal(out[r], oracle.reach(og, x, *win), err_msg=f"REACH x={x} win={win}")
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_reach_bitlane_random(tg, seed):
+    """pred = NULL runs TG_REACH on the bit-lane engine (64 sources per u64 word over
+    the departure nodes): equal to the oracle's reachability
+    for 100 sources (two words), several windows incl. alpha == omega."""
+    n, u, v, t, lam, w = tgsynth.tiny_random(seed + 6100, n_max=120, m_max=2500, t_max=60, lam_max=6)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    for opts in ({}, {"walk_min": 2}, {"relabel": 1}):
+        g = _gpu_graph(tg, n, u, v, t, lam, w, **opts)
+        srcs = list(range(min(n, 100)))
+        for win in [(0, 10**6), (5, 40), (7, 7), (20, 21)]:
+            _check_reach(tg, g, og, srcs, win)
+        g.close()
+
+
+def test_reach_bitlane_hubs_and_host(tg):
+    """A hub with thousands of departure nodes (long wait-edge scans, queued edge chunks),
+    long chains, duplicates and self-loops; host-memory output."""
+    rng = np.random.default_rng(61)
+    n = 700
+    parts = []
+    # hub 0: 6000 out-edges at distinct-ish times; chains 1 -> 2 -> ... -> 60 at increasing times
+    parts.append((np.zeros(6000), rng.integers(0, n, 6000), rng.integers(0, 3000, 6000), rng.integers(1, 4, 6000)))
+    parts.append((np.arange(1, 61), np.arange(2, 62), np.arange(1, 61) * 3, np.full(60, 2)))
+    parts.append((rng.integers(0, n, 9000), rng.integers(0, n, 9000), rng.integers(0, 3000, 9000),
+                  rng.integers(1, 9, 9000)))
+    parts.append((np.full(50, 5), np.full(50, 5), np.arange(50), np.ones(50)))  # self-loops
+    u, v, t, lam = (np.concatenate([p[i] for p in parts]).astype(np.uint32) for i in range(4))
+    og = oracle.Graph(n, u, v, t, lam)
+    g = _gpu_graph(tg, n, u, v, t, lam, walk_min=2)
+    srcs = [0, 1, 5] + [int(x) for x in rng.choice(n, 70, replace=False)]
+    for win in [(0, 10**6), (100, 2000)]:
+        _check_reach(tg, g, og, srcs, win)
+        _check_reach(tg, g, og, srcs[:9], win, host=True)
+    g.close()
+
+
+def test_reach_bitlane_c2_small(tg):
+    ge = tgsynth.make_graph("C2", scale_shift=-4)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d)
+    og = oracle.Graph(n, u, v, t, d)
+    srcs = tgsynth.config_sources("C2", ge)
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        _check_reach(tg, g, og, srcs, win)
+    g.close()

@@ -22,7 +22,7 @@ ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--sub-batch", type=int, default=0)
 ap.add_argument("--shortcuts", type=int, default=1)
 ap.add_argument("--walk-min", type=int, default=0)
-ap.add_argument("--relabel", type=int, default=1)
+ap.add_argument("--relabel", type=int, default=0)
 ap.add_argument("--stats", type=int, default=0)
 a = ap.parse_args()
 
@@ -31,6 +31,8 @@ cfg = tgsynth.CONFIGS[a.config]
 w = ge.w if cfg["kind"] == "wikitalk" else None
 g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, w, device=0)
 g.set_option("relabel", a.relabel)
+if a.problem != "ld":
+    g.set_option("mirror", 0)
 if a.walk_min:
     g.set_option("walk_min", a.walk_min)
 g.build()
