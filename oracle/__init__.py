@@ -13,6 +13,8 @@ Functions (all inputs are numpy uint32 edge arrays u, v, t, lam[, w]):
 * ``sp``    shortest path, P:L115 (dist = sum W_e), Pareto-list scan
 * ``fp``    fastest path, P:L114 (duration = end - start, reading A6), Pareto-list scan
 * ``reach`` reachability, P:L112 (= EAT reached)
+* ``lds``   single-source latest departure (reading R5), Pareto-list scan
+* ``topk`` / ``summary``  top-K nearest / (reached, sum) of a row (f4), plain numpy
 * ``chains``     Alg. 1 chain partition of the transformed DAG
 * ``shortcuts``  Alg. 2 shortcut generation
 * ``mirror``     the reversed-time graph used by reading A5's identity (pins only)
@@ -58,6 +60,8 @@ def _load():
         lib.oracle_sp.argtypes = [u32, u64, P, P, P, P, P, P, u32, u32, u32, P]
         lib.oracle_fp.restype = ctypes.c_int
         lib.oracle_fp.argtypes = [u32, u64, P, P, P, P, P, u32, u32, u32, P]
+        lib.oracle_lds.restype = ctypes.c_int
+        lib.oracle_lds.argtypes = [u32, u64, P, P, P, P, P, u32, u32, u32, P]
         lib.oracle_chains.restype = i64
         lib.oracle_chains.argtypes = [u32, u64, P, P, P, P, P, P, P]
         lib.oracle_shortcuts.restype = None
@@ -156,6 +160,41 @@ def fp(g: Graph, x: int, alpha: int = 0, omega: int = 0x7FFFFFFE):
     if lib.oracle_fp(*g._args(), _p(g.order), x, alpha, omega, _p(out)) != 0:
         raise MemoryError
     return out
+
+
+def lds(g: Graph, x: int, alpha: int = 0, omega: int = 0x7FFFFFFE):
+    """Single-source latest departure (reading R5): for every v the latest departure
+    from x (first edge, >= alpha) of a legal path reaching v by omega; x itself: omega."""
+    _check_query(g, x, alpha, omega)
+    lib = _load()
+    out = np.empty(g.n, np.uint32)
+    if lib.oracle_lds(*g._args(), _p(g.order), x, alpha, omega, _p(out)) != 0:
+        raise MemoryError
+    return out
+
+
+def topk(row: np.ndarray, x: int, K: int):
+    """Top-K nearest of a query row: the K reached vertices v != x
+    with the smallest values, ties by vertex id; padded with (NONE, NONE).
+    Returns (vertices, values) as uint32[K]."""
+    row = np.asarray(row, np.uint32)
+    cand = np.nonzero(row != NONE)[0]
+    cand = cand[cand != x]
+    order = np.lexsort((cand, row[cand]))[:K]
+    vs = np.full(K, NONE, np.uint32)
+    vals = np.full(K, NONE, np.uint32)
+    vs[: len(order)] = cand[order]
+    vals[: len(order)] = row[cand[order]]
+    return vs, vals
+
+
+def summary(row: np.ndarray, x: int):
+    """Closeness-style row summary (f4, all-source batches): (number of reached
+    vertices v != x, sum of their values) -- exact integers."""
+    row = np.asarray(row, np.uint32)
+    mask = row != NONE
+    mask[x] = False
+    return int(mask.sum()), int(row[mask].astype(np.uint64).sum())
 
 
 def reach(g: Graph, x: int, alpha: int = 0, omega: int = 0x7FFFFFFE):

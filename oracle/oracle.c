@@ -233,6 +233,35 @@ int oracle_fp(uint32_t n, uint64_t m, const uint32_t *u, const uint32_t *v,
     return 0;
 }
 
+/* Single-SOURCE latest departure (the variant named by reading A5;
+ * DESIGN.md reading R5): out[v] = the latest start(P) (departure of the first edge,
+ * >= alpha) over legal paths P from x to v with end(P) <= omega; out[x] = omega;
+ * unreached = NONE.  The same one-pass scan as FP: the floor of L_u at t is
+ * the latest start among paths that are at u by time t (latest starts increase with
+ * the arrival in a Pareto list), so every relaxation offers its start to v. */
+int oracle_lds(uint32_t n, uint64_t m, const uint32_t *u, const uint32_t *v,
+               const uint32_t *t, const uint32_t *lam, const int64_t *order,
+               uint32_t x, uint32_t alpha, uint32_t omega, uint32_t *out) {
+    plist_t *Ls = (plist_t *)calloc(n, sizeof(plist_t));
+    if (!Ls) return -1;
+    for (uint32_t i = 0; i < n; i++) out[i] = ORACLE_NONE;
+    for (uint64_t k = 0; k < m; k++) {
+        int64_t e = order[k];
+        if (t[e] >= omega) break;
+        if (!valid_edge(t[e], lam[e], alpha, omega)) continue;
+        if (u[e] == x) fp_insert(&Ls[x], t[e], t[e]); /* a path may start here, now */
+        int64_t f = plist_floor(&Ls[u[e]], t[e]);
+        if (f < 0) continue;
+        uint32_t s = Ls[u[e]].p[f].val;
+        fp_insert(&Ls[v[e]], t[e] + lam[e], s);
+        if (out[v[e]] == ORACLE_NONE || s > out[v[e]]) out[v[e]] = s;
+    }
+    out[x] = omega;
+    for (uint32_t i = 0; i < n; i++) free(Ls[i].p);
+    free(Ls);
+    return 0;
+}
+
 /* ------------------------------------------------------------------------- */
 /* Alg. 1 "Chain-based Transformation on CPU" (§4.1) on the
  * transformed DAG of P:L123 / P:L204 as fixed by reading A11:

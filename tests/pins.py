@@ -57,6 +57,21 @@ def brute_force(n, u, v, t, lam, w, x, alpha, omega):
     return dict(eat=eat, eat_pred=pred, sp=sp, fp=fp)
 
 
+def brute_force_lds(n, u, v, t, lam, w, x, alpha, omega):
+    """Single-source latest departure (reading R5): for every v != x the max start over
+    legal walks x -> v in the window; x itself gets omega."""
+    L = [NONE] * n
+    L[x] = omega
+    for path in _walks_from(n, u, v, t, lam, w, x, alpha, omega):
+        y = int(v[path[-1]])
+        if y == x:
+            continue
+        st = int(t[path[0]])
+        if L[y] == NONE or st > L[y]:
+            L[y] = st
+    return L
+
+
 def brute_force_ld(n, u, v, t, lam, w, x, alpha, omega):
     """Latest departure towards target x (reading A5): for every v != x, the max
     start over legal walks v -> x in the window; succ = min first-edge id."""

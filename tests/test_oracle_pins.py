@@ -13,7 +13,7 @@ from scipy.sparse.csgraph import shortest_path
 
 import oracle
 import tgsynth
-from tests.pins import NONE, brute_force, brute_force_ld, gx_dp
+from tests.pins import NONE, brute_force, brute_force_ld, brute_force_lds, gx_dp
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "figure1.json")
 
@@ -124,6 +124,46 @@ def test_bruteforce_ld(block):
                 L, S, _ = oracle.ld(g, x, a, o)
                 bL, bS = brute_force_ld(n, u, v, t, lam, w, x, a, o)
                 assert L.tolist() == bL and S.tolist() == bS, (seed, x, a, o)
+
+
+@pytest.mark.parametrize("block", range(4))
+def test_bruteforce_lds(block):
+    """Single-source latest departure (f4, reading R5) against walk enumeration."""
+    for seed in range(block * 150, (block + 1) * 150):
+        n, u, v, t, lam, w = tgsynth.tiny_random(seed + 81000)
+        g = oracle.Graph(n, u, v, t, lam, w)
+        for (a, o) in _windows(seed):
+            for x in range(min(n, 3)):
+                assert oracle.lds(g, x, a, o).tolist() == brute_force_lds(n, u, v, t, lam, w, x, a, o), \
+                    (seed, x, a, o)
+
+
+def test_lds_closed_form_via_eat():
+    """LDS(v) = max departure time s >= alpha of x with EAT_{x,[s,omega]}(v) reached
+    (a path leaving x at s or later exists), for every v != x."""
+    for seed in range(200):
+        n, u, v, t, lam, w = tgsynth.tiny_random(seed + 9100, n_max=8, m_max=20, t_max=12)
+        g = oracle.Graph(n, u, v, t, lam, w)
+        for x in range(min(n, 2)):
+            a, o = 1, 14
+            best = np.full(n, NONE, np.int64)
+            for s in sorted({int(tt) for uu, tt in zip(u, t) if uu == x and tt >= a}):
+                A, _, _ = oracle.eat(g, x, s, o)
+                best[A != NONE] = s  # ascending s: the last reaching s wins
+            best[x] = o
+            np.testing.assert_array_equal(oracle.lds(g, x, a, o), best.astype(np.uint32))
+
+
+def test_topk_and_summary_plain():
+    """top-K / summary of a row: hand-checked cases (ties by vertex id, the source and
+    unreached excluded, padding)."""
+    row = np.array([0, 5, NONE, 3, 5, 1, 3], np.uint32)
+    vs, vals = oracle.topk(row, 0, 4)
+    assert vs.tolist() == [5, 3, 6, 1] and vals.tolist() == [1, 3, 3, 5]
+    vs, vals = oracle.topk(row, 5, 9)
+    assert vs.tolist() == [0, 3, 6, 1, 4, NONE, NONE, NONE, NONE]
+    assert vals.tolist()[:5] == [0, 3, 3, 5, 5]
+    assert oracle.summary(row, 0) == (5, 5 + 3 + 5 + 1 + 3)
 
 
 @pytest.mark.parametrize("block", range(4))
