@@ -64,7 +64,9 @@ typedef enum {
     TG_LD = 1,       /* latest departure from v of a path reaching the target by omega */
     TG_FASTEST = 2,  /* min duration(P) = end(P) - start(P), P:L114 (reading A6)       */
     TG_SHORTEST = 3, /* min dist(P) = sum of w_e, P:L115 / P:L185 (reading A7)         */
-    TG_REACH = 4     /* reachability P(u,v) != {}: out = 1 or 0                */
+    TG_REACH = 4,    /* reachability P(u,v) != {}: out = 1 or 0                */
+    TG_LD_SOURCE = 5 /* single-SOURCE latest departure (reading R5): the latest start(P)
+                        >= t_alpha of a path from the source reaching v by t_omega      */
 } tg_problem;
 
 typedef struct {
@@ -115,10 +117,13 @@ TG_API tg_status tg_build_chains(tg_graph *g);
  *   out         uint32[n_sources * n_vertices], row r = query sources[r]
  *               (host or device).  EAT: arrival time (source: t_alpha);
  *               LD: latest departure (target: t_omega); FASTEST / SHORTEST:
- *               min duration / distance (source: 0); REACH: 1 or 0.
+ *               min duration / distance (source: 0); REACH: 1 or 0;
+ *               LD_SOURCE: latest departure from the source (source: t_omega).
  *               Unreached vertices read TG_UNREACHED (REACH: 0).
  *   pred        NULL or uint32[n_sources * n_vertices] (host or device), only
- *               for TG_EAT / TG_LD / TG_REACH (else TG_ERR_INVALID).  EAT/REACH: the smallest
+ *               for TG_EAT / TG_LD / TG_REACH (else TG_ERR_INVALID).  TG_REACH with
+ *               pred == NULL runs on the bit-lane engine (64 sources per u64 word
+ *               over the departure nodes).  EAT/REACH: the smallest
  *               edge id among valid edges e=(u->v) with EAT(u) <= t_e and
  *               t_e + duration_e = EAT(v); LD: the smallest id among first
  *               edges of latest-departure paths (reading A9).  Source/target
@@ -130,6 +135,30 @@ TG_API tg_status tg_build_chains(tg_graph *g);
  */
 TG_API tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t n_sources,
                    tg_window w, uint32_t *out, uint32_t *pred, void *cuda_stream);
+
+/*
+ * tg_query_topk -- top-K nearest neighbours per source (the
+ * nearest-neighbour workload of P:L116 / P:L134): for source row r, the K vertices
+ * v != sources[r] reached by problem p with the smallest values, ascending by
+ * (value, vertex id).
+ *   p           TG_EAT, TG_FASTEST or TG_SHORTEST (else TG_ERR_INVALID).
+ *   K           >= 1.
+ *   out_vertex, out_value  uint32[n_sources * K] (host or device), row r at r * K;
+ *               rows with fewer than K reached vertices are padded with
+ *               TG_UNREACHED in both arrays.
+ * The rows are computed with tg_query (same errors) into temporary device memory.
+ */
+TG_API tg_status tg_query_topk(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t n_sources, tg_window w,
+                               uint32_t K, uint32_t *out_vertex, uint32_t *out_value, void *cuda_stream);
+
+/*
+ * tg_query_summary -- closeness-style summary of every source row (f4, all-source
+ * batches): out_count[r] = number of vertices v != sources[r] with a value (reached),
+ * out_sum[r] = the sum of those values (exact, uint64).  HOST arrays uint64[n_sources].
+ *   p           TG_EAT, TG_LD, TG_FASTEST, TG_SHORTEST or TG_LD_SOURCE.
+ */
+TG_API tg_status tg_query_summary(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t n_sources,
+                                  tg_window w, uint64_t *out_count, uint64_t *out_sum, void *cuda_stream);
 
 TG_API void tg_graph_destroy(tg_graph *g); /* NULL-safe */
 

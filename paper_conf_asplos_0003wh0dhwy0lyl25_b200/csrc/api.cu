@@ -362,7 +362,7 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
     if (!g) { tg_set_error("graph is NULL"); return TG_ERR_INVALID; }
     if (!g->built) { tg_set_error("tg_query before tg_build_chains"); return TG_ERR_STATE; }
     if (!sources || !out || n_sources == 0) { tg_set_error("sources/out NULL or n_sources == 0"); return TG_ERR_INVALID; }
-    if ((int)p < 0 || (int)p > TG_REACH) { tg_set_error("unknown problem"); return TG_ERR_INVALID; }
+    if ((int)p < 0 || (int)p > TG_LD_SOURCE) { tg_set_error("unknown problem"); return TG_ERR_INVALID; }
     if (pred && !(p == TG_EAT || p == TG_LD || p == TG_REACH)) {
         tg_set_error("pred is only defined for TG_EAT / TG_LD / TG_REACH");
         return TG_ERR_INVALID;

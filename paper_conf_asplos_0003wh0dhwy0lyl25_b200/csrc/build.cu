@@ -190,7 +190,7 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
                                 const uint32_t *__restrict__ tn, const uint32_t *__restrict__ node_of,
                                 int4 *__restrict__ slots, uint32_t *__restrict__ slot_w,
                                 uint32_t *__restrict__ slot_tn, uint32_t *__restrict__ occ_slot,
-                                uint2 *__restrict__ lc, int4 *__restrict__ sc,
+                                uint2 *__restrict__ occ_rec, uint2 *__restrict__ lc, int4 *__restrict__ sc,
                                 unsigned long long *__restrict__ sc_sumw, uint32_t *__restrict__ sc_elapsed,
                                 const uint32_t *__restrict__ id_map, uint32_t walk_min) {
     GRID_STRIDE(p, m) {
@@ -216,6 +216,10 @@ __global__ void k_chain_scatter(const uint32_t *__restrict__ head, const uint32_
             slot_w[s] = r.z;
             slot_tn[s] = tn[q];
             occ_slot[q] = s;
+            // occurrence-ordered {head, arrival | walked-chain flag}: the activation reads a
+            // vertex's newly usable out-edges as one contiguous run (P:L344's coalescing of
+            // the chains leaving one vertex) instead of index + scattered 16-byte slot
+            occ_rec[q] = make_uint2(r.x, r.y | (cw != TG_SINGLE ? 0x80000000u : 0u));
             sumw += r.z;  // GenerateShortcut: accumulate W_e (Alg. 2 line 5)
             s++;
             q = succ[q];
@@ -515,12 +519,13 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     TG_TRY(A.alloc((void **)&cg->slot_w, m * 4));
     TG_TRY(A.alloc((void **)&cg->slot_tn, m * 4));
     TG_TRY(A.alloc((void **)&cg->occ_slot, m * 4));
+    TG_TRY(A.alloc((void **)&cg->occ_rec, m * 8));
     TG_TRY(A.alloc((void **)&cg->lc, std::max<uint64_t>(L, 1) * 8));
     TG_TRY(A.alloc((void **)&cg->sc, std::max<uint64_t>(L, 1) * 16));
     TG_TRY(A.alloc((void **)&cg->sc_sumw, std::max<uint64_t>(L, 1) * 8));
     TG_TRY(A.alloc((void **)&cg->sc_elapsed, std::max<uint64_t>(L, 1) * 4));
     TG_LAUNCH(k_chain_scatter, blocks_for(m, 4), BT, 0, s, head, cidx, succ, m, cg->chain_first, chain_len, lidx, sid,
-              srec, rec, tn, node_of, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->lc, cg->sc,
+              srec, rec, tn, node_of, cg->slots, cg->slot_w, cg->slot_tn, cg->occ_slot, cg->occ_rec, cg->lc, cg->sc,
               cg->sc_sumw, cg->sc_elapsed, id_map, (uint32_t)std::max<int64_t>(2, g->opt_walk_min));
 
     for (void *p : {(void *)sid, (void *)d_cnt, (void *)tn, (void *)srec, (void *)rec, (void *)hub,
@@ -560,11 +565,15 @@ tg_status tg_relabel(tg_graph *g, cudaStream_t s) {
     return TG_OK;
 }
 
-tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cudaStream_t s) {
-    QueryScratch &Q = g->qs;
-    TG_TRY_CUDA(cudaMemcpyAsync(Q.srcs, sources, (uint64_t)k * 4, cudaMemcpyHostToDevice, s));
-    TG_LAUNCH(k_map_sources, 1, 64, 0, s, Q.srcs, k, g->relabeled ? g->perm : nullptr, Q.srcs_int);
+tg_status tg_load_sources_to(tg_graph *g, const uint32_t *sources, uint32_t k, uint32_t *d_srcs, uint32_t *d_int,
+                             cudaStream_t s) {
+    TG_TRY_CUDA(cudaMemcpyAsync(d_srcs, sources, (uint64_t)k * 4, cudaMemcpyHostToDevice, s));
+    TG_LAUNCH(k_map_sources, 1, 64, 0, s, d_srcs, k, g->relabeled ? g->perm : nullptr, d_int);
     return TG_OK;
+}
+
+tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cudaStream_t s) {
+    return tg_load_sources_to(g, sources, k, g->qs.srcs, g->qs.srcs_int, s);
 }
 
 tg_status tg_build_mirror(tg_graph *g, cudaStream_t s) {

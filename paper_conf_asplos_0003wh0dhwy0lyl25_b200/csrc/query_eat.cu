@@ -59,6 +59,7 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 
 struct EatP {
     const uint32_t *vnode_off, *node_t, *node_eoff, *occ_slot;
+    const uint2 *occ_rec;
     const int4 *slots;
     const uint2 *lc;
     const int4 *sc;
@@ -233,8 +234,21 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         uint32_t s = 0;
         int4 sl = make_int4(0, -1, 0, 0);
         if (p < pend) {
-            s = __ldg(P.occ_slot + p);
-            sl = tg_ld_slot(P.slots + s);
+            if (PK) {  // the pred needs the edge id: the full slot
+                s = __ldg(P.occ_slot + p);
+                sl = tg_ld_slot(P.slots + s);
+            } else {
+                // one coalesced 8-byte record per occurrence; only edges on walked chains
+                // (claims, shortcut, walk) need their slot
+                const uint2 r = __ldg(P.occ_rec + p);
+                if (r.y >> 31) {
+                    s = __ldg(P.occ_slot + p);
+                    sl = tg_ld_slot(P.slots + s);
+                } else {
+                    sl = make_int4((int)r.x, (int)r.y, 0, (int)TG_SINGLE);
+                    if (P.stats) s = __ldg(P.occ_slot + p);  // distinct-slot counter
+                }
+            }
         }
         // mask of queries for which edge pb+k is newly usable (lane k keeps its own):
         // each query lane's range as a row of block bits, transposed across the warp
@@ -752,6 +766,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     if (work) {
         EatP P{};
         P.vnode_off = cgr.vnode_off; P.node_t = cgr.node_t; P.node_eoff = cgr.node_eoff; P.occ_slot = cgr.occ_slot;
+        P.occ_rec = cgr.occ_rec;
         P.slots = cgr.slots; P.lc = cgr.lc; P.sc = cgr.sc;
         P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
         P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
@@ -967,6 +982,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 P.touched = Q.touched + bit_off;
                 bit_off += (cg.m + 31) / 32;
                 P.vnode_off = cg.vnode_off; P.node_t = cg.node_t; P.node_eoff = cg.node_eoff; P.occ_slot = cg.occ_slot;
+                P.occ_rec = cg.occ_rec;
                 P.slots = cg.slots; P.lc = cg.lc; P.sc = cg.sc;
                 P.ctl = Q.ctl + pi;
                 P.ub0 = g->part_vb[pi] * G;

@@ -252,6 +252,7 @@ tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg
         TG_TRY(A.alloc((void **)&X.ctl, sizeof(RoundCtl)));
         TG_TRY(A.alloc((void **)&X.cnt, 64));
         TG_TRY(A.alloc((void **)&X.srcs, 64 * 4));
+        TG_TRY(A.alloc((void **)&X.srcs_int, 64 * 4));
         TG_TRY(A.alloc((void **)&X.stage[0], 64 * n * 4));
         TG_TRY_CUDA(tg_pinned_get((void **)&X.h_ctr));
     }
@@ -269,7 +270,7 @@ tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg
     uint64_t relax_total = 0, scans_total = 0;
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
-        TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
+        TG_TRY(tg_load_sources_to(g, sources + b0, Sb, X.srcs, X.srcs_int, s));
         TG_TRY_CUDA(cudaMemsetAsync(X.R, 0, std::max<uint64_t>(nn, 1) * 8, s));
         TG_TRY_CUDA(cudaMemsetAsync(X.VR, 0, n * 8, s));
         if (P.stats) TG_TRY_CUDA(cudaMemsetAsync(X.cnt, 0, 64, s));
@@ -277,7 +278,7 @@ tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg
         uint32_t rounds = 0;
         if (g->m > 0 && w.t_alpha < w.t_omega) {
             P.round = 0;  // init pushes into round 1's frontier
-            TG_LAUNCH(k_reach_init, 1, 64, 0, s, P, g->qs.srcs_int, Sb, w.t_alpha);
+            TG_LAUNCH(k_reach_init, 1, 64, 0, s, P, X.srcs_int, Sb, w.t_alpha);
             uint32_t r = 1;
             for (;;) {
                 for (int i = 0; i < group; i++, r++) {

@@ -108,7 +108,7 @@ __device__ __forceinline__ void push_node(const SpP &P, const RoundV &R, uint32_
 }
 
 // Walk the chain from slot s (entered with head-node value cur).
-template <bool FP>
+template <int MODE>
 __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s, uint32_t s_end, uint32_t cur) {
     uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
     uint32_t *vo = P.vout + (size_t)q * P.n;
@@ -118,9 +118,12 @@ __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s,
         if (arr > P.omega) return;
         uint32_t cand;
         uint32_t val;
-        if (FP) {
+        if (MODE == 1) {
             cand = cur;                          // latest start is preserved along the path
             val = arr - (0xFFFFFFFEu - cur);     // duration = end - start (reading A6)
+        } else if (MODE == 2) {
+            cand = cur;                          // LDS: the latest start reaching v (key = ~LS)
+            val = cur;
         } else {
             cand = cur + __ldg(P.slot_w + s);    // Propagate: src + w
             val = cand;
@@ -136,7 +139,7 @@ __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s,
     }
 }
 
-template <bool FP>
+template <int MODE>
 __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_t q, uint32_t p) {
     const uint32_t s = __ldg(P.occ_slot + p);
     const uint32_t j = __ldg(P.occ_node + p);
@@ -155,9 +158,12 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_
             if ((uint32_t)scv.y <= P.omega) {
                 const uint32_t tn = __ldg(P.slot_tn + s_end - 1);
                 uint32_t cand;
-                if (FP) {
+                if (MODE == 1) {
                     cand = cur;
                     atomicMin(P.vout + (size_t)q * P.n + scv.x, (uint32_t)scv.y - (0xFFFFFFFEu - cur));
+                } else if (MODE == 2) {
+                    cand = cur;
+                    atomicMin(P.vout + (size_t)q * P.n + scv.x, cur);
                 } else {
                     cand = cur + (uint32_t)__ldg(P.sc_sumw + l);
                     atomicMin(P.vout + (size_t)q * P.n + scv.x, cand);
@@ -169,10 +175,10 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_
             }
         }
     }
-    spfp_walk<FP>(P, R, q, s, s_end, cur);
+    spfp_walk<MODE>(P, R, q, s, s_end, cur);
 }
 
-template <bool FP>
+template <int MODE>
 __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
     const RoundV R = round_view(P);
     clear_later_rounds(P);
@@ -209,9 +215,13 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
                 // (that node's own value is being propagated past it)
                 const uint32_t nseg = (vend - jend + WAIT_SEG - 1) / WAIT_SEG;
                 const uint32_t k = atomicAdd(R.wait_cnt, nseg);
+                // all or nothing: a partly queued walk would let its first segments write d
+                // into the nodes the retry walk starts from
+                const bool fits = (uint64_t)k + nseg <= P.waitcap;
                 for (uint32_t c = 0; c < nseg && k + c < P.waitcap; c++)
-                    P.waitq[k + c] = make_uint4(q, jend + c * WAIT_SEG, min(vend, jend + (c + 1) * WAIT_SEG), d);
-                if (k + nseg > P.waitcap) push_node(P, R, q, jend - 1);  // queue full: continue next round
+                    P.waitq[k + c] = fits ? make_uint4(q, jend + c * WAIT_SEG, min(vend, jend + (c + 1) * WAIT_SEG), d)
+                                          : make_uint4(q, vend, vend, d);  // reserved, empty
+                if (!fits) push_node(P, R, q, jend - 1);  // queue full: continue next round
             }
             e0 = __ldg(P.node_eoff + j);
             cnt = __ldg(P.node_eoff + jend) - e0;
@@ -222,7 +232,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             for (uint32_t c = 0; c < nch; c++) {
                 const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
                 if (k + c < P.bigcap) P.bigq[k + c] = make_uint4(q, b0, b1, 0);
-                else for (uint32_t p = b0; p < b1; p++) spfp_edge<FP>(P, R, q, p);
+                else for (uint32_t p = b0; p < b1; p++) spfp_edge<MODE>(P, R, q, p);
             }
             cnt = 0;
         }
@@ -246,7 +256,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
             const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
             const uint32_t oq = __shfl_sync(0xffffffffu, q, own);
-            if (g < total) spfp_edge<FP>(P, R, oq, oe0 + (g - oex));
+            if (g < total) spfp_edge<MODE>(P, R, oq, oe0 + (g - oex));
         }
     }
 }
@@ -256,7 +266,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
 // out-edges are queued as chunks for k_spfp_big of the same round.  Nodes past the
 // first non-improving one that still improved (legal: waiting is transitive) are
 // pushed to the next frontier.
-template <bool FP>
+template <int MODE>
 __global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
     const RoundV R = round_view(P);
     const uint32_t NW = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.wait_cnt, P.waitcap);
@@ -293,13 +303,13 @@ __global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
             for (uint32_t cc = lane; cc < nch; cc += 32) {
                 const uint32_t b0 = e0 + cc * CHUNK, b1 = min(e1, b0 + CHUNK);
                 if (k + cc < P.bigcap) P.bigq[k + cc] = make_uint4(q, b0, b1, 0);
-                else for (uint32_t pp = b0; pp < b1; pp++) spfp_edge<FP>(P, R, q, pp);
+                else for (uint32_t pp = b0; pp < b1; pp++) spfp_edge<MODE>(P, R, q, pp);
             }
         }
     }
 }
 
-template <bool FP>
+template <int MODE>
 __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
     const RoundV R = round_view(P);
     const uint32_t B = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.big_cnt, P.bigcap);
@@ -308,7 +318,7 @@ __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
-        for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<FP>(P, R, c.x, p);
+        for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<MODE>(P, R, c.x, p);
     }
 }
 
@@ -319,7 +329,7 @@ __global__ void k_spfp_ctl_init(RoundCtl *ctl) {
         for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
 }
 
-template <bool FP>
+template <int MODE>
 __global__ void k_spfp_init(SpP P, const uint32_t *srcs, uint32_t S) {
     const RoundV R = round_view(P);
     const uint32_t q = blockIdx.y;
@@ -330,24 +340,28 @@ __global__ void k_spfp_init(SpP P, const uint32_t *srcs, uint32_t S) {
     for (uint32_t j = j0 + blockIdx.x * blockDim.x + threadIdx.x; j < b; j += gridDim.x * blockDim.x) {
         const uint32_t tau = P.node_t[j];
         if (tau >= P.omega) break;
-        P.dnode[(size_t)q * P.nnodes + j] = FP ? (0xFFFFFFFEu - tau) : 0u;
+        P.dnode[(size_t)q * P.nnodes + j] = MODE ? (0xFFFFFFFEu - tau) : 0u;
         push_node(P, R, q, j);
     }
 }
 
+// SP / FP: the per-vertex minimum (source 0); LDS: latest start = ~key (source omega)
 __global__ void k_spfp_extract(const uint32_t *__restrict__ vout, uint32_t n, const uint32_t *__restrict__ srcs,
-                               uint32_t *__restrict__ out, const uint32_t *__restrict__ perm) {
+                               uint32_t *__restrict__ out, const uint32_t *__restrict__ perm, int lds,
+                               uint32_t omega) {
     const uint32_t q = blockIdx.y;
     const uint32_t src = srcs[q];  // caller's vertex ids
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
         const size_t i = (size_t)q * n + v;
-        out[i] = (v == src) ? 0u : vout[(size_t)q * n + (perm ? perm[v] : v)];
+        const uint32_t x = vout[(size_t)q * n + (perm ? perm[v] : v)];
+        if (lds) out[i] = (v == src) ? omega : (x == TG_NONE ? TG_NONE : 0xFFFFFFFEu - x);
+        else out[i] = (v == src) ? 0u : x;
     }
 }
 
 }  // namespace
 
-template <bool FP>
+template <int MODE>
 static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t omega, cudaStream_t s,
                              uint32_t *rounds_out) {
     QueryScratch &Q = g->qs;
@@ -372,7 +386,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
         P.round = 0;  // k_spfp_init pushes with round 0's view: output buffer 1, count cnt[1][0]
         P.stamp = ++Q.stamp;
         dim3 grid(64, Sb);  // a hub source has many departure nodes
-        TG_LAUNCH(k_spfp_init<FP>, grid, 256, 0, s, P, Q.srcs_int, Sb);
+        TG_LAUNCH(k_spfp_init<MODE>, grid, 256, 0, s, P, Q.srcs_int, Sb);
     }
     const uint32_t grid = tg_grid_persistent(8);
     const int group = (int)std::max<int64_t>(1, g->opt_round_group);
@@ -387,11 +401,11 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
             P.round = r;
             P.stamp = ++Q.stamp;
             if (trace) cudaEventRecord(tev[0], s);
-            TG_LAUNCH(k_spfp_activate<FP>, grid, QT, 0, s, P);
+            TG_LAUNCH(k_spfp_activate<MODE>, grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[1], s);
-            TG_LAUNCH(k_spfp_wait<FP>, grid, QT, 0, s, P);
+            TG_LAUNCH(k_spfp_wait<MODE>, grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[2], s);
-            TG_LAUNCH(k_spfp_big<FP>, grid, QT, 0, s, P);
+            TG_LAUNCH(k_spfp_big<MODE>, grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[3], s);
         }
         TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
@@ -402,7 +416,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
             for (int i = 0; i < 3; i++) cudaEventElapsedTime(&ms[i], tev[i], tev[i + 1]);
             const uint32_t last = r - 1;
             fprintf(stderr, "[tg] %s S=%u round %u: frontier %u wait-walks %u big-chunks %u | activate %.3f wait %.3f "
-                    "big %.3f ms\n", FP ? "FP" : "SP", Sb, last, h->cnt[last & 3][0], h->cnt[last & 3][2],
+                    "big %.3f ms\n", MODE == 0 ? "SP" : (MODE == 1 ? "FP" : "LDS"), Sb, last, h->cnt[last & 3][0], h->cnt[last & 3][2],
                     h->cnt[last & 3][1], ms[0], ms[1], ms[2]);
         }
         // r is the next round: its input count was written by the round just finished
@@ -417,7 +431,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
 
 tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                       bool out_dev, cudaStream_t s) {
-    const bool fp = (p == TG_FASTEST);
+    const int mode = (p == TG_FASTEST) ? 1 : (p == TG_LD_SOURCE ? 2 : 0);
     const uint32_t S = tg_pick_sub_batch(g, k, true);
     TG_TRY(tg_ensure_scratch(g, S, true));
     QueryScratch &Q = g->qs;
@@ -429,15 +443,17 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
         const uint32_t Sb = std::min(S, k - b0);
         TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
         uint32_t rounds = 0;
-        if (fp) TG_TRY((spfp_rounds<true>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
-        else TG_TRY((spfp_rounds<false>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
+        if (mode == 1) TG_TRY((spfp_rounds<1>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
+        else if (mode == 2) TG_TRY((spfp_rounds<2>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
+        else TG_TRY((spfp_rounds<0>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
         g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;
         const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
         uint32_t *o = out_dev ? out + (size_t)b0 * n : nullptr, *no_pred = nullptr;
         TG_TRY(tg_sink_target(g, bi, !out_dev, false, &o, &no_pred, s));
         dim3 grid((unsigned)std::min<uint64_t>((n + 255) / 256, 1024), Sb);
-        TG_LAUNCH(k_spfp_extract, grid, 256, 0, s, Q.vout, g->n, Q.srcs, o, g->relabeled ? g->perm : (const uint32_t *)nullptr);
+        TG_LAUNCH(k_spfp_extract, grid, 256, 0, s, Q.vout, g->n, Q.srcs, o, g->relabeled ? g->perm : (const uint32_t *)nullptr,
+                  mode == 2 ? 1 : 0, w.t_omega);
         TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n, nullptr, (size_t)Sb * n * 4, s));
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));

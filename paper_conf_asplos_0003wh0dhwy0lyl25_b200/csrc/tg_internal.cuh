@@ -67,7 +67,8 @@ struct DevArena {
 // One direction of the transformed graph (forward, or the LD mirror).
 // Layout in HBM:
 //   departure nodes (v, tau) in (v, tau) order:   vnode_off[n+1], node_t[N], node_u[N], node_eoff[N+1]
-//   sorted edges (by (u, t, id)), "occurrences": occ_slot[m] -> slot index, occ_node[m] -> node
+//   sorted edges (by (u, t, id)), "occurrences": occ_slot[m] -> slot index, occ_node[m] -> node,
+//       occ_rec uint2[m] = {v, arrival | walked-chain flag} (the activation's coalesced edge read)
 //   slots in chain-major order (chains ordered by head (u, t, first id)):
 //       slots int4[m] = {v, arr = t + duration, edge id, long-chain index of a walked chain | TG_SINGLE}
 //       slot_w[m], slot_tn[m] (tail departure node or TG_NONE)   -- SP/FP only
@@ -83,6 +84,7 @@ struct ChainGraph {
     uint32_t *vnode_off = nullptr, *node_t = nullptr, *node_u = nullptr, *node_eoff = nullptr;
     uint32_t *occ_slot = nullptr;
     uint32_t *occ_node = nullptr;  // sorted-edge position -> departure node (SP/FP entry state)
+    uint2 *occ_rec = nullptr;      // sorted-edge position -> {head v, arrival | 1 << 31 if on a walked chain}
     int4 *slots = nullptr;
     uint32_t *slot_w = nullptr, *slot_tn = nullptr;
     uint2 *lc = nullptr;
@@ -155,7 +157,7 @@ struct ReachScratch {
     uint64_t bigcap = 0;
     struct RoundCtl *ctl = nullptr;
     unsigned long long *cnt = nullptr;
-    uint32_t *srcs = nullptr;
+    uint32_t *srcs = nullptr, *srcs_int = nullptr;
     uint32_t *stage[1] = {nullptr};
     uint32_t *h_ctr = nullptr;
     DevArena arena;
@@ -238,6 +240,8 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
 tg_status tg_relabel(tg_graph *g, cudaStream_t s);
 // sources of a sub-batch: copy (host) and map to the internal vertex order
 tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cudaStream_t s);
+tg_status tg_load_sources_to(tg_graph *g, const uint32_t *sources, uint32_t k, uint32_t *d_srcs, uint32_t *d_int,
+                             cudaStream_t s);
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,
                              int dirs);  // dirs: bit 0 forward, bit 1 mirror
 
@@ -252,8 +256,6 @@ tg_status tg_sink_target(tg_graph *g, uint32_t b, bool out_host, bool pred_host,
 tg_status tg_sink_flush(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *host_pred, size_t bytes, cudaStream_t s);
 tg_status tg_sink_end(tg_graph *g);
 void tg_sink_destroy(tg_graph *g);
-tg_status tg_run_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
-                       uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
 
 // ----------------------------------------------------------------------------- device helpers
 __device__ __forceinline__ uint32_t tg_lower_bound(const uint32_t *__restrict__ a, uint32_t lo, uint32_t hi,

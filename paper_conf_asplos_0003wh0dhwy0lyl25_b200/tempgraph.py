@@ -18,16 +18,17 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libtempgraph.so")
 
 TG_OK, TG_ERR_INVALID, TG_ERR_RANGE, TG_ERR_NOMEM, TG_ERR_CUDA, TG_ERR_STATE, TG_ERR_NCCL = range(7)
-TG_EAT, TG_LD, TG_FASTEST, TG_SHORTEST, TG_REACH = range(5)
+TG_EAT, TG_LD, TG_FASTEST, TG_SHORTEST, TG_REACH, TG_LD_SOURCE = range(6)
 PROBLEMS = {"eat": TG_EAT, "ld": TG_LD, "fp": TG_FASTEST, "fastest": TG_FASTEST,
-            "sp": TG_SHORTEST, "shortest": TG_SHORTEST, "reach": TG_REACH}
+            "sp": TG_SHORTEST, "shortest": TG_SHORTEST, "reach": TG_REACH, "lds": TG_LD_SOURCE}
 TG_UNREACHED = 0xFFFFFFFF
 TG_TMAX = 0x7FFFFFFE
 
 EXPORTED = ["tg_graph_create", "tg_build_chains", "tg_query", "tg_graph_destroy", "tg_status_string",
             "tg_last_error", "tg_graph_info", "tg_export_chains", "tg_last_query_stats", "tg_set_option",
             "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report", "tg_release_cached_memory",
-            "tg_nccl_unique_id", "tg_comm_create", "tg_comm_destroy", "tg_graph_attach_comm"]
+            "tg_nccl_unique_id", "tg_comm_create", "tg_comm_destroy", "tg_graph_attach_comm",
+            "tg_query_topk", "tg_query_summary"]
 
 
 class TGError(RuntimeError):
@@ -73,6 +74,10 @@ def load_library(path: str = LIB_PATH):
     lib.tg_build_chains.argtypes = [P]
     lib.tg_query.restype = st
     lib.tg_query.argtypes = [P, ctypes.c_int, P, u32, tg_window, P, P, P]
+    lib.tg_query_topk.restype = st
+    lib.tg_query_topk.argtypes = [P, ctypes.c_int, P, u32, tg_window, u32, P, P, P]
+    lib.tg_query_summary.restype = st
+    lib.tg_query_summary.argtypes = [P, ctypes.c_int, P, u32, tg_window, P, P, P]
     lib.tg_graph_destroy.restype = None
     lib.tg_graph_destroy.argtypes = [P]
     lib.tg_status_string.restype = ctypes.c_char_p
@@ -153,6 +158,28 @@ def tg_query(g, problem, sources, window, out, pred=None, stream=None):
     if stream is not None:
         s = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
     _check(lib.tg_query(g, int(problem), src.ctypes.data, int(src.shape[0]), w, _ptr(out), _ptr(pred), s))
+
+
+def tg_query_topk(g, problem, sources, window, K, out_vertex, out_value, stream=None):
+    lib = load_library()
+    src = np.ascontiguousarray(np.asarray(sources, dtype=np.uint32))
+    w = tg_window(int(window[0]), int(window[1]))
+    s = None if stream is None else (stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+    _check(lib.tg_query_topk(g, int(problem), src.ctypes.data, int(src.shape[0]), w, int(K), _ptr(out_vertex),
+                             _ptr(out_value), s))
+
+
+def tg_query_summary(g, problem, sources, window, stream=None):
+    """Returns (count uint64[k], sum uint64[k]) host arrays."""
+    lib = load_library()
+    src = np.ascontiguousarray(np.asarray(sources, dtype=np.uint32))
+    w = tg_window(int(window[0]), int(window[1]))
+    cnt = np.zeros(len(src), np.uint64)
+    sm = np.zeros(len(src), np.uint64)
+    s = None if stream is None else (stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+    _check(lib.tg_query_summary(g, int(problem), src.ctypes.data, int(src.shape[0]), w, cnt.ctypes.data,
+                                sm.ctypes.data, s))
+    return cnt, sm
 
 
 def tg_graph_destroy(g):
@@ -271,6 +298,20 @@ class Graph:
             pred = torch.empty((k, self.n), dtype=torch.int32, device=dev)
         tg_query(self.h, p, sources, window, out, pred, stream)
         return (out, pred) if with_pred else out
+
+    def topk(self, problem, sources, K, window=(0, TG_TMAX)):
+        """(vertices, values): torch.int32 CUDA tensors [k, K] (uint32 bits)."""
+        import torch
+        p = PROBLEMS[problem] if isinstance(problem, str) else int(problem)
+        dev = torch.device("cuda", self.device)
+        ov = torch.empty((len(sources), K), dtype=torch.int32, device=dev)
+        oval = torch.empty((len(sources), K), dtype=torch.int32, device=dev)
+        tg_query_topk(self.h, p, sources, window, K, ov, oval)
+        return ov, oval
+
+    def summary(self, problem, sources, window=(0, TG_TMAX)):
+        p = PROBLEMS[problem] if isinstance(problem, str) else int(problem)
+        return tg_query_summary(self.h, p, sources, window)
 
     def export_chains(self, mirrored=False, shortcuts=True):
         info = self.info()

@@ -551,3 +551,65 @@ def test_reach_bitlane_c2_small(tg):
     for win in tgsynth.CONFIGS["C2"]["windows"]:
         _check_reach(tg, g, og, srcs, win)
     g.close()
+
+
+# --------------------------------------------------------------------------- f4: LDS, top-K, summaries
+@pytest.mark.parametrize("seed", range(10))
+def test_lds_random(tg, seed):
+    """Single-source latest departure (reading R5) on the FP node-state engine: equal to
+    the oracle's one-pass scan, several windows, walk thresholds and relabelling."""
+    n, u, v, t, lam, w = tgsynth.tiny_random(seed + 7300, n_max=60, m_max=900, t_max=40, lam_max=5)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    for opts in ({}, {"walk_min": 2, "relabel": 1}):
+        g = _gpu_graph(tg, n, u, v, t, lam, w, **opts)
+        srcs = list(range(min(n, 20)))
+        for win in [(0, 10**6), (4, 30), (9, 9)]:
+            out = tg.as_u32(g.query("lds", srcs, win))
+            for r, x in enumerate(srcs):
+                np.testing.assert_array_equal(out[r], oracle.lds(og, x, *win), err_msg=f"LDS x={x} win={win}")
+        g.close()
+
+
+def test_lds_c1(tg):
+    ge = tgsynth.make_graph("C1")
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d, w)
+    g = _gpu_graph(tg, n, u, v, t, d, w)
+    for win in tgsynth.CONFIGS["C1"]["windows"]:
+        out = tg.as_u32(g.query("lds", [0, 3, 77], win))
+        for r, x in enumerate([0, 3, 77]):
+            np.testing.assert_array_equal(out[r], oracle.lds(og, x, *win), err_msg=f"LDS C1 x={x} win={win}")
+    g.close()
+
+
+@pytest.mark.parametrize("problem", ["eat", "fp", "sp"])
+def test_topk_and_summary(tg, problem):
+    """top-K nearest (ties by vertex id, source and unreached excluded, padding) and the
+    (reached, sum) row summary against the oracle rows; device and host outputs."""
+    import torch
+    rng = np.random.default_rng(7)
+    n, m = 2000, 30000
+    u = rng.integers(0, n, m).astype(np.uint32); v = rng.integers(0, n, m).astype(np.uint32)
+    t = rng.integers(0, 400, m).astype(np.uint32); lam = rng.integers(1, 8, m).astype(np.uint32)
+    w = rng.integers(0, 9, m).astype(np.uint32)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    g = _gpu_graph(tg, n, u, v, t, lam, w)
+    srcs = [int(x) for x in rng.choice(n, 40, replace=False)]
+    fn = {"eat": lambda x, win: oracle.eat(og, x, *win)[0], "fp": lambda x, win: oracle.fp(og, x, *win),
+          "sp": lambda x, win: oracle.sp(og, x, *win)}[problem]
+    for win, K in [((0, 10**6), 50), ((100, 200), 3000)]:
+        ov, oval = g.topk(problem, srcs, K, win)
+        ov, oval = tg.as_u32(ov), tg.as_u32(oval)
+        hv = torch.empty((len(srcs), K), dtype=torch.int32)
+        hx = torch.empty((len(srcs), K), dtype=torch.int32)
+        tg.tg_query_topk(g.h, tg.PROBLEMS[problem], srcs, win, K, hv, hx)
+        cnt, sm = g.summary(problem, srcs, win)
+        for r, x in enumerate(srcs):
+            row = fn(x, win)
+            ev, ex = oracle.topk(row, x, K)
+            np.testing.assert_array_equal(ov[r], ev, err_msg=f"top-K vertices x={x}")
+            np.testing.assert_array_equal(oval[r], ex, err_msg=f"top-K values x={x}")
+            np.testing.assert_array_equal(tg.as_u32(hv[r]), ev)
+            np.testing.assert_array_equal(tg.as_u32(hx[r]), ex)
+            assert (int(cnt[r]), int(sm[r])) == oracle.summary(row, x)
+    g.close()
