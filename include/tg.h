@@ -160,6 +160,20 @@ TG_API tg_status tg_query_topk(tg_graph *g, tg_problem p, const uint32_t *source
 TG_API tg_status tg_query_summary(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t n_sources,
                                   tg_window w, uint64_t *out_count, uint64_t *out_sum, void *cuda_stream);
 
+/*
+ * tg_graph_insert_edges -- dynamic temporal graphs (§5.6: batches of
+ * edge insertions followed by re-transformation).  Appends k edges
+ * (same arrays and validation as tg_graph_create; ids continue at the current edge
+ * count).  weight must be non-NULL iff the graph was created with weights.  For a
+ * built graph the transformation is redone incrementally: the batch alone is sorted
+ * and merged into the kept (u, t, id) order of each direction, then nodes, chains,
+ * shortcuts and the occurrence index are regenerated; this needs option "dynamic" = 1
+ * before tg_build_chains (else TG_ERR_STATE).  Not for partitioned / relabelled graphs
+ * (TG_ERR_STATE).  On a validation error the graph keeps its previous edges.
+ */
+TG_API tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32_t *u, const uint32_t *v,
+                                       const uint32_t *t_start, const uint32_t *duration, const uint32_t *weight);
+
 TG_API void tg_graph_destroy(tg_graph *g); /* NULL-safe */
 
 TG_API const char *tg_status_string(tg_status s);
@@ -249,6 +263,8 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *                partition then derives its next frontier from the combined state, as
  *                the ranks of a multi-GPU run do (tests; default 0: one process shares
  *                one state and frontier)
+ *   "dynamic"    1 = keep each direction's sorted edge order (before build; 4 B per edge
+ *                and direction) so tg_graph_insert_edges re-transforms incrementally
  *   "packed_state" 1 = EAT/LD/REACH keep the packed u64 (arrival << 32 | pred) state even
  *                when pred == NULL (default 0: without pred the state is the u32 arrival
  *                alone -- half the state bytes; values are identical) */

@@ -9,5 +9,5 @@ from .tempgraph import (  # noqa: F401
     PROBLEMS, TG_EAT, TG_FASTEST, TG_LD, TG_REACH, TG_SHORTEST, TG_TMAX, TG_UNREACHED, Graph, TGError,
     as_u32, load_library, tg_build_chains, tg_export_chains, tg_graph_create, tg_graph_destroy, tg_graph_info,
     tg_kernel_launch_count, tg_last_query_stats, tg_nccl_unique_id, tg_comm_create, tg_comm_destroy,
-    tg_graph_attach_comm, tg_profile_enable, tg_query_topk, tg_query_summary, TG_LD_SOURCE, tg_profile_report, tg_release_cached_memory, tg_query, tg_set_option,
+    tg_graph_attach_comm, tg_profile_enable, tg_query_topk, tg_query_summary, TG_LD_SOURCE, tg_graph_insert_edges, tg_profile_report, tg_release_cached_memory, tg_query, tg_set_option,
 )

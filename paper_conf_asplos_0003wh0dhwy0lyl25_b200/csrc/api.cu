@@ -200,6 +200,12 @@ struct DeviceGuard {
 };
 }  // namespace
 
+uint64_t tg_graph_bytes(const tg_graph *g) {
+    uint64_t b = g->arena.total + g->qs.arena.total + g->rs.arena.total + g->fwd.arena.total + g->mir.arena.total;
+    for (int p = 0; p < TG_MAXP; p++) b += g->pf[p].arena.total + g->pm[p].arena.total;
+    return b;
+}
+
 extern "C" {
 
 const char *tg_status_string(tg_status s) {
@@ -411,6 +417,9 @@ void tg_graph_destroy(tg_graph *g) {
     tg_pinned_put(g->qs.h_ctr);
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);
+    g->fwd.arena.free_all();
+    g->mir.arena.free_all();
+    for (int p = 0; p < TG_MAXP; p++) { g->pf[p].arena.free_all(); g->pm[p].arena.free_all(); }
     g->arena.free_all();
     delete[] g->last_relax;
     delete g;
@@ -432,7 +441,7 @@ tg_status tg_graph_info(const tg_graph *g, tg_info *info) {
         info->max_chain_len = std::max(info->max_chain_len, g->pf[p].maxlen);
     }
     info->c_mirror = g->max_arr;
-    info->device_bytes = g->arena.total + g->qs.arena.total;
+    info->device_bytes = tg_graph_bytes(g);
     info->build_ms = g->build_ms;
     info->built = g->built ? 1 : 0;
     info->n_chains_mirror = g->mir.nchains;
@@ -548,6 +557,10 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     }
     else if (k == "exchange") g->opt_exchange = value ? 1 : 0;
     else if (k == "packed_state") g->opt_packed_state = value ? 1 : 0;
+    else if (k == "dynamic") {
+        if (g->built) { tg_set_error("set dynamic before tg_build_chains"); return TG_ERR_STATE; }
+        g->opt_dynamic = value ? 1 : 0;
+    }
     else if (k == "walk_min") {
         if (g->built) { tg_set_error("set walk_min before tg_build_chains"); return TG_ERR_STATE; }
         g->opt_walk_min = value < 2 ? 2 : value;

@@ -39,6 +39,17 @@ __global__ void k_make_keys(const uint32_t *__restrict__ u, const uint32_t *__re
     }
 }
 
+// keys of edges given in sorted order (ids[i]): the same (u << tbits | t) encoding
+__global__ void k_keys_of_order(const uint32_t *__restrict__ ids, const uint32_t *__restrict__ u,
+                                const uint32_t *__restrict__ t, uint64_t m, int tbits,
+                                unsigned long long *__restrict__ keys, uint32_t *__restrict__ out_ids) {
+    GRID_STRIDE(i, m) {
+        const uint32_t e = ids[i];
+        keys[i] = ((unsigned long long)u[e] << tbits) | t[e];
+        out_ids[i] = e;
+    }
+}
+
 // departure-node boundaries in (u, t)-sorted order
 __global__ void k_node_flags(const unsigned long long *__restrict__ keys, uint64_t m, uint32_t *__restrict__ flag) {
     GRID_STRIDE(p, m) flag[p] = (p == 0 || keys[p] != keys[p - 1]) ? 1u : 0u;
@@ -372,12 +383,12 @@ static void bmark(cudaStream_t s, const char *label) {
 
 tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
                              const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
-                             uint32_t tmax, cudaStream_t s) {
+                             uint32_t tmax, cudaStream_t s, const uint32_t *presorted) {
     const uint32_t n = g->n;
     cg->n = n;
     cg->m = m;
     bmark(s, nullptr);
-    DevArena &A = g->arena;
+    DevArena &A = cg->arena;
     TG_TRY(A.alloc((void **)&cg->vnode_off, ((size_t)n + 1) * 4));
     if (m == 0) {
         TG_TRY_CUDA(cudaMemsetAsync(cg->vnode_off, 0, ((size_t)n + 1) * 4, s));
@@ -393,10 +404,19 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     uint32_t *sid = nullptr;
     TG_TRY_CUDA(tg_malloc_async((void **)&keys, m * 8, s));
     TG_TRY_CUDA(tg_malloc_async((void **)&sid, m * 4, s));
-    TG_LAUNCH(k_make_keys, blocks_for(m, 4), BT, 0, s, u, t, m, tbits, keys, sid);
-    unsigned long long *sk;
-    uint32_t *sv;
-    TG_TRY(tg_radix_sort_pairs(keys, sid, m, tbits + ubits, &sk, &sv, s));
+    if (presorted) {
+        // an insertion merged the new edges into the kept order: keys by gather
+        TG_LAUNCH(k_keys_of_order, blocks_for(m, 4), BT, 0, s, presorted, u, t, m, tbits, keys, sid);
+    } else {
+        TG_LAUNCH(k_make_keys, blocks_for(m, 4), BT, 0, s, u, t, m, tbits, keys, sid);
+        unsigned long long *sk;
+        uint32_t *sv;
+        TG_TRY(tg_radix_sort_pairs(keys, sid, m, tbits + ubits, &sk, &sv, s));
+    }
+    if (g->opt_dynamic) {
+        TG_TRY(A.alloc((void **)&cg->order, m * 4));
+        TG_TRY_CUDA(cudaMemcpyAsync(cg->order, sid, m * 4, cudaMemcpyDeviceToDevice, s));
+    }
 
     bmark(s, "sort");
     // ---- 2. departure nodes

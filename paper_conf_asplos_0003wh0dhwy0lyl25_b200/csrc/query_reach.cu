@@ -276,9 +276,9 @@ tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg
         if (P.stats) TG_TRY_CUDA(cudaMemsetAsync(X.cnt, 0, 64, s));
         TG_LAUNCH(k_reach_ctl, 1, 1, 0, s, X.ctl);
         uint32_t rounds = 0;
+        P.round = 0;  // init pushes into round 1's frontier
+        TG_LAUNCH(k_reach_init, 1, 64, 0, s, P, X.srcs_int, Sb, w.t_alpha);  // sources reach themselves
         if (g->m > 0 && w.t_alpha < w.t_omega) {
-            P.round = 0;  // init pushes into round 1's frontier
-            TG_LAUNCH(k_reach_init, 1, 64, 0, s, P, X.srcs_int, Sb, w.t_alpha);
             uint32_t r = 1;
             for (;;) {
                 for (int i = 0; i < group; i++, r++) {

@@ -92,6 +92,8 @@ struct ChainGraph {
     unsigned long long *sc_sumw = nullptr;
     uint32_t *sc_elapsed = nullptr;
     uint32_t *chain_first = nullptr;
+    uint32_t *order = nullptr;  // option "dynamic": the edge ids in (u, t, id) order, kept for insertions
+    DevArena arena;             // every array of this direction
 };
 
 // Device-side round control of one GAC loop (no host round trip per round): a ring
@@ -203,6 +205,7 @@ struct tg_graph {
     int opt_mirror = 1;
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
+    int64_t opt_dynamic = 0;   // 1 = keep each direction's sorted edge order for tg_graph_insert_edges
     int64_t opt_walk_min = 6;  // chains with fewer edges are not walked (RemoveChain threshold, build time)
     bool mirror_built = false;
     // host-memory outputs: copy stream and per-staging-buffer events (host_out.cu)
@@ -234,9 +237,11 @@ tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uin
                                    unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s,
                                    int snap_bits, uint32_t *snap_vals);
 
+// presorted: NULL, or the m edge ids already in (u, t, id) order (an insertion's merge)
 tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint32_t *u, const uint32_t *v,
                              const uint32_t *t, const uint32_t *dur, const uint32_t *w, const uint32_t *id_map,
-                             uint32_t tmax, cudaStream_t s);
+                             uint32_t tmax, cudaStream_t s, const uint32_t *presorted = nullptr);
+uint64_t tg_graph_bytes(const tg_graph *g);
 tg_status tg_relabel(tg_graph *g, cudaStream_t s);
 // sources of a sub-batch: copy (host) and map to the internal vertex order
 tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cudaStream_t s);

@@ -28,7 +28,7 @@ EXPORTED = ["tg_graph_create", "tg_build_chains", "tg_query", "tg_graph_destroy"
             "tg_last_error", "tg_graph_info", "tg_export_chains", "tg_last_query_stats", "tg_set_option",
             "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report", "tg_release_cached_memory",
             "tg_nccl_unique_id", "tg_comm_create", "tg_comm_destroy", "tg_graph_attach_comm",
-            "tg_query_topk", "tg_query_summary"]
+            "tg_query_topk", "tg_query_summary", "tg_graph_insert_edges"]
 
 
 class TGError(RuntimeError):
@@ -74,6 +74,8 @@ def load_library(path: str = LIB_PATH):
     lib.tg_build_chains.argtypes = [P]
     lib.tg_query.restype = st
     lib.tg_query.argtypes = [P, ctypes.c_int, P, u32, tg_window, P, P, P]
+    lib.tg_graph_insert_edges.restype = st
+    lib.tg_graph_insert_edges.argtypes = [P, u64, P, P, P, P, P]
     lib.tg_query_topk.restype = st
     lib.tg_query_topk.argtypes = [P, ctypes.c_int, P, u32, tg_window, u32, P, P, P]
     lib.tg_query_summary.restype = st
@@ -144,6 +146,11 @@ def tg_graph_create(n_vertices, u, v, t_start, duration, weight=None, device=0):
     _check(lib.tg_graph_create(int(n_vertices), m, _ptr(u), _ptr(v), _ptr(t_start), _ptr(duration), _ptr(weight),
                                int(device), ctypes.byref(h)))
     return h
+
+
+def tg_graph_insert_edges(g, u, v, t_start, duration, weight=None):
+    _check(load_library().tg_graph_insert_edges(g, int(u.shape[0]), _ptr(u), _ptr(v), _ptr(t_start), _ptr(duration),
+                                                _ptr(weight)))
 
 
 def tg_build_chains(g):
@@ -277,6 +284,11 @@ class Graph:
 
     def build(self):
         tg_build_chains(self.h)
+        return self
+
+    def insert_edges(self, u, v, t, dur, w=None):
+        tg_graph_insert_edges(self.h, u, v, t, dur, w)
+        self.m += int(u.shape[0])
         return self
 
     def info(self):

@@ -613,3 +613,73 @@ def test_topk_and_summary(tg, problem):
             np.testing.assert_array_equal(tg.as_u32(hx[r]), ex)
             assert (int(cnt[r]), int(sm[r])) == oracle.summary(row, x)
     g.close()
+
+
+# --------------------------------------------------------------------------- f3: dynamic insertions
+def _t32(a):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a, np.uint32).view(np.int32)).cuda()
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_insert_edges_incremental(tg, seed):
+    """Batches of insertions into a built graph: after each batch the
+    incrementally re-transformed chains equal Alg. 1 / Alg. 2 of the oracle on the whole
+    edge list (ids continue), and every problem equals the oracle."""
+    rng = np.random.default_rng(seed + 4400)
+    n = 300
+    m0 = 3000
+    cols = lambda m, tmax: (rng.integers(0, n, m), rng.integers(0, n, m), rng.integers(0, tmax, m),
+                            rng.integers(1, 7, m), rng.integers(0, 9, m))
+    U, V, T, L, W = (np.asarray(c, np.uint32) for c in cols(m0, 200))
+    g = _gpu_graph(tg, n, U, V, T, L, W, dynamic=1)
+    for b, (k, tmax) in enumerate([(500, 200), (1200, 400), (1, 50), (800, 600)]):
+        bu, bv, bt, bl, bw = (np.asarray(c, np.uint32) for c in cols(k, tmax))
+        g.insert_edges(_t32(bu), _t32(bv), _t32(bt), _t32(bl), _t32(bw))
+        U, V, T, L, W = (np.concatenate([a, c]) for a, c in zip((U, V, T, L, W), (bu, bv, bt, bl, bw)))
+        og = oracle.Graph(n, U, V, T, L, W)
+        off, ce = oracle.chains(og)
+        sc = oracle.shortcuts(og, off, ce)
+        ch = g.export_chains()
+        np.testing.assert_array_equal(ch["chain_off"], off, err_msg=f"batch {b}")
+        np.testing.assert_array_equal(ch["chain_edges"], ce, err_msg=f"batch {b}")
+        for key in ("tail_v", "arr", "elapsed", "sum_w"):
+            np.testing.assert_array_equal(ch[key], sc[key], err_msg=key)
+        gr, _ = oracle.mirror(og)
+        moff, mce = oracle.chains(gr)
+        mch = g.export_chains(mirrored=True, shortcuts=False)
+        np.testing.assert_array_equal(mch["chain_edges"], mce)
+        srcs = [int(x) for x in rng.choice(n, 12, replace=False)]
+        for win in [(0, 10**6), (40, 300)]:
+            for p in ("eat", "ld", "sp", "fp", "reach"):
+                _check_rows(tg, g, og, p, srcs, win)
+            _check_reach(tg, g, og, srcs, win)
+    g.close()
+
+
+def test_insert_edges_errors_and_unbuilt(tg):
+    rng = np.random.default_rng(3)
+    n, m = 50, 400
+    U, V, T, L = (rng.integers(0, n, m).astype(np.uint32), rng.integers(0, n, m).astype(np.uint32),
+                  rng.integers(0, 90, m).astype(np.uint32), rng.integers(1, 4, m).astype(np.uint32))
+    f = _t32
+    # built without "dynamic": refused
+    g = _gpu_graph(tg, n, U, V, T, L)
+    with pytest.raises(tg.TGError) as e:
+        g.insert_edges(f(U[:5]), f(V[:5]), f(T[:5]), f(L[:5]))
+    assert e.value.status == 5
+    g.close()
+    # unbuilt: edges appended, the first build sees all of them; a bad batch rolls back
+    g = tg.Graph(n, f(U), f(V), f(T), f(L), None, device=0)
+    g.set_option("dynamic", 1)
+    g.insert_edges(f(V[:100]), f(U[:100]), f(T[:100] + 5), f(L[:100]))
+    with pytest.raises(tg.TGError) as e:
+        g.insert_edges(f(np.array([n], np.uint32)), f(U[:1]), f(T[:1]), f(L[:1]))  # endpoint out of range
+    assert e.value.status == 2
+    g.build()
+    U2, V2 = np.concatenate([U, V[:100]]), np.concatenate([V, U[:100]])
+    T2, L2 = np.concatenate([T, T[:100] + 5]), np.concatenate([L, L[:100]])
+    og = oracle.Graph(n, U2, V2, T2, L2)
+    _check_rows(tg, g, og, "eat", list(range(10)), (0, 10**6))
+    _check_rows(tg, g, og, "ld", list(range(10)), (0, 10**6))
+    g.close()
