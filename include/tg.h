@@ -174,6 +174,25 @@ TG_API tg_status tg_query_summary(tg_graph *g, tg_problem p, const uint32_t *sou
 TG_API tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32_t *u, const uint32_t *v,
                                        const uint32_t *t_start, const uint32_t *duration, const uint32_t *weight);
 
+/*
+ * tg_graph_create_streamed -- a graph larger than the device memory (
+ * P:L342-346 §4.5 "Supporting of Out-of-GPU-Memory Processing").  Same edge arrays and
+ * validation as tg_graph_create, but they must be HOST memory and are never resident
+ * on the device as a whole: they are validated chunk by chunk and cut into blocks of
+ * consecutive departure times holding at most block_edges edges each (a topological
+ * order of the transformed DAG; one departure time with more edges forms a block of
+ * its own), kept in pinned host memory.  tg_build_chains transforms every block on
+ * the device (Alg. 1 / Alg. 2 / occurrence index) and keeps the result in pinned host
+ * memory; tg_query (TG_EAT, TG_REACH; else TG_ERR_STATE) streams the blocks in time
+ * order through two device slots, copying block b+1 while block b is computed.
+ * Results are identical to a device-resident graph's.  tg_graph_info reports
+ * n_blocks and host_bytes.  Options other than sub_batch / stats / round_group /
+ * shortcuts / walk_min have no effect.
+ */
+TG_API tg_status tg_graph_create_streamed(uint32_t n_vertices, uint64_t n_edges, const uint32_t *u, const uint32_t *v,
+                                          const uint32_t *t_start, const uint32_t *duration, const uint32_t *weight,
+                                          int device, uint64_t block_edges, tg_graph **out_graph);
+
 TG_API void tg_graph_destroy(tg_graph *g); /* NULL-safe */
 
 TG_API const char *tg_status_string(tg_status s);
@@ -192,6 +211,8 @@ typedef struct {
     double build_ms;         /* last tg_build_chains wall time                              */
     int built;
     uint64_t n_chains_mirror; /* chains of the LD mirror graph                              */
+    uint64_t host_bytes;      /* streamed graphs: pinned host memory holding the time blocks */
+    uint32_t n_blocks;        /* streamed graphs: time blocks (0 = device-resident graph)    */
 } tg_info;
 
 TG_API tg_status tg_graph_info(const tg_graph *g, tg_info *info);

@@ -203,6 +203,7 @@ struct DeviceGuard {
 uint64_t tg_graph_bytes(const tg_graph *g) {
     uint64_t b = g->arena.total + g->qs.arena.total + g->rs.arena.total + g->fwd.arena.total + g->mir.arena.total;
     for (int p = 0; p < TG_MAXP; p++) b += g->pf[p].arena.total + g->pm[p].arena.total;
+    if (g->stream) b += g->stream->slot_arena.total;
     return b;
 }
 
@@ -331,7 +332,10 @@ tg_status tg_build_chains(tg_graph *g) {
     if (g->built) return TG_OK;
     DeviceGuard dg(g->device);
     auto t0 = std::chrono::steady_clock::now();
-    if (g->comm && g->comm_mode == 1) {
+    if (g->stream) {
+        // out-of-memory graph: every time block transformed on the device, kept in host memory
+        TG_TRY(tg_build_streamed(g));
+    } else if (g->comm && g->comm_mode == 1) {
         // this rank's vertex range of a single partitioned query batch
         const int r = tg_comm_rank(g->comm), P = tg_comm_world(g->comm);
         g->nparts = 1;
@@ -385,6 +389,13 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
     cudaStream_t s = (cudaStream_t)cuda_stream;
     const bool out_dev = is_device_ptr(out);
     const bool pred_dev = is_device_ptr(pred);
+    if (g->stream) {
+        if (!(p == TG_EAT || p == TG_REACH)) {
+            tg_set_error("streamed (out-of-memory) graphs answer TG_EAT / TG_REACH");
+            return TG_ERR_STATE;
+        }
+        return tg_run_eat_streamed(g, sources, n_sources, w, out, pred, out_dev, pred_dev, p == TG_REACH ? 2 : 0, s);
+    }
     if (p == TG_LD && !g->mirror_built) {  // lazily built mirror (option "mirror" = 0)
         if (g->nparts > 0) {
             for (int pi = 0; pi < g->nparts; pi++)
@@ -413,6 +424,7 @@ void tg_graph_destroy(tg_graph *g) {
     DeviceGuard dg(g->device);
     cudaDeviceSynchronize();
     tg_sink_destroy(g);
+    tg_stream_free(g);
     g->qs.arena.free_all();
     tg_pinned_put(g->qs.h_ctr);
     g->rs.arena.free_all();
@@ -434,6 +446,11 @@ tg_status tg_graph_info(const tg_graph *g, tg_info *info) {
     info->n_chains = g->fwd.nchains;
     info->n_long_chains = g->fwd.nlong;
     info->max_chain_len = g->fwd.maxlen;
+    if (g->stream)
+        for (const HostBlock &b : g->stream->blocks) {  // streamed: totals over the time blocks
+            info->n_nodes += b.nn;
+            info->n_long_chains += b.L;
+        }
     for (int p = 0; p < g->nparts; p++) {  // partitioned: totals over this process's partitions
         info->n_nodes += g->pf[p].nnodes;
         info->n_chains += g->pf[p].nchains;
@@ -445,6 +462,10 @@ tg_status tg_graph_info(const tg_graph *g, tg_info *info) {
     info->build_ms = g->build_ms;
     info->built = g->built ? 1 : 0;
     info->n_chains_mirror = g->mir.nchains;
+    if (g->stream) {
+        info->n_blocks = (uint32_t)g->stream->blocks.size();
+        for (const HostBlock &b : g->stream->blocks) info->host_bytes += b.bytes;
+    }
     return TG_OK;
 }
 
@@ -452,7 +473,7 @@ tg_status tg_export_chains(const tg_graph *g, int mirrored, uint64_t *chain_off,
                            uint32_t *sc_tail_v, uint32_t *sc_arr, uint64_t *sc_sum_w, uint32_t *sc_elapsed) {
     if (!g || !chain_off || !chain_edges) { tg_set_error("NULL argument"); return TG_ERR_INVALID; }
     if (!g->built) { tg_set_error("graph not built"); return TG_ERR_STATE; }
-    if (g->nparts > 0) { tg_set_error("chain export is for unpartitioned graphs"); return TG_ERR_STATE; }
+    if (g->nparts > 0 || g->stream) { tg_set_error("chain export is for unpartitioned, device-resident graphs"); return TG_ERR_STATE; }
     if (mirrored && !g->mirror_built) { tg_set_error("the mirror graph has not been built"); return TG_ERR_STATE; }
     DeviceGuard dg(g->device);
     const ChainGraph &c = mirrored ? g->mir : g->fwd;

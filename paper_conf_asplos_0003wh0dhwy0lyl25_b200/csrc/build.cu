@@ -338,16 +338,28 @@ __global__ void k_mirror(const uint32_t *__restrict__ t, const uint32_t *__restr
 
 }  // namespace
 
+// validation of a chunk of edges, accumulated into res[5] (device; initialised to
+// {0, 0, 0, 0, 0xFFFFFFFF}); w may be NULL (weight = duration)
+tg_status tg_validate_launch(const uint32_t *u, const uint32_t *v, const uint32_t *t, const uint32_t *dur,
+                             const uint32_t *w, uint64_t m, uint32_t n, uint32_t *res, cudaStream_t s) {
+    if (m) TG_LAUNCH(k_validate, blocks_for(m, 4), BT, 0, s, u, v, t, dur, w, m, n, res);
+    return TG_OK;
+}
+
 tg_status tg_validate_edges(tg_graph *g, cudaStream_t s) {
     uint32_t *res = nullptr;
     TG_TRY_CUDA(tg_malloc_async((void **)&res, 5 * 4, s));
     uint32_t init[5] = {0, 0, 0, 0, 0xFFFFFFFFu};
     TG_TRY_CUDA(cudaMemcpyAsync(res, init, sizeof(init), cudaMemcpyHostToDevice, s));
-    if (g->m) TG_LAUNCH(k_validate, blocks_for(g->m, 4), BT, 0, s, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, g->m, g->n, res);
+    TG_TRY(tg_validate_launch(g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, g->m, g->n, res, s));
     uint32_t h[5];
     TG_TRY_CUDA(cudaMemcpyAsync(h, res, sizeof(h), cudaMemcpyDeviceToHost, s));
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     TG_TRY_CUDA(cudaFreeAsync(res, s));
+    return tg_validate_finish(g, h);
+}
+
+tg_status tg_validate_finish(tg_graph *g, const uint32_t *h) {
     if (h[0] & 1u) { tg_set_error("edge endpoint >= n_vertices"); return TG_ERR_RANGE; }
     if (h[0] & 2u) { tg_set_error("edge duration 0 (durations must be >= 1, reading A2)"); return TG_ERR_INVALID; }
     if (h[0] & 4u) { tg_set_error("t + duration > TG_TMAX"); return TG_ERR_RANGE; }

@@ -638,6 +638,23 @@ __global__ void k_state_min_exchange(void *__restrict__ st_, uint32_t P, uint64_
     }
 }
 
+// Streamed graphs: the frontier at the start of a time block = every (v, q) already
+// reached (its out-edges in this block may be usable); one thread per frontier word.
+template <bool PK>
+__global__ void k_frontier_reached(const void *__restrict__ st_, uint64_t n, uint32_t S, uint32_t G,
+                                   uint32_t *__restrict__ fb) {
+    const typename StW<PK>::T *st = (const typename StW<PK>::T *)st_;
+    const typename StW<PK>::T INF = (typename StW<PK>::T)~0ull;
+    for (uint64_t u = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; u < n * G; u += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t v = u / G;
+        const uint32_t g = (uint32_t)(u - v * G);
+        uint32_t w = 0;
+        for (uint32_t k = 0; k < 32 && g * 32 + k < S; k++)
+            if (st[v * S + g * 32 + k] != INF) w |= 1u << k;
+        fb[u] = w;
+    }
+}
+
 __global__ void k_popcount(const uint32_t *__restrict__ w, uint64_t nw, unsigned long long *__restrict__ out) {
     unsigned long long c = 0;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x)
@@ -668,7 +685,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     tg_pinned_put(Q.h_ctr);
     Q.h_ctr = nullptr;
     Q = QueryScratch{};
-    const uint64_t n = g->n, m = g->m;
+    const uint64_t n = g->n, m = g->stream ? g->stream->max_m : g->m;  // streamed: the largest block
     Q.S = S;
     Q.n = g->n;
     Q.nnodes = nnodes;
@@ -743,6 +760,10 @@ uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
 
 tg_status tg_ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) { return ensure_scratch(g, S, nodes_state); }
 
+template <bool PK>
+static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
+                          cudaStream_t s, uint32_t *rounds_out);
+
 // Run the GAC rounds of one sub-batch on direction cg; returns rounds used.
 template <bool PK>
 static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
@@ -757,13 +778,25 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
     if (g->opt_stats) {
         TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8 + 8 + 64, s));
-        TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, Q.bit_words * 4, s));
     }
     const bool work = any_work && g->m > 0 && alpha < omega;
     TG_LAUNCH(k_eat_init<PK>, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
+    *rounds_out = 0;
+    if (work) TG_TRY(eat_loop<PK>(g, cgr, S, alpha, omega, s, rounds_out));
+    return TG_OK;
+}
+
+// The GAC rounds over direction cgr from the frontier in Q.fb[1] (round 1) with the
+// round control reset; stops at the first round whose frontier was empty.
+template <bool PK>
+static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
+                          cudaStream_t s, uint32_t *rounds_out) {
+    QueryScratch &Q = g->qs;
+    const uint32_t G = (S + 31) / 32;
     uint32_t rounds = 0;
-    if (work) {
+    {
         EatP P{};
         P.vnode_off = cgr.vnode_off; P.node_t = cgr.node_t; P.node_eoff = cgr.node_eoff; P.occ_slot = cgr.occ_slot;
         P.occ_rec = cgr.occ_rec;
@@ -946,7 +979,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
         TG_TRY_CUDA(cudaMemsetAsync(Q.pcount, 0, 4, s));
         if (g->opt_stats) {
             TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8 + 8 + 64, s));
-            TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, ((g->m + 31) / 32 + TG_MAXP + 1) * 4, s));
+            TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, Q.bit_words * 4, s));
         }
         // One process holds every partition (logical partitions, or a world of 1): the
         // partitions share the state and the frontier bitmaps, so the bits the relaxations
@@ -1074,4 +1107,100 @@ tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
     if (pred != nullptr || g->opt_packed_state)
         return eat_partitioned<true>(g, p, sources, k, w, out, pred, out_dev, pred_dev, s);
     return eat_partitioned<false>(g, p, sources, k, w, out, pred, out_dev, pred_dev, s);
+}
+
+// ============================================================================ streamed graphs
+tg_status tg_stream_load(tg_graph *g, uint32_t b, int i);
+
+// EAT (mode 0) / REACH (mode 2) on a graph streamed in time blocks (stream.cu): the
+// rounds of block b start from every reached (v, q) with fresh activation boundaries
+// (block-local occurrence indices) and claim bits; block b + 1 is copied into the
+// other device slot on the copy stream while block b computes.
+template <bool PK>
+static tg_status eat_streamed(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
+                              uint32_t *pred, bool out_dev, bool pred_dev, int mode, cudaStream_t s) {
+    StreamGraph &SG = *g->stream;
+    const uint32_t S = tg_pick_sub_batch(g, k, false);
+    TG_TRY(ensure_scratch(g, S, false));
+    QueryScratch &Q = g->qs;
+    const uint64_t n = g->n;
+    const uint32_t alpha = w.t_alpha, omega = w.t_omega;
+    TG_TRY(tg_sink_begin(g, !out_dev, pred && !pred_dev));
+    g->last = tg_query_stats{};
+    if (g->opt_stats) {
+        delete[] g->last_relax;
+        g->last_relax = new uint64_t[k];
+        g->last_relax_len = k;
+    }
+    const uint64_t launches0 = g_tg_launches;
+    SG.h2d_bytes = 0;
+    const uint32_t B = (uint32_t)SG.blocks.size();
+    // blocks that can hold a valid edge: t >= alpha and t < omega
+    std::vector<uint32_t> todo;
+    for (uint32_t b = 0; b < B; b++)
+        if (SG.blocks[b].m && SG.blocks[b].t_hi > alpha && SG.blocks[b].t_lo < omega) todo.push_back(b);
+    const uint64_t tw = (SG.max_m + 31) / 32 + TG_MAXP + 1;
+    for (uint32_t b0 = 0; b0 < k; b0 += S) {
+        const uint32_t Sb = std::min(S, k - b0);
+        const uint32_t G = (Sb + 31) / 32;
+        TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, Sb * n * (PK ? 8 : 4), s));
+        if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, Sb * 8 + 8 + 64, s));
+        TG_LAUNCH(k_eat_init<PK>, (Sb + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, Sb, alpha, Q.fb[1], Q.ctl, 0);
+        uint32_t rounds = 0;
+        uint64_t wu = 0;
+        // slots: block todo[i] goes to slot i & 1; the first two are loaded up front
+        for (size_t i = 0; i < todo.size() && i < 2; i++) TG_TRY(tg_stream_load(g, todo[i], (int)(i & 1)));
+        for (size_t i = 0; i < todo.size(); i++) {
+            const int si = (int)(i & 1);
+            TG_TRY_CUDA(cudaStreamWaitEvent(s, SG.ready[si], 0));
+            const ChainGraph &cgr = SG.slot[si];
+            TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, Sb * n * 4, s));
+            TG_TRY_CUDA(cudaMemsetAsync(Q.bits, 0, Sb * ((cgr.m + 31) / 32 + 1) * 4, s));
+            TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
+            if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, tw * 4, s));
+            TG_LAUNCH(k_frontier_reached<PK>, (unsigned)std::min<uint64_t>((n * G + 255) / 256, 148ull * 16), 256, 0,
+                      s, Q.st, n, Sb, G, Q.fb[1]);
+            TG_LAUNCH(k_ctl_reset, 1, 1, 0, s, Q.ctl);
+            uint32_t r = 0;
+            TG_TRY(eat_loop<PK>(g, cgr, Sb, alpha, omega, s, &r));
+            rounds += r;
+            if (g->opt_stats) {
+                TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, Q.touched, tw,
+                          Q.relax_cnt + Sb);
+            }
+            TG_TRY_CUDA(cudaEventRecord(SG.freed[si], s));
+            if (i + 2 < todo.size()) TG_TRY(tg_stream_load(g, todo[i + 2], si));
+        }
+        (void)wu;
+        g->last.rounds = std::max(g->last.rounds, rounds);
+        g->last.sub_batches++;
+        const uint32_t bi = b0 / S;
+        uint32_t *o = out_dev ? out + (size_t)b0 * n : nullptr;
+        uint32_t *pr = pred ? (pred_dev ? pred + (size_t)b0 * n : pred) : nullptr;
+        TG_TRY(tg_sink_target(g, bi, !out_dev, pred && !pred_dev, &o, &pr, s));
+        const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
+        TG_LAUNCH(k_eat_extract<PK>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, 0u, omega, o, pr,
+                  (const uint32_t *)nullptr);
+        TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n,
+                             (pred && !pred_dev) ? pred + (size_t)b0 * n : nullptr, (size_t)Sb * n * 4, s));
+        if (g->opt_stats) {
+            std::vector<unsigned long long> h(Sb + 1);
+            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, (Sb + 1) * 8, cudaMemcpyDeviceToHost, s));
+            TG_TRY_CUDA(cudaStreamSynchronize(s));
+            for (uint32_t q = 0; q < Sb; q++) { g->last_relax[b0 + q] = h[q]; g->last.slots_relaxed += h[q]; }
+            g->last.slots_union += h[Sb];
+        }
+    }
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    TG_TRY(tg_sink_end(g));
+    g->last.kernel_launches = g_tg_launches - launches0;
+    return TG_OK;
+}
+
+tg_status tg_run_eat_streamed(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
+                              uint32_t *pred, bool out_dev, bool pred_dev, int mode, cudaStream_t s) {
+    if (pred != nullptr || g->opt_packed_state)
+        return eat_streamed<true>(g, sources, k, w, out, pred, out_dev, pred_dev, mode, s);
+    return eat_streamed<false>(g, sources, k, w, out, pred, out_dev, pred_dev, mode, s);
 }

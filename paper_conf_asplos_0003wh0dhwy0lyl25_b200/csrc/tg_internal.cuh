@@ -148,6 +148,36 @@ struct QueryScratch {
     DevArena arena;
 };
 
+// Out-of-memory graphs (stream.cu; §4.5): the edges are cut
+// into blocks of consecutive departure times (a topological order of the transformed
+// DAG); each block's chain structure lives in pinned host memory and is streamed to one
+// of two device slots while the previous block is being computed.
+struct HostBlock {
+    uint64_t m = 0, nn = 0, L = 0;
+    uint32_t t_lo = 0, t_hi = 0;  // departure times [t_lo, t_hi)
+    uint32_t *vnode_off = nullptr, *node_t = nullptr, *node_eoff = nullptr, *occ_slot = nullptr;
+    uint2 *occ_rec = nullptr;
+    int4 *slots = nullptr;
+    uint2 *lc = nullptr;
+    int4 *sc = nullptr;
+    void *pinned = nullptr;
+    uint64_t bytes = 0;
+};
+struct StreamGraph {
+    uint64_t block_edges = 0;
+    std::vector<HostBlock> blocks;
+    // the input, organised by block (pinned): u, v, t, dur, w, id per block
+    std::vector<uint32_t *> bedges;
+    std::vector<void *> bedges_pinned;
+    bool weighted = false;
+    uint64_t max_m = 0, max_nn = 0, max_L = 0;
+    ChainGraph slot[2];
+    DevArena slot_arena;
+    cudaStream_t cs = nullptr;
+    cudaEvent_t ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr};
+    uint64_t h2d_bytes = 0;  // streamed by the last query
+};
+
 // Bit-lane reachability scratch (query_reach.cu): one u64 word per departure node and
 // per vertex for a sub-batch of up to 64 sources.
 struct ReachScratch {
@@ -196,6 +226,7 @@ struct tg_graph {
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
     ReachScratch rs;
+    StreamGraph *stream = nullptr;  // out-of-memory graph (tg_graph_create_streamed)
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
     // options
     int64_t opt_sub_batch = 0;
@@ -247,6 +278,13 @@ tg_status tg_relabel(tg_graph *g, cudaStream_t s);
 tg_status tg_load_sources(tg_graph *g, const uint32_t *sources, uint32_t k, cudaStream_t s);
 tg_status tg_load_sources_to(tg_graph *g, const uint32_t *sources, uint32_t k, uint32_t *d_srcs, uint32_t *d_int,
                              cudaStream_t s);
+tg_status tg_validate_launch(const uint32_t *u, const uint32_t *v, const uint32_t *t, const uint32_t *dur,
+                             const uint32_t *w, uint64_t m, uint32_t n, uint32_t *res, cudaStream_t s);
+tg_status tg_validate_finish(tg_graph *g, const uint32_t *h);  // h: the 5 accumulated words
+tg_status tg_build_streamed(tg_graph *g);
+void tg_stream_free(tg_graph *g);
+tg_status tg_run_eat_streamed(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
+                              uint32_t *pred, bool out_dev, bool pred_dev, int mode, cudaStream_t s);
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,
                              int dirs);  // dirs: bit 0 forward, bit 1 mirror
 

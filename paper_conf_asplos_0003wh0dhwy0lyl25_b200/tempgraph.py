@@ -28,7 +28,7 @@ EXPORTED = ["tg_graph_create", "tg_build_chains", "tg_query", "tg_graph_destroy"
             "tg_last_error", "tg_graph_info", "tg_export_chains", "tg_last_query_stats", "tg_set_option",
             "tg_kernel_launch_count", "tg_profile_enable", "tg_profile_report", "tg_release_cached_memory",
             "tg_nccl_unique_id", "tg_comm_create", "tg_comm_destroy", "tg_graph_attach_comm",
-            "tg_query_topk", "tg_query_summary", "tg_graph_insert_edges"]
+            "tg_query_topk", "tg_query_summary", "tg_graph_insert_edges", "tg_graph_create_streamed"]
 
 
 class TGError(RuntimeError):
@@ -46,7 +46,7 @@ class tg_info(ctypes.Structure):
                 ("n_chains", ctypes.c_uint64), ("n_long_chains", ctypes.c_uint64),
                 ("max_chain_len", ctypes.c_uint32), ("c_mirror", ctypes.c_uint32),
                 ("device_bytes", ctypes.c_uint64), ("build_ms", ctypes.c_double), ("built", ctypes.c_int),
-                ("n_chains_mirror", ctypes.c_uint64)]
+                ("n_chains_mirror", ctypes.c_uint64), ("host_bytes", ctypes.c_uint64), ("n_blocks", ctypes.c_uint32)]
 
 
 class tg_query_stats(ctypes.Structure):
@@ -74,6 +74,8 @@ def load_library(path: str = LIB_PATH):
     lib.tg_build_chains.argtypes = [P]
     lib.tg_query.restype = st
     lib.tg_query.argtypes = [P, ctypes.c_int, P, u32, tg_window, P, P, P]
+    lib.tg_graph_create_streamed.restype = st
+    lib.tg_graph_create_streamed.argtypes = [u32, u64, P, P, P, P, P, ctypes.c_int, u64, ctypes.POINTER(P)]
     lib.tg_graph_insert_edges.restype = st
     lib.tg_graph_insert_edges.argtypes = [P, u64, P, P, P, P, P]
     lib.tg_query_topk.restype = st
@@ -151,6 +153,16 @@ def tg_graph_create(n_vertices, u, v, t_start, duration, weight=None, device=0):
 def tg_graph_insert_edges(g, u, v, t_start, duration, weight=None):
     _check(load_library().tg_graph_insert_edges(g, int(u.shape[0]), _ptr(u), _ptr(v), _ptr(t_start), _ptr(duration),
                                                 _ptr(weight)))
+
+
+def tg_graph_create_streamed(n_vertices, u, v, t_start, duration, weight=None, device=0, block_edges=1 << 26):
+    """Out-of-memory graph (host arrays only; see include/tg.h)."""
+    lib = load_library()
+    h = ctypes.c_void_p()
+    m = int(u.shape[0])
+    _check(lib.tg_graph_create_streamed(int(n_vertices), m, _ptr(u), _ptr(v), _ptr(t_start), _ptr(duration),
+                                        _ptr(weight), int(device), int(block_edges), ctypes.byref(h)))
+    return h
 
 
 def tg_build_chains(g):
@@ -276,11 +288,16 @@ def tg_profile_report() -> dict:
 class Graph:
     """Owning wrapper: Graph(n, u, v, t, dur, w=None, device=0).build().query(...)."""
 
-    def __init__(self, n, u, v, t, dur, w=None, device=0):
+    def __init__(self, n, u, v, t, dur, w=None, device=0, block_edges=None):
+        """block_edges: None = device-resident graph; else an out-of-memory graph
+        streamed in time blocks of at most that many edges (host arrays)."""
         self.n = int(n)
         self.m = int(u.shape[0])
         self.device = device
-        self.h = tg_graph_create(n, u, v, t, dur, w, device)
+        if block_edges is None:
+            self.h = tg_graph_create(n, u, v, t, dur, w, device)
+        else:
+            self.h = tg_graph_create_streamed(n, u, v, t, dur, w, device, block_edges)
 
     def build(self):
         tg_build_chains(self.h)

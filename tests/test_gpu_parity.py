@@ -683,3 +683,55 @@ def test_insert_edges_errors_and_unbuilt(tg):
     _check_rows(tg, g, og, "eat", list(range(10)), (0, 10**6))
     _check_rows(tg, g, og, "ld", list(range(10)), (0, 10**6))
     g.close()
+
+
+# --------------------------------------------------------------------------- f1: out-of-memory graphs
+def _streamed(tg, n, u, v, t, lam, w=None, block_edges=64, **opts):
+    import torch
+    f = lambda a: torch.from_numpy(np.ascontiguousarray(a, np.uint32).view(np.int32))  # HOST tensors
+    g = tg.Graph(n, f(u), f(v), f(t), f(lam), None if w is None else f(w), device=0, block_edges=block_edges)
+    for k, val in opts.items():
+        g.set_option(k, val)
+    return g.build()
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_streamed_blocks_random(tg, seed):
+    """Graphs cut into time blocks (§4.5), transformed per block, kept in host
+    memory and streamed through two device slots: EAT values, preds and first-touch W,
+    REACH, equal to the oracle for block sizes from a few edges to the whole graph."""
+    rng = np.random.default_rng(seed + 5100)
+    n, m = 200 + 40 * seed, 3000
+    u = rng.integers(0, n, m).astype(np.uint32); v = rng.integers(0, n, m).astype(np.uint32)
+    t = rng.integers(0, 120 + 400 * (seed % 2), m).astype(np.uint32); lam = rng.integers(1, 9, m).astype(np.uint32)
+    og = oracle.Graph(n, u, v, t, lam)
+    srcs = [int(x) for x in rng.choice(n, 37, replace=False)]
+    for be in (1, 37, 500, 10**6):
+        g = _streamed(tg, n, u, v, t, lam, block_edges=be, stats=1)
+        info = g.info()
+        assert info["n_blocks"] >= 1 and (be >= m or info["n_blocks"] > 1)
+        for win in [(0, 10**6), (30, 90), (50, 50)]:
+            _check_rows(tg, g, og, "eat", srcs, win, stats=True)
+            _check_values(tg, g, og, "eat", srcs, win)
+            _check_values(tg, g, og, "reach", srcs, win)
+        with pytest.raises(tg.TGError) as e:
+            g.query("ld", srcs[:2], (0, 100))
+        assert e.value.status == 5
+        g.close()
+
+
+def test_streamed_c2_small_and_host_out(tg):
+    import torch
+    ge = tgsynth.make_graph("C2", scale_shift=-4)
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d)
+    g = _streamed(tg, n, u, v, t, d, block_edges=100_000)
+    assert g.info()["n_blocks"] >= 10
+    srcs = tgsynth.config_sources("C2", ge)
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        _check_values(tg, g, og, "eat", srcs, win)
+    hout = torch.empty((8, n), dtype=torch.int32)
+    tg.tg_query(g.h, tg.TG_EAT, srcs[:8], (0, 10**9), hout)
+    for r, x in enumerate(srcs[:8]):
+        np.testing.assert_array_equal(tg.as_u32(hout[r]), oracle.eat(og, x, 0, 10**9)[0])
+    g.close()
