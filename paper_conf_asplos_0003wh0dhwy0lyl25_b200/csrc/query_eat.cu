@@ -44,8 +44,14 @@ namespace cg = cooperative_groups;
 namespace {
 
 constexpr int QT = 256;                 // threads per block
-constexpr uint32_t BIG_T = 128;         // unions longer than this are split into chunks
-constexpr uint32_t CHUNK = 128;         // edges per chunk (one warp)
+#ifndef TG_BIG_T
+#define TG_BIG_T 128
+#endif
+#ifndef TG_CHUNK
+#define TG_CHUNK 128
+#endif
+constexpr uint32_t BIG_T = TG_BIG_T;    // unions longer than this are split into chunks
+constexpr uint32_t CHUNK = TG_CHUNK;    // edges per chunk (one warp)
 constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in the activating thread
 #ifndef TG_MLP
 #define TG_MLP 4                        // state reads in flight per lane in the pair loop
@@ -71,6 +77,7 @@ struct EatP {
     uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
     uint32_t alpha, omega;
     int use_sc, stats;
+    int omega_all;  // omega > every departure time: a vertex's window end is its last edge (no search)
     RoundCtl *ctl;
     uint32_t round;       // GAC round of this launch (host loop counter; parity picks the bitmaps)
     uint32_t *fb0, *fb1;  // frontier masks [n][G] (bit = query within the group), by round parity
@@ -338,7 +345,8 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
             pending &= pending - 1;
             const uint32_t qm = __shfl_sync(0xffffffffu, word, sl);
             const uint32_t unit = ub + sl;
-            const uint32_t v = unit / P.G;
+            // G is 1 or 2 for sub-batches <= 64 (a uniform branch instead of an integer division)
+            const uint32_t v = P.G == 1 ? unit : (P.G == 2 ? unit >> 1 : unit / P.G);
             const uint32_t g = unit - v * P.G;
             const uint32_t q = g * 32 + lane;
             uint32_t lo = 0, hi = 0;
@@ -368,9 +376,9 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
             // a first activation starts from the window end (t + duration <= omega needs t < omega)
             if (__any_sync(0xffffffffu, hi == TG_NONE)) {
 #if TG_COOP_SEARCH
-                const uint32_t ehi = __ldg(P.node_eoff + tg_warp_lower_bound(P.node_t, a, b, P.omega));
+                const uint32_t ehi = __ldg(P.node_eoff + (P.omega_all ? b : tg_warp_lower_bound(P.node_t, a, b, P.omega)));
 #else
-                const uint32_t ehi = __ldg(P.node_eoff + tg_lower_bound(P.node_t, a, b, P.omega));
+                const uint32_t ehi = __ldg(P.node_eoff + (P.omega_all ? b : tg_lower_bound(P.node_t, a, b, P.omega)));
 #endif
                 if (hi == TG_NONE) hi = ehi;
             }
@@ -417,6 +425,148 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         }
     }
     if (lane == 0 && my_units) atomicAdd(R.words_cnt, my_units);  // per warp: no block barrier
+}
+
+// Single-query sub-batches (S == 1; the paper's own workload, P:L110 / P:L373): lane
+// per frontier vertex instead of warp per unit.  Each lane computes its vertex's newly
+// usable range by its own binary search; vertices with many departure nodes are
+// searched by the whole warp, one at a time (a lane's long dependent search would stall
+// its warp).  Ranges longer than BIG_T go to k_eat_big (a record with the range in
+// lane 0); the rest are relaxed by the warp together: each lane takes one edge of the
+// concatenated ranges (owner found by a shuffle search over the prefix sums).
+constexpr uint32_t LANE_SEARCH_MAX = 64;  // departure nodes a lane searches alone
+template <bool PK>
+__global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
+    const RoundV R = round_view(P);
+    clear_next_round(P);
+    uint32_t my_units = 0;
+    const uint32_t NU = P.ub1;
+    const int lane = threadIdx.x & 31;
+    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t ub = P.ub0 + gw * 32; ub < NU; ub += nw * 32) {
+        const uint32_t v = ub + lane;  // G == 1: unit = vertex
+        const uint32_t word = (v < NU) ? R.fin[v] : 0u;
+        const bool on = word != 0;
+        if (on) R.fin[v] = 0u;  // consume
+        const uint32_t onm = __ballot_sync(0xffffffffu, on);
+        if (!onm) continue;
+        my_units += (lane == 0) ? __popc(onm) : 0u;
+        uint32_t prev = 0, now = 0, a = 0, b = 0, lo = 0, hi = 0;
+        if (on) {
+            prev = __ldcg(P.act + v);
+            now = StW<PK>::time(__ldcg((const typename StW<PK>::T *)P.st + v));
+            a = __ldg(P.vnode_off + v);
+            b = __ldg(P.vnode_off + v + 1);
+        }
+        const uint32_t key = max(now, P.alpha);
+        const bool small = on && b - a <= LANE_SEARCH_MAX;
+        uint32_t j0 = 0, jw = 0;
+        if (small) {
+            j0 = tg_lower_bound(P.node_t, a, b, key);
+            if (prev == TG_NONE) jw = P.omega_all ? b : tg_lower_bound(P.node_t, a, b, P.omega);
+        }
+        uint32_t bigm = __ballot_sync(0xffffffffu, on && !small);
+        while (bigm) {  // hubs: warp-cooperative searches, results to their lane
+            const int o = __ffs(bigm) - 1;
+            bigm &= bigm - 1;
+            const uint32_t oa = __shfl_sync(0xffffffffu, a, o), ob = __shfl_sync(0xffffffffu, b, o);
+            const uint32_t ok = __shfl_sync(0xffffffffu, key, o);
+            const uint32_t op = __shfl_sync(0xffffffffu, prev, o);
+            const uint32_t r0 = tg_warp_lower_bound(P.node_t, oa, ob, ok);
+            const uint32_t r1 = (op == TG_NONE) ? (P.omega_all ? ob : tg_warp_lower_bound(P.node_t, oa, ob, P.omega)) : 0u;
+            if (lane == o) { j0 = r0; jw = r1; }
+        }
+        if (on) {
+            const uint32_t elo = __ldg(P.node_eoff + j0);
+            hi = (prev == TG_NONE) ? __ldg(P.node_eoff + jw) : prev;  // first activation: up to the window end
+            if (elo < hi) {
+                lo = elo;
+                P.act[v] = elo;  // (v, 0) is activated by this lane alone in this round
+            } else {
+                hi = 0;
+            }
+        }
+        if (P.stats) {
+            const uint32_t act_n = __popc(__ballot_sync(0xffffffffu, lo < hi));
+            if (lane == 0) {
+                atomicAdd(P.diag + 3, (unsigned long long)act_n);
+                atomicAdd(P.diag + 4, (unsigned long long)__popc(onm));
+            }
+        }
+        // long ranges: chunks for k_eat_big (query 0's range in lane 0 of the record)
+        const bool big = lo < hi && hi - lo > BIG_T;
+        uint32_t bm = __ballot_sync(0xffffffffu, big);
+        while (bm) {
+            const int o = __ffs(bm) - 1;
+            bm &= bm - 1;
+            const uint32_t olo = __shfl_sync(0xffffffffu, lo, o), ohi = __shfl_sync(0xffffffffu, hi, o);
+            const uint32_t nch = (ohi - olo + CHUNK - 1) / CHUNK;
+            uint32_t rec = 0, k0 = 0;
+            if (lane == 0) {
+                rec = atomicAdd(R.rec_cnt, 1u);
+                k0 = atomicAdd(R.big_cnt, nch);
+            }
+            rec = __shfl_sync(0xffffffffu, rec, 0);
+            k0 = __shfl_sync(0xffffffffu, k0, 0);
+            const bool rec_ok = rec < P.reccap;
+            if (rec_ok) P.recs[(size_t)rec * 32 + lane] = lane == 0 ? make_uint2(olo, ohi) : make_uint2(0, 0);
+            uint32_t queued = 0;
+            if (k0 < P.bigcap) queued = min(nch, (uint32_t)(P.bigcap - k0));
+            for (uint32_t c = lane; c < queued; c += 32) {
+                const uint32_t b0 = olo + c * CHUNK;
+                P.bigq[k0 + c] = rec_ok ? make_uint4(rec, b0, min(ohi, b0 + CHUNK), 0) : make_uint4(0, 0, 0, 0);
+            }
+            // whatever is not queued stays with the owner lane for the shared pass below
+            if (lane == o) {
+                if (rec_ok && queued == nch) { lo = 0; hi = 0; }
+                else if (rec_ok) lo = olo + queued * CHUNK;
+            }
+        }
+        // the remaining ranges, concatenated: lane takes edge t of the concatenation
+        uint32_t cnt = lo < hi ? hi - lo : 0;
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+        if (P.stats && lane == 0 && total) atomicAdd(P.diag + 0, (unsigned long long)total);
+        for (uint32_t t0 = 0; t0 < total; t0 += 32) {
+            const uint32_t t = t0 + lane;
+            uint32_t k = 0;  // owner: first lane with incl > t
+#pragma unroll
+            for (uint32_t st = 16; st; st >>= 1) {
+                const uint32_t y = __shfl_sync(0xffffffffu, incl, k + st - 1);
+                if (y <= t) k += st;
+            }
+            k &= 31;
+            const uint32_t olo = __shfl_sync(0xffffffffu, lo, k);
+            const uint32_t oex = __shfl_sync(0xffffffffu, incl - cnt, k);
+            if (t >= total) continue;
+            const uint32_t p = olo + (t - oex);
+            uint32_t s = 0;
+            int4 sl;
+            if (PK) {
+                s = __ldg(P.occ_slot + p);
+                sl = tg_ld_slot(P.slots + s);
+            } else {
+                const uint2 r = __ldg(P.occ_rec + p);
+                if (r.y >> 31) {
+                    s = __ldg(P.occ_slot + p);
+                    sl = tg_ld_slot(P.slots + s);
+                } else {
+                    sl = make_int4((int)r.x, (int)r.y, 0, (int)TG_SINGLE);
+                    if (P.stats) s = __ldg(P.occ_slot + p);
+                }
+            }
+            if ((uint32_t)sl.y > P.omega) continue;  // past the window end: never usable
+            if ((uint32_t)sl.w == TG_SINGLE) eat_relax<PK>(P, R, 0, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+            else eat_long<PK>(P, R, 0, s, sl);
+        }
+    }
+    if (lane == 0 && my_units) atomicAdd(R.words_cnt, my_units);
 }
 
 // Chunks of long unions: one warp per chunk, the unit's 32 query ranges from its record.
@@ -764,6 +914,12 @@ template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
                           cudaStream_t s, uint32_t *rounds_out);
 
+// largest departure time of a direction: forward max t; the LD mirror's departures are
+// C - (t + lambda) <= C - min t - 1 (a bound is enough: it only enables a shortcut)
+static uint32_t dir_max_t(const tg_graph *g, const ChainGraph &cg) {
+    return (&cg == &g->mir || (g->nparts && &cg >= g->pm && &cg < g->pm + TG_MAXP)) ? g->max_arr - g->min_t : g->max_t;
+}
+
 // Run the GAC rounds of one sub-batch on direction cg; returns rounds used.
 template <bool PK>
 static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
@@ -805,6 +961,7 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
         P.ub0 = 0; P.ub1 = g->n * G;
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
+        P.omega_all = omega > dir_max_t(g, cgr) ? 1 : 0;
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         P.touched = Q.touched;
@@ -820,7 +977,8 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
             for (int k = 0; k < group; k++, r++) {
                 P.round = r;
                 if (trace) cudaEventRecord(tev[0], s);
-                TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, P);
+                if (S == 1) TG_LAUNCH_RELAX(k_eat_activate1<PK>, grid, QT, 0, s, P);
+                else TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, P);
                 if (trace) cudaEventRecord(tev[1], s);
                 TG_LAUNCH_RELAX(k_eat_big<PK>, grid, QT, 0, s, P);
                 if (trace) cudaEventRecord(tev[2], s);
@@ -1001,6 +1159,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
             base.st = Q.st; base.act = Q.act; base.bits = Q.bits; base.bit_words = Q.bit_words;
             base.n = g->n; base.S = Sb; base.G = G; base.alpha = alpha; base.omega = omega;
             base.use_sc = (int)g->opt_shortcuts; base.stats = (int)g->opt_stats;
+            base.omega_all = 0;  // (per partition below)
             base.fb0 = Q.fb[0]; base.fb1 = Q.fb[1]; base.recs = Q.recs; base.reccap = Q.reccap;
             base.bigq = Q.bigq; base.bigcap = Q.bigcap; base.chq = Q.chq; base.chcap = Q.chcap;
             base.relax_cnt = Q.relax_cnt;
@@ -1016,6 +1175,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 bit_off += (cg.m + 31) / 32;
                 P.vnode_off = cg.vnode_off; P.node_t = cg.node_t; P.node_eoff = cg.node_eoff; P.occ_slot = cg.occ_slot;
                 P.occ_rec = cg.occ_rec;
+                P.omega_all = omega > dir_max_t(g, cg) ? 1 : 0;
                 P.slots = cg.slots; P.lc = cg.lc; P.sc = cg.sc;
                 P.ctl = Q.ctl + pi;
                 P.ub0 = g->part_vb[pi] * G;
@@ -1040,7 +1200,8 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 for (int pi = 0; pi < g->nparts; pi++) {
                     if (parts[pi].ub0 == parts[pi].ub1) continue;  // no vertices: never any work
                     parts[pi].round = r;
-                    TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, parts[pi]);
+                    if (Sb == 1) TG_LAUNCH_RELAX(k_eat_activate1<PK>, grid, QT, 0, s, parts[pi]);
+                    else TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, parts[pi]);
                     TG_LAUNCH_RELAX(k_eat_big<PK>, grid, QT, 0, s, parts[pi]);
                     TG_LAUNCH_RELAX(k_eat_chain<PK>, 148, QT, 0, s, parts[pi]);
                 }

@@ -34,6 +34,7 @@ constexpr uint32_t RBIG = 128;    // a 32-node scan chunk with more changed out-
 
 struct ReachP {
     const uint32_t *vnode_off, *node_t, *node_eoff, *occ_slot, *occ_node, *slot_tn;
+    const uint4 *occ_rch;
     const int4 *slots;
     const uint2 *lc;
     unsigned long long *R;   // [nnodes] node words
@@ -65,9 +66,22 @@ __device__ __forceinline__ void mark_dirty(const ReachP &P, uint32_t j, uint32_t
 // Relax out-occurrence p (sorted-edge position) of a node holding word w; walked
 // chains continue with the bits their tail node gained.
 __device__ __forceinline__ void reach_edge(const ReachP &P, uint32_t p, unsigned long long w) {
+    // one coalesced 16-byte record {v, arrival | walked, tail node, tail tau}: a one-edge
+    // (or not walked) chain needs nothing else
+    const uint4 rc = __ldg(P.occ_rch + p);
+    if ((rc.y & 0x7FFFFFFFu) > P.omega) return;  // arrival past the window: not valid
+    if (!(rc.y >> 31)) {
+        if (P.stats) atomicAdd(P.cnt + 0, 1ull);
+        if (w & ~__ldcg(P.VR + rc.x)) atomicOr(P.VR + rc.x, w);
+        if (rc.z == TG_NONE || rc.w >= P.omega) return;  // sink / nothing valid departs later
+        unsigned long long nb = w & ~__ldcg(P.R + rc.z);
+        if (!nb) return;
+        nb &= ~atomicOr(P.R + rc.z, nb);
+        if (nb) mark_dirty(P, rc.z, rc.x);
+        return;
+    }
     uint32_t s = __ldg(P.occ_slot + p);
     int4 sl = tg_ld_slot(P.slots + s);
-    if ((uint32_t)sl.y > P.omega) return;  // arrival past the window: not valid
     uint32_t s_end = s + 1;
     if ((uint32_t)sl.w != TG_SINGLE) {
         const uint2 info = __ldg(P.lc + (uint32_t)sl.w);
@@ -206,6 +220,17 @@ __global__ void k_reach_init(ReachP P, const uint32_t *srcs, uint32_t S, uint32_
     }
 }
 
+// the bit-lane engine's occurrence records (built once per direction, on first use)
+__global__ void k_reach_records(const uint2 *__restrict__ occ_rec, const uint32_t *__restrict__ occ_slot,
+                                const uint32_t *__restrict__ slot_tn, const uint32_t *__restrict__ node_t, uint64_t m,
+                                uint4 *__restrict__ out) {
+    for (uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; p < m; p += (uint64_t)gridDim.x * blockDim.x) {
+        const uint2 r = occ_rec[p];
+        const uint32_t tn = slot_tn[occ_slot[p]];
+        out[p] = make_uint4(r.x, r.y, tn, tn == TG_NONE ? 0xFFFFFFFFu : node_t[tn]);
+    }
+}
+
 __global__ void k_reach_ctl(RoundCtl *ctl) {
     for (int i = 0; i < TG_RING; i++)
         for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
@@ -224,7 +249,12 @@ __global__ void k_reach_extract(const unsigned long long *__restrict__ VR, uint3
 
 tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                             bool out_dev, cudaStream_t s) {
-    const ChainGraph &c = g->fwd;
+    ChainGraph &c = g->fwd;
+    if (!c.occ_rch && g->m) {
+        TG_TRY(c.arena.alloc((void **)&c.occ_rch, g->m * 16));
+        TG_LAUNCH(k_reach_records, (unsigned)std::min<uint64_t>((g->m + 255) / 256, 148ull * 32), 256, 0, s, c.occ_rec,
+                  c.occ_slot, c.slot_tn, c.node_t, g->m, c.occ_rch);
+    }
     const uint64_t n = g->n, nn = c.nnodes;
     const uint32_t S = std::min<uint32_t>(64, k);
     ReachScratch &X = g->rs;
@@ -260,7 +290,7 @@ tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg
     const uint64_t launches0 = g_tg_launches;
     ReachP P{};
     P.vnode_off = c.vnode_off; P.node_t = c.node_t; P.node_eoff = c.node_eoff; P.occ_slot = c.occ_slot;
-    P.occ_node = c.occ_node; P.slot_tn = c.slot_tn; P.slots = c.slots; P.lc = c.lc;
+    P.occ_node = c.occ_node; P.slot_tn = c.slot_tn; P.slots = c.slots; P.lc = c.lc; P.occ_rch = c.occ_rch;
     P.R = X.R; P.VR = X.VR;
     for (int i = 0; i < 2; i++) { P.D[i] = X.D[i]; P.dmin[i] = X.dmin[i]; P.dmax[i] = X.dmax[i]; P.vf[i] = X.vf[i]; }
     P.bigq = X.bigq; P.bigcap = X.bigcap; P.ctl = X.ctl; P.n = g->n; P.omega = w.t_omega;

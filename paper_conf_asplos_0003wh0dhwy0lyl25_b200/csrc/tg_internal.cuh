@@ -85,6 +85,7 @@ struct ChainGraph {
     uint32_t *occ_slot = nullptr;
     uint32_t *occ_node = nullptr;  // sorted-edge position -> departure node (SP/FP entry state)
     uint2 *occ_rec = nullptr;      // sorted-edge position -> {head v, arrival | 1 << 31 if on a walked chain}
+    uint4 *occ_rch = nullptr;      // bit-lane reach (built on first use): {v, arrival | walked flag, tail node, tail tau}
     int4 *slots = nullptr;
     uint32_t *slot_w = nullptr, *slot_tn = nullptr;
     uint2 *lc = nullptr;

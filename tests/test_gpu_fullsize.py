@@ -3,8 +3,10 @@
 fixpoint + witness + tie-rule conditions of tests/props.py (which determine EAT / LD
 rows uniquely; pinned against the oracle in tests/test_props_cpu.py).  The u32-state
 path (no preds, what the bench times) must give the same values as the packed path."""
+import numpy as np
 import pytest
 
+import oracle
 import tgsynth
 from tests import props
 
@@ -86,7 +88,81 @@ def test_c5_full_vertex_partitioned(tg):
     g.set_option("mirror", 0)
     g.build()
     srcs = tgsynth.config_sources("C5", ge)
-    _certify(tg, ge, g, srcs, tgsynth.CONFIGS["C5"]["windows"][0], problems=("eat",))
+    win = tgsynth.CONFIGS["C5"]["windows"][0]
+    _certify(tg, ge, g, srcs, win, problems=("eat",))
     g.close()
+    # the cross-rank algorithm (private state per partition, min exchange every round,
+    # frontier from the exchanged state): the max-degree source's row element by element
+    # against the oracle, values and preds
+    g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, None, device=0)
+    g.set_option("partitions", 8)
+    g.set_option("exchange", 1)
+    g.set_option("mirror", 0)
+    g.build()
+    out, pred = g.query("eat", srcs[:1], win, with_pred=True)
+    out, pred = tg.as_u32(out)[0], tg.as_u32(pred)[0]
+    g.close()
+    n, u, v, t, d, _ = ge.numpy()
     del ge
     torch.cuda.empty_cache()
+    A, P, _ = oracle.eat(oracle.Graph(n, u, v, t, d), srcs[0], *win)
+    np.testing.assert_array_equal(out, A)
+    np.testing.assert_array_equal(pred, P)
+
+
+def test_c4_rows_vs_oracle(tg):
+    """configs[3] at full size in the bench's launch configuration (u32 states, 64-source
+    sub-batch): two rows element by element against the oracle."""
+    import torch
+    ge = tgsynth.make_graph("C4", device="cuda")
+    g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, None, device=0)
+    g.set_option("mirror", 0)
+    g.build()
+    srcs = tgsynth.config_sources("C4", ge)[:64]
+    win = tgsynth.CONFIGS["C4"]["windows"][0]
+    out = tg.as_u32(g.query("eat", srcs, win))
+    g.close()
+    n, u, v, t, d, _ = ge.numpy()
+    del ge
+    torch.cuda.empty_cache()
+    og = oracle.Graph(n, u, v, t, d)
+    for r in (0, 63):
+        np.testing.assert_array_equal(out[r], oracle.eat(og, srcs[r], *win)[0], err_msg=f"C4 row {r}")
+
+
+def test_c2_weighted_sp_fp_sampled(tg):
+    """SP / FP / LDS on a high-reach graph at full C2 size (16.8 M edges, w ~ U[1,100]):
+    sampled rows of a 4-source batch element by element against the oracle."""
+    ge = tgsynth.make_graph("C2", device="cuda")
+    g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, ge.w, device=0)
+    g.set_option("mirror", 0)
+    g.build()
+    srcs = tgsynth.config_sources("C2", ge)[:4]
+    win = tgsynth.CONFIGS["C2"]["windows"][1]
+    rows = {p: tg.as_u32(g.query(p, srcs, win)) for p in ("sp", "fp", "lds")}
+    g.close()
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d, w)
+    for r in (0, 3):
+        np.testing.assert_array_equal(rows["sp"][r], oracle.sp(og, srcs[r], *win), err_msg=f"SP row {r}")
+        np.testing.assert_array_equal(rows["fp"][r], oracle.fp(og, srcs[r], *win), err_msg=f"FP row {r}")
+        np.testing.assert_array_equal(rows["lds"][r], oracle.lds(og, srcs[r], *win), err_msg=f"LDS row {r}")
+
+
+def test_c2_streamed_full(tg):
+    """configs[1] as an out-of-memory graph (8 time blocks of ~2.1 M edges streamed from
+    host memory): the bench's 64-source EAT batch equals the device-resident graph's."""
+    import torch
+    ge = tgsynth.make_graph("C2", device="cuda")
+    srcs = tgsynth.config_sources("C2", ge)
+    win = tgsynth.CONFIGS["C2"]["windows"][0]
+    g = tg.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, None, device=0).build()
+    ref = g.query("eat", srcs, win)
+    g.close()
+    hu, hv, ht, hd = (x.cpu() for x in (ge.u, ge.v, ge.t, ge.dur))
+    gs = tg.Graph(ge.n, hu, hv, ht, hd, None, device=0, block_edges=ge.m // 8 + 1).build()
+    assert gs.info()["n_blocks"] >= 8
+    out = gs.query("eat", srcs, win)
+    torch.cuda.synchronize()
+    assert torch.equal(out, ref)
+    gs.close()

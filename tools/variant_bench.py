@@ -32,16 +32,17 @@ torch.cuda.synchronize()
 torch.cuda.empty_cache()
 g = T.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, None, device=0)
 for kk, vv in opts.items():
-    if kk != "engine":
-        g.set_option(kk, vv)
+    g.set_option(kk, vv)
 g.build()
-if "engine" in opts:
-    g.set_option("engine", opts["engine"])
 out = torch.empty((k, ge.n), dtype=torch.int32, device="cuda")
 pred = torch.empty((k, ge.n), dtype=torch.int32, device="cuda") if with_pred else None
 win = tgsynth.CONFIGS[cfg]["windows"][0]
 res = {}
-for p in ("eat", "ld"):
+problems = [a[len("--problems="):] for a in sys.argv if a.startswith("--problems=")]
+problems = problems[0].split(",") if problems else ["eat", "ld"]
+if "ld" not in problems:
+    pass
+for p in problems:
     ts = []
     for it in range(7):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -62,8 +63,7 @@ if "--check" in sys.argv:
     ref = T.Graph(ge.n, ge.u, ge.v, ge.t, ge.dur, None, device=0)
     ref.set_option("packed_state", 1)
     ref.build()
-    ref.set_option("engine", 1)  # GAC rounds
-    for p in ("eat", "ld"):
+    for p in problems:
         o2 = torch.empty_like(out)
         ref.query(p, src, win, out=o2)
         print(f"check {p}: {'OK' if torch.equal(o2, res[p][2]) else 'MISMATCH'} (vs packed-state path)", flush=True)
