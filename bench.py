@@ -38,7 +38,7 @@ import numpy as np  # noqa: E402
 HBM_FALLBACK_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
 METRIC = "temporal-path queries/s (EAT; plus LD/FP/SP where the config lists them)"
 UNIT = "queries/s"
-RELAX_KERNELS = ("k_eat_activate", "k_eat_big", "k_eat_chain")
+RELAX_KERNELS = ("k_eat_activate", "k_eat_big", "k_eat_chain", "k_reach_scan", "k_reach_big")
 
 
 def parse_args(argv=None):
@@ -65,6 +65,9 @@ def parse_args(argv=None):
     ap.add_argument("--partitions", type=int, default=1, help="logical vertex-range partitions per GPU")
     ap.add_argument("--exchange", type=int, default=0, help="vertex mode: cross-rank exchange algorithm")
     ap.add_argument("--cpu-threads", type=int, default=0, help="oracle threads (0 = all host cores)")
+    ap.add_argument("--problems", default=None, help="comma list overriding the config's problems (e.g. reach)")
+    ap.add_argument("--stream-blocks", type=int, default=0,
+                    help="out-of-memory mode: the graph streamed from host memory in this many time blocks")
     return ap.parse_args(argv)
 
 
@@ -171,6 +174,8 @@ def workload(cfg_name, k_job, rank, world, device, mode="replicate", scaling="st
         job = (job * (want // max(1, len(job)) + 1))[:want]
     mine = plan_sources(job, rank, world, scaling, mode)
     problems = list(cfg["problems"]) or ["eat"]
+    if getattr(workload, "problems", None):
+        problems = list(workload.problems)
     win = cfg["windows"][0]
     weighted = cfg["kind"] == "wikitalk"
     return ge, job, mine, problems, win, weighted, cfg
@@ -234,12 +239,18 @@ def run_ours(a, rank, world, local_rank):
     w_arg = ge.w if weighted else None
     outs = {p: torch.empty((k, n), dtype=torch.int32, device=dev) for p in problems}
     torch.cuda.synchronize()
+    host_edges = None
+    if a.stream_blocks:  # out-of-memory mode: the library takes HOST arrays and streams time blocks
+        host_edges = [x.cpu() for x in (ge.u, ge.v, ge.t, ge.dur)] + [ge.w.cpu() if weighted else None]
     comm = None
     if a.mode == "vertex":
         from paper_conf_asplos_0003wh0dhwy0lyl25_b200.distributed import make_comm
         comm = make_comm(rank, world, local_rank, bcast_device=dev)
 
     def make_graph():
+        if host_edges is not None:
+            g = tg.Graph(n, *host_edges, device=local_rank, block_edges=m // a.stream_blocks + 1)
+            return g.build()
         g = tg.Graph(n, ge.u, ge.v, ge.t, ge.dur, w_arg, device=local_rank)
         if a.sub_batch:
             g.set_option("sub_batch", a.sub_batch)
@@ -282,6 +293,11 @@ def run_ours(a, rank, world, local_rank):
     gstat.set_option("stats", 1)
     W_by_problem, Wu_by_problem = {}, {}
     for p in problems:
+        if p == "reach":
+            # the bit-lane engine's usable edges are the EAT union of the same batch
+            gstat.query("eat", mine, win, out=outs[p])
+            Wu_by_problem[p] = int(gstat.last_stats(k)["slots_union"])
+            continue
         if p not in ("eat", "ld"):
             continue  # the first-touch work counters cover the EAT-family engine
         gstat.query(p, mine, win, out=outs[p])
@@ -355,10 +371,15 @@ def run_ours(a, rank, world, local_rank):
         # (u32 arrivals: pred = NULL): every slot relaxed by some query of a sub-batch is read
         # once (16 B slot + 4 B occurrence), every relaxation touches 4 B of state:
         # B = 20 B x W_union + 4 B x sum_q W_q.  (The survey's packed 8-B word is reported too.)
+        # bit-lane reach (f2): per usable edge one 16-B occurrence record, the 8-B head word
+        # and the 8-B tail-node word (64 sources per word); per sub-batch the vertex words
         W_steps = W_local * a.steps
-        Wu_steps = sum(Wu_by_problem.values()) * a.steps
-        relax_bytes = 20 * Wu_steps + 4 * W_steps
-        relax_bytes_pk = 20 * Wu_steps + 8 * W_steps
+        Wu_eat = sum(v for p, v in Wu_by_problem.items() if p != "reach") * a.steps
+        Wu_reach = Wu_by_problem.get("reach", 0) * a.steps
+        reach_bytes = 32 * Wu_reach + 8 * n * (-(-k // 64)) * a.steps * ("reach" in problems)
+        relax_bytes = 20 * Wu_eat + 4 * W_steps + reach_bytes
+        relax_bytes_pk = 20 * Wu_eat + 8 * W_steps + reach_bytes
+        Wu_steps = Wu_eat + Wu_reach
         traffic = None
         tf = os.path.join(ROOT, "profiles", "round2", f"relax_traffic_{a.config}.json")
         if os.path.exists(tf) and a.mode == "replicate" and a.partitions == 1 and world == 1 and not a.k:
@@ -366,7 +387,7 @@ def run_ours(a, rank, world, local_rank):
         ach = relax_bytes / (relax_ms / 1e3) / 1e9 if relax_ms else None
         roof = {
             "bound": "hbm",
-            "kernel": "relax phase (k_eat_activate + k_eat_big + k_eat_chain)",
+            "kernel": "relax phase (" + " + ".join(sorted({x.split("<")[0] for x in relax_names})) + ")",
             "achieved": ach,
             "peak": peak,
             "unit": "GB/s",
@@ -375,8 +396,9 @@ def run_ours(a, rank, world, local_rank):
             "traffic_source": (os.path.relpath(tf, ROOT) + ": " + traffic["source"]) if traffic else None,
             "peak_source": peak_src,
             "algorithmic_bytes_per_step": relax_bytes / a.steps,
-            "algorithmic_bytes_formula": "20 B x W_union + 4 B x sum_q W_q (SURVEY 8(d) batched source lanes, "
-                                         "u32 state as timed)",
+            "algorithmic_bytes_formula": ("20 B x W_union + 4 B x sum_q W_q (SURVEY 8(d) batched source lanes, "
+                                          "u32 state as timed)") if "reach" not in problems else
+                                         "32 B x W_union + 8 B x n per 64-source word (bit-lane reach, DESIGN 5.5)",
             "achieved_packed_8B_formula": relax_bytes_pk / (relax_ms / 1e3) / 1e9 if relax_ms else None,
             "W_union_per_step": Wu_steps / a.steps,
             "W_sum_per_step": W_steps / a.steps,
@@ -397,7 +419,7 @@ def run_ours(a, rank, world, local_rank):
     torch.cuda.synchronize()
     torch.cuda.empty_cache()
     e2e = None
-    if not a.no_e2e and comm is None:
+    if not a.no_e2e and comm is None and not a.stream_blocks:
         e2e = run_e2e(a, tg, ge, mine, k_job, problems, win, weighted, world, dev)
 
     cpu = None
@@ -428,6 +450,7 @@ def run_ours(a, rank, world, local_rank):
                       "create+validate, build_chains (" + ("fwd+mirror" if "ld" in problems else "fwd") + "), ")
                      + " + ".join(f"{p} x{k}" for p in problems) + " per rank"),
             "query_only": a.query_only,
+            "streamed_blocks": info.get("n_blocks", 0) if a.stream_blocks else 0,
             "l2": "inputs larger than L2 (edge list %.0f MB, chain structure %.0f MB > 126 MB)" % (
                 m * (20 if weighted else 16) / 1e6, info["device_bytes"] / 1e6),
             "sub_batch": a.sub_batch or "auto",
@@ -587,6 +610,8 @@ def run_reference(a, rank, world):
 def main():
     os.environ.setdefault("NCCL_DEBUG", "WARN")  # keep NCCL's version banner off stdout (one JSON line)
     a = parse_args()
+    if a.problems:
+        workload.problems = a.problems.split(",")
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))

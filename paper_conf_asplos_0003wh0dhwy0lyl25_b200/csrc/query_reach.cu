@@ -24,7 +24,11 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include <cooperative_groups.h>
+
 #include "tg_internal.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace {
 
@@ -52,13 +56,20 @@ struct ReachP {
 };
 
 // node j of vertex v gained bits in round P.round: it is scanned in round + 1
+// Only the first-node atomicMin returns a value (it decides the vertex's single push);
+// the dirty bit and the last dirty node are fire-and-forget reductions, so a relaxation
+// waits on one atomic round trip, not on a chain of them.
 __device__ __forceinline__ void mark_dirty(const ReachP &P, uint32_t j, uint32_t v) {
     const int o = (P.round + 1) & 1;
-    const uint32_t bit = 1u << (j & 31);
-    if (atomicOr(P.D[o] + (j >> 5), bit) & bit) return;  // already dirty for the next round
+    atomicOr(P.D[o] + (j >> 5), 1u << (j & 31));
     atomicMax(P.dmax[o] + v, j);
     if (atomicMin(P.dmin[o] + v, j) == TG_NONE) {
-        const uint32_t k = atomicAdd(&P.ctl->cnt[(P.round + 1) & (TG_RING - 1)][0], 1u);
+        // one counter atomic per group of pushing lanes (a single-address counter hit by
+        // every push serialises)
+        cg::coalesced_group grp = cg::coalesced_threads();
+        uint32_t k = 0;
+        if (grp.thread_rank() == 0) k = atomicAdd(&P.ctl->cnt[(P.round + 1) & (TG_RING - 1)][0], grp.size());
+        k = grp.shfl(k, 0) + grp.thread_rank();
         P.vf[o][k] = v;  // at most once per vertex per round: k < n
     }
 }
@@ -74,10 +85,12 @@ __device__ __forceinline__ void reach_edge(const ReachP &P, uint32_t p, unsigned
         if (P.stats) atomicAdd(P.cnt + 0, 1ull);
         if (w & ~__ldcg(P.VR + rc.x)) atomicOr(P.VR + rc.x, w);
         if (rc.z == TG_NONE || rc.w >= P.omega) return;  // sink / nothing valid departs later
-        unsigned long long nb = w & ~__ldcg(P.R + rc.z);
+        // the filter read decides (bits only grow: a stale read can only add redundant
+        // bits, which the OR absorbs and the next scan finds already present)
+        const unsigned long long nb = w & ~__ldcg(P.R + rc.z);
         if (!nb) return;
-        nb &= ~atomicOr(P.R + rc.z, nb);
-        if (nb) mark_dirty(P, rc.z, rc.x);
+        atomicOr(P.R + rc.z, nb);
+        mark_dirty(P, rc.z, rc.x);
         return;
     }
     uint32_t s = __ldg(P.occ_slot + p);
@@ -94,10 +107,9 @@ __device__ __forceinline__ void reach_edge(const ReachP &P, uint32_t p, unsigned
         const uint32_t tn = __ldg(P.slot_tn + s);
         if (tn == TG_NONE) return;  // sink: no later departure of v
         if (__ldg(P.node_t + tn) >= P.omega) return;  // nothing valid departs at >= omega
-        unsigned long long nb = w & ~__ldcg(P.R + tn);
+        const unsigned long long nb = w & ~__ldcg(P.R + tn);
         if (!nb) return;
-        nb &= ~atomicOr(P.R + tn, nb);
-        if (!nb) return;
+        atomicOr(P.R + tn, nb);
         mark_dirty(P, tn, v);
         if (++s >= s_end) return;
         sl = tg_ld_slot(P.slots + s);  // the chain's next edge departs from node tn
@@ -106,8 +118,85 @@ __device__ __forceinline__ void reach_edge(const ReachP &P, uint32_t p, unsigned
     }
 }
 
-// Warp per dirty vertex: prefix OR over the vertex's nodes (wait edges) from its first
-// dirty node; out-edges of the nodes whose word changed are relaxed (or queued).
+// Warp-cooperative scan of one dirty vertex with many departure nodes: prefix OR over
+// the vertex's nodes (wait edges) 32 at a time from its first dirty node; out-edges of
+// the nodes whose word changed are relaxed (or queued).
+__device__ void scan_vertex_warp(const ReachP &P, int ib, uint32_t j0, uint32_t j1, uint32_t vend, uint32_t *big_cnt) {
+    const int lane = threadIdx.x & 31;
+    unsigned long long carry = 0;
+    for (uint32_t jb = j0; jb < vend; jb += 32) {
+        const uint32_t j = jb + lane;
+        const bool valid = j < vend && __ldg(P.node_t + j) < P.omega;  // later nodes have no valid out-edge
+        bool dirty = false;
+        unsigned long long w = 0;
+        if (valid) {
+            const uint32_t bit = 1u << (j & 31);
+            // this round's dirty bits were all set in the previous round (marks of this
+            // round go to the other parity): a plain read decides, the clear is a RED
+            if (j <= j1 && (__ldcg(P.D[ib] + (j >> 5)) & bit)) {
+                dirty = true;
+                atomicAnd(P.D[ib] + (j >> 5), ~bit);
+            }
+            w = __ldcg(P.R + j);
+        }
+        // inclusive prefix OR of the chunk's words, with the carry of earlier chunks
+        unsigned long long incl = w;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl |= y;
+        }
+        unsigned long long excl = __shfl_up_sync(0xffffffffu, incl, 1);
+        if (lane == 0) excl = 0;
+        excl |= carry;
+        const unsigned long long add = valid ? (excl & ~w) : 0ull;
+        if (add) atomicOr(P.R + j, add);
+        const bool changed = valid && (add != 0 || dirty);
+        const unsigned long long nw_ = w | excl;  // the node's word after the wait edges
+        carry = __shfl_sync(0xffffffffu, incl, 31) | carry;
+        if (P.stats && lane == 0) atomicAdd(P.cnt + 1, (unsigned long long)min(32u, vend - jb));
+        const uint32_t cm = __ballot_sync(0xffffffffu, changed);
+        if (cm) {
+            const uint32_t lo = __ffs(cm) - 1, hi = 31 - __clz(cm);
+            const uint32_t p0 = __ldg(P.node_eoff + jb + lo), p1 = __ldg(P.node_eoff + jb + hi + 1);
+            if (p1 - p0 > RBIG) {
+                const uint32_t nch = (p1 - p0 + RCHUNK - 1) / RCHUNK;
+                uint32_t k = 0;
+                if (lane == 0) k = atomicAdd(big_cnt, nch);
+                k = __shfl_sync(0xffffffffu, k, 0);
+                for (uint32_t c = lane; c < nch; c += 32) {
+                    const uint32_t b0 = p0 + c * RCHUNK, b1 = min(p1, b0 + RCHUNK);
+                    if (k + c < P.bigcap) {
+                        P.bigq[k + c] = make_uint4(b0, b1, jb, cm);
+                    } else {
+                        for (uint32_t p = b0; p < b1; p++) {
+                            const uint32_t jn = __ldg(P.occ_node + p);
+                            if ((cm >> (jn - jb)) & 1u) reach_edge(P, p, __ldcg(P.R + jn));
+                        }
+                    }
+                }
+            } else {
+                for (uint32_t pb = p0; pb < p1; pb += 32) {
+                    const uint32_t p = pb + lane;
+                    const uint32_t jn = p < p1 ? __ldg(P.occ_node + p) : jb;
+                    const uint32_t src = jn - jb;  // owner node's lane in this chunk
+                    const unsigned long long ow = __shfl_sync(0xffffffffu, nw_, src);
+                    if (p < p1 && ((cm >> src) & 1u)) reach_edge(P, p, ow);
+                }
+            }
+        }
+        if (!__shfl_sync(0xffffffffu, valid, 31)) break;  // past the window or the node list
+        // past the last dirty node and the carry added nothing to the chunk's last
+        // node: later nodes already hold it (prefix-closed, or dirty for next round)
+        const bool last_ok = __shfl_sync(0xffffffffu, add == 0 && !dirty, 31);
+        if (jb + 31 >= j1 && last_ok) break;
+    }
+}
+
+// Round: lane per dirty vertex (most have a handful of departure nodes: the lane runs the
+// prefix OR over them serially, independent loads across the warp's 32 vertices); a
+// vertex with more than SCAN_LANE_MAX nodes left is scanned by the whole warp.
+constexpr uint32_t SCAN_LANE_MAX = 48;
 __global__ void __launch_bounds__(RT) k_reach_scan(ReachP P) {
     const int lane = threadIdx.x & 31;
     const uint32_t r = P.round;
@@ -117,74 +206,49 @@ __global__ void __launch_bounds__(RT) k_reach_scan(ReachP P) {
     uint32_t *big_cnt = &P.ctl->cnt[r & (TG_RING - 1)][1];
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
-    for (uint32_t i = gw; i < F; i += nw) {
-        const uint32_t v = P.vf[ib][i];
-        const uint32_t j0 = P.dmin[ib][v], j1 = P.dmax[ib][v];
-        __syncwarp();
-        if (lane == 0) { P.dmin[ib][v] = TG_NONE; P.dmax[ib][v] = 0; }
-        const uint32_t vend = __ldg(P.vnode_off + v + 1);
-        unsigned long long carry = 0;
-        for (uint32_t jb = j0; jb < vend; jb += 32) {
-            const uint32_t j = jb + lane;
-            const bool valid = j < vend && __ldg(P.node_t + j) < P.omega;  // later nodes have no valid out-edge
-            bool dirty = false;
-            unsigned long long w = 0;
-            if (valid) {
-                const uint32_t bit = 1u << (j & 31);
-                if (j <= j1 && (__ldcg(P.D[ib] + (j >> 5)) & bit)) dirty = (atomicAnd(P.D[ib] + (j >> 5), ~bit) & bit) != 0;
-                w = __ldcg(P.R + j);
-            }
-            // inclusive prefix OR of the chunk's words, with the carry of earlier chunks
-            unsigned long long incl = w;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, o);
-                if (lane >= o) incl |= y;
-            }
-            unsigned long long excl = __shfl_up_sync(0xffffffffu, incl, 1);
-            if (lane == 0) excl = 0;
-            excl |= carry;
-            const unsigned long long add = valid ? (excl & ~w) : 0ull;
-            if (add) atomicOr(P.R + j, add);
-            const bool changed = valid && (add != 0 || dirty);
-            const unsigned long long nw_ = w | excl;  // the node's word after the wait edges
-            carry = __shfl_sync(0xffffffffu, incl, 31) | carry;
-            if (P.stats && lane == 0) atomicAdd(P.cnt + 1, (unsigned long long)min(32u, vend - jb));
-            const uint32_t cm = __ballot_sync(0xffffffffu, changed);
-            if (cm) {
-                const uint32_t lo = __ffs(cm) - 1, hi = 31 - __clz(cm);
-                const uint32_t p0 = __ldg(P.node_eoff + jb + lo), p1 = __ldg(P.node_eoff + jb + hi + 1);
-                if (p1 - p0 > RBIG) {
-                    const uint32_t nch = (p1 - p0 + RCHUNK - 1) / RCHUNK;
-                    uint32_t k = 0;
-                    if (lane == 0) k = atomicAdd(big_cnt, nch);
-                    k = __shfl_sync(0xffffffffu, k, 0);
-                    for (uint32_t c = lane; c < nch; c += 32) {
-                        const uint32_t b0 = p0 + c * RCHUNK, b1 = min(p1, b0 + RCHUNK);
-                        if (k + c < P.bigcap) {
-                            P.bigq[k + c] = make_uint4(b0, b1, jb, cm);
-                        } else {
-                            for (uint32_t p = b0; p < b1; p++) {
-                                const uint32_t jn = __ldg(P.occ_node + p);
-                                if ((cm >> (jn - jb)) & 1u) reach_edge(P, p, __ldcg(P.R + jn));
-                            }
-                        }
-                    }
-                } else {
-                    for (uint32_t pb = p0; pb < p1; pb += 32) {
-                        const uint32_t p = pb + lane;
-                        const uint32_t jn = p < p1 ? __ldg(P.occ_node + p) : jb;
-                        const uint32_t src = jn - jb;  // owner node's lane in this chunk
-                        const unsigned long long ow = __shfl_sync(0xffffffffu, nw_, src);
-                        if (p < p1 && ((cm >> src) & 1u)) reach_edge(P, p, ow);
+    for (uint32_t base = gw * 32; base < F; base += nw * 32) {
+        const uint32_t i = base + lane;
+        uint32_t v = TG_NONE, j0 = 0, j1 = 0, vend = 0;
+        if (i < F) {
+            v = P.vf[ib][i];
+            j0 = P.dmin[ib][v];
+            j1 = P.dmax[ib][v];
+            P.dmin[ib][v] = TG_NONE;
+            P.dmax[ib][v] = 0;
+            vend = __ldg(P.vnode_off + v + 1);
+        }
+        const bool wide = v != TG_NONE && vend - j0 > SCAN_LANE_MAX;
+        if (v != TG_NONE && !wide) {
+            unsigned long long carry = 0;
+            for (uint32_t j = j0; j < vend; j++) {
+                if (__ldg(P.node_t + j) >= P.omega) break;  // no valid out-edge from here on
+                bool dirty = false;
+                if (j <= j1) {
+                    const uint32_t bit = 1u << (j & 31);
+                    if (__ldcg(P.D[ib] + (j >> 5)) & bit) {
+                        dirty = true;
+                        atomicAnd(P.D[ib] + (j >> 5), ~bit);
                     }
                 }
+                const unsigned long long w = __ldcg(P.R + j);
+                const unsigned long long add = carry & ~w;
+                if (add) atomicOr(P.R + j, add);
+                const unsigned long long nwv = w | carry;
+                if (add || dirty) {
+                    const uint32_t p0 = __ldg(P.node_eoff + j), p1 = __ldg(P.node_eoff + j + 1);
+                    for (uint32_t p = p0; p < p1; p++) reach_edge(P, p, nwv);
+                }
+                carry = nwv;
+                if (P.stats) atomicAdd(P.cnt + 1, 1ull);
+                if (j >= j1 && !add && !dirty) break;  // later nodes hold the carry already
             }
-            if (!__shfl_sync(0xffffffffu, valid, 31)) break;  // past the window or the node list
-            // past the last dirty node and the carry added nothing to the chunk's last
-            // node: later nodes already hold it (prefix-closed, or dirty for next round)
-            const bool last_ok = __shfl_sync(0xffffffffu, add == 0 && !dirty, 31);
-            if (jb + 31 >= j1 && last_ok) break;
+        }
+        uint32_t wm = __ballot_sync(0xffffffffu, wide);
+        while (wm) {
+            const int o = __ffs(wm) - 1;
+            wm &= wm - 1;
+            scan_vertex_warp(P, ib, __shfl_sync(0xffffffffu, j0, o), __shfl_sync(0xffffffffu, j1, o),
+                             __shfl_sync(0xffffffffu, vend, o), big_cnt);
         }
     }
 }
