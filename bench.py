@@ -66,6 +66,7 @@ def parse_args(argv=None):
     ap.add_argument("--exchange", type=int, default=0, help="vertex mode: cross-rank exchange algorithm")
     ap.add_argument("--cpu-threads", type=int, default=0, help="oracle threads (0 = all host cores)")
     ap.add_argument("--problems", default=None, help="comma list overriding the config's problems (e.g. reach)")
+    ap.add_argument("--reach-bits", action="store_true", help="TG_REACH on the bit-lane engine (option reach_bits)")
     ap.add_argument("--stream-blocks", type=int, default=0,
                     help="out-of-memory mode: the graph streamed from host memory in this many time blocks")
     return ap.parse_args(argv)
@@ -260,6 +261,8 @@ def run_ours(a, rank, world, local_rank):
             g.set_option("partitions", a.partitions)
         if a.exchange:
             g.set_option("exchange", 1)
+        if a.reach_bits:
+            g.set_option("reach_bits", 1)
         if comm is not None:
             tg.tg_graph_attach_comm(g.h, comm, 1)
         return g.build()
@@ -293,12 +296,12 @@ def run_ours(a, rank, world, local_rank):
     gstat.set_option("stats", 1)
     W_by_problem, Wu_by_problem = {}, {}
     for p in problems:
-        if p == "reach":
+        if p == "reach" and a.reach_bits:
             # the bit-lane engine's usable edges are the EAT union of the same batch
             gstat.query("eat", mine, win, out=outs[p])
             Wu_by_problem[p] = int(gstat.last_stats(k)["slots_union"])
             continue
-        if p not in ("eat", "ld"):
+        if p not in ("eat", "ld", "reach"):
             continue  # the first-touch work counters cover the EAT-family engine
         gstat.query(p, mine, win, out=outs[p])
         st = gstat.last_stats(k)
@@ -374,9 +377,10 @@ def run_ours(a, rank, world, local_rank):
         # bit-lane reach (f2): per usable edge one 16-B occurrence record, the 8-B head word
         # and the 8-B tail-node word (64 sources per word); per sub-batch the vertex words
         W_steps = W_local * a.steps
-        Wu_eat = sum(v for p, v in Wu_by_problem.items() if p != "reach") * a.steps
-        Wu_reach = Wu_by_problem.get("reach", 0) * a.steps
-        reach_bytes = 32 * Wu_reach + 8 * n * (-(-k // 64)) * a.steps * ("reach" in problems)
+        bits = "reach" in problems and a.reach_bits
+        Wu_eat = sum(v for p, v in Wu_by_problem.items() if not (p == "reach" and bits)) * a.steps
+        Wu_reach = Wu_by_problem.get("reach", 0) * a.steps if bits else 0
+        reach_bytes = (32 * Wu_reach + 8 * n * (-(-k // 64)) * a.steps) if bits else 0
         relax_bytes = 20 * Wu_eat + 4 * W_steps + reach_bytes
         relax_bytes_pk = 20 * Wu_eat + 8 * W_steps + reach_bytes
         Wu_steps = Wu_eat + Wu_reach
@@ -397,7 +401,7 @@ def run_ours(a, rank, world, local_rank):
             "peak_source": peak_src,
             "algorithmic_bytes_per_step": relax_bytes / a.steps,
             "algorithmic_bytes_formula": ("20 B x W_union + 4 B x sum_q W_q (SURVEY 8(d) batched source lanes, "
-                                          "u32 state as timed)") if "reach" not in problems else
+                                          "u32 state as timed)") if not ("reach" in problems and a.reach_bits) else
                                          "32 B x W_union + 8 B x n per 64-source word (bit-lane reach, DESIGN 5.5)",
             "achieved_packed_8B_formula": relax_bytes_pk / (relax_ms / 1e3) / 1e9 if relax_ms else None,
             "W_union_per_step": Wu_steps / a.steps,

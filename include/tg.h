@@ -122,8 +122,9 @@ TG_API tg_status tg_build_chains(tg_graph *g);
  *               Unreached vertices read TG_UNREACHED (REACH: 0).
  *   pred        NULL or uint32[n_sources * n_vertices] (host or device), only
  *               for TG_EAT / TG_LD / TG_REACH (else TG_ERR_INVALID).  TG_REACH with
- *               pred == NULL runs on the bit-lane engine (64 sources per u64 word
- *               over the departure nodes).  EAT/REACH: the smallest
+ *               pred == NULL and option "reach_bits" = 1 runs on the bit-lane engine
+ *               (64 sources per u64 word over the departure nodes).
+ *               EAT/REACH: the smallest
  *               edge id among valid edges e=(u->v) with EAT(u) <= t_e and
  *               t_e + duration_e = EAT(v); LD: the smallest id among first
  *               edges of latest-departure paths (reading A9).  Source/target
@@ -284,6 +285,10 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *                partition then derives its next frontier from the combined state, as
  *                the ranks of a multi-GPU run do (tests; default 0: one process shares
  *                one state and frontier)
+ *   "reach_bits" 1 = TG_REACH without pred runs the bit-lane engine: one bit per (departure
+ *                node, source), 64 sources per u64 word (8 B per node per 64 sources instead of
+ *                4 B of arrival + 4 B of boundary per (vertex, source)); default 0: the EAT
+ *                engine, which is faster on the measured configs
  *   "dynamic"    1 = keep each direction's sorted edge order (before build; 4 B per edge
  *                and direction) so tg_graph_insert_edges re-transforms incrementally
  *   "packed_state" 1 = EAT/LD/REACH keep the packed u64 (arrival << 32 | pred) state even

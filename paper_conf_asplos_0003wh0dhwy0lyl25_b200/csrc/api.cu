@@ -412,7 +412,7 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
         }
         return tg_run_eat_partitioned(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     }
-    if (p == TG_REACH && !pred) return tg_run_reach_bits(g, sources, n_sources, w, out, out_dev, s);
+    if (p == TG_REACH && !pred && g->opt_reach_bits) return tg_run_reach_bits(g, sources, n_sources, w, out, out_dev, s);
     if (p == TG_EAT || p == TG_LD || p == TG_REACH) {
         return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     }
@@ -578,6 +578,7 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     }
     else if (k == "exchange") g->opt_exchange = value ? 1 : 0;
     else if (k == "packed_state") g->opt_packed_state = value ? 1 : 0;
+    else if (k == "reach_bits") g->opt_reach_bits = value ? 1 : 0;
     else if (k == "dynamic") {
         if (g->built) { tg_set_error("set dynamic before tg_build_chains"); return TG_ERR_STATE; }
         g->opt_dynamic = value ? 1 : 0;

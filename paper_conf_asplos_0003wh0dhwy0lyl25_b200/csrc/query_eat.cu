@@ -56,6 +56,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_MLP
 #define TG_MLP 4                        // state reads in flight per lane in the pair loop
 #endif
+#ifndef TG_GAP_SKIP
+#define TG_GAP_SKIP 1                   // jump over union gaps no query lane's range covers
+#endif
 #ifndef TG_COOP_SEARCH
 #define TG_COOP_SEARCH 1                // warp-cooperative departure-time search in the activation
 #endif
@@ -236,7 +239,17 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         atomicAdd(P.diag + 0, (unsigned long long)(pend - pbeg));
         atomicAdd(P.diag + 1, 1ull);
     }
-    for (uint32_t pb = pbeg; pb < pend; pb += 32) {
+    for (uint32_t pb = pbeg; pb < pend;) {
+        // gaps between the query lanes' ranges (a re-activated query's new segment far
+        // below another query's suffix) are jumped over, not scanned
+#if TG_GAP_SKIP
+        {
+            const uint32_t nxt = (lo < hi && hi > pb) ? max(lo, pb) : 0xFFFFFFFFu;
+            const uint32_t first = __reduce_min_sync(0xffffffffu, nxt);
+            if (first >= pend) break;
+            pb = first;
+        }
+#endif
         const uint32_t p = pb + lane;
         uint32_t s = 0;
         int4 sl = make_int4(0, -1, 0, 0);
@@ -269,7 +282,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
             if (lane >= o) incl += y;
         }
         const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-        if (total == 0) continue;
+        if (total == 0) { pb += 32; continue; }
         if (P.stats && lane == 0) atomicAdd(P.diag + 2, (unsigned long long)total);
         // expand: edge lane k writes its pairs at [incl - cnt, incl) in edge-major order
         ws.slot[lane] = sl;
@@ -313,6 +326,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
             }
         }
         __syncwarp();
+        pb += 32;
     }
 }
 

@@ -193,10 +193,8 @@ __device__ void scan_vertex_warp(const ReachP &P, int ib, uint32_t j0, uint32_t 
     }
 }
 
-// Round: lane per dirty vertex (most have a handful of departure nodes: the lane runs the
-// prefix OR over them serially, independent loads across the warp's 32 vertices); a
-// vertex with more than SCAN_LANE_MAX nodes left is scanned by the whole warp.
-constexpr uint32_t SCAN_LANE_MAX = 48;
+// Round: warp per dirty vertex (a lane-per-vertex serial scan measured 1.7x slower:
+// every node of a lane's vertex is a dependent step).
 __global__ void __launch_bounds__(RT) k_reach_scan(ReachP P) {
     const int lane = threadIdx.x & 31;
     const uint32_t r = P.round;
@@ -206,50 +204,12 @@ __global__ void __launch_bounds__(RT) k_reach_scan(ReachP P) {
     uint32_t *big_cnt = &P.ctl->cnt[r & (TG_RING - 1)][1];
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
-    for (uint32_t base = gw * 32; base < F; base += nw * 32) {
-        const uint32_t i = base + lane;
-        uint32_t v = TG_NONE, j0 = 0, j1 = 0, vend = 0;
-        if (i < F) {
-            v = P.vf[ib][i];
-            j0 = P.dmin[ib][v];
-            j1 = P.dmax[ib][v];
-            P.dmin[ib][v] = TG_NONE;
-            P.dmax[ib][v] = 0;
-            vend = __ldg(P.vnode_off + v + 1);
-        }
-        const bool wide = v != TG_NONE && vend - j0 > SCAN_LANE_MAX;
-        if (v != TG_NONE && !wide) {
-            unsigned long long carry = 0;
-            for (uint32_t j = j0; j < vend; j++) {
-                if (__ldg(P.node_t + j) >= P.omega) break;  // no valid out-edge from here on
-                bool dirty = false;
-                if (j <= j1) {
-                    const uint32_t bit = 1u << (j & 31);
-                    if (__ldcg(P.D[ib] + (j >> 5)) & bit) {
-                        dirty = true;
-                        atomicAnd(P.D[ib] + (j >> 5), ~bit);
-                    }
-                }
-                const unsigned long long w = __ldcg(P.R + j);
-                const unsigned long long add = carry & ~w;
-                if (add) atomicOr(P.R + j, add);
-                const unsigned long long nwv = w | carry;
-                if (add || dirty) {
-                    const uint32_t p0 = __ldg(P.node_eoff + j), p1 = __ldg(P.node_eoff + j + 1);
-                    for (uint32_t p = p0; p < p1; p++) reach_edge(P, p, nwv);
-                }
-                carry = nwv;
-                if (P.stats) atomicAdd(P.cnt + 1, 1ull);
-                if (j >= j1 && !add && !dirty) break;  // later nodes hold the carry already
-            }
-        }
-        uint32_t wm = __ballot_sync(0xffffffffu, wide);
-        while (wm) {
-            const int o = __ffs(wm) - 1;
-            wm &= wm - 1;
-            scan_vertex_warp(P, ib, __shfl_sync(0xffffffffu, j0, o), __shfl_sync(0xffffffffu, j1, o),
-                             __shfl_sync(0xffffffffu, vend, o), big_cnt);
-        }
+    for (uint32_t i = gw; i < F; i += nw) {
+        const uint32_t v = P.vf[ib][i];
+        const uint32_t j0 = P.dmin[ib][v], j1 = P.dmax[ib][v];
+        __syncwarp();
+        if (lane == 0) { P.dmin[ib][v] = TG_NONE; P.dmax[ib][v] = 0; }
+        scan_vertex_warp(P, ib, j0, j1, __ldg(P.vnode_off + v + 1), big_cnt);
     }
 }
 

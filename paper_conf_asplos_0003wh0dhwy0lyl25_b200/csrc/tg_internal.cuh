@@ -237,6 +237,7 @@ struct tg_graph {
     int opt_mirror = 1;
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
+    int64_t opt_reach_bits = 0;  // 1 = TG_REACH without pred on the bit-lane engine (query_reach.cu)
     int64_t opt_dynamic = 0;   // 1 = keep each direction's sorted edge order for tg_graph_insert_edges
     int64_t opt_walk_min = 6;  // chains with fewer edges are not walked (RemoveChain threshold, build time)
     bool mirror_built = false;

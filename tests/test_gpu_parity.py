@@ -513,7 +513,7 @@ def test_reach_bitlane_random(tg, seed):
     n, u, v, t, lam, w = tgsynth.tiny_random(seed + 6100, n_max=120, m_max=2500, t_max=60, lam_max=6)
     og = oracle.Graph(n, u, v, t, lam, w)
     for opts in ({}, {"walk_min": 2}, {"relabel": 1}):
-        g = _gpu_graph(tg, n, u, v, t, lam, w, **opts)
+        g = _gpu_graph(tg, n, u, v, t, lam, w, reach_bits=1, **opts)
         srcs = list(range(min(n, 100)))
         for win in [(0, 10**6), (5, 40), (7, 7), (20, 21)]:
             _check_reach(tg, g, og, srcs, win)
@@ -534,7 +534,7 @@ def test_reach_bitlane_hubs_and_host(tg):
     parts.append((np.full(50, 5), np.full(50, 5), np.arange(50), np.ones(50)))  # self-loops
     u, v, t, lam = (np.concatenate([p[i] for p in parts]).astype(np.uint32) for i in range(4))
     og = oracle.Graph(n, u, v, t, lam)
-    g = _gpu_graph(tg, n, u, v, t, lam, walk_min=2)
+    g = _gpu_graph(tg, n, u, v, t, lam, walk_min=2, reach_bits=1)
     srcs = [0, 1, 5] + [int(x) for x in rng.choice(n, 70, replace=False)]
     for win in [(0, 10**6), (100, 2000)]:
         _check_reach(tg, g, og, srcs, win)
@@ -545,12 +545,13 @@ def test_reach_bitlane_hubs_and_host(tg):
 def test_reach_bitlane_c2_small(tg):
     ge = tgsynth.make_graph("C2", scale_shift=-4)
     n, u, v, t, d, w = ge.numpy()
-    g = _gpu_graph(tg, n, u, v, t, d)
     og = oracle.Graph(n, u, v, t, d)
     srcs = tgsynth.config_sources("C2", ge)
-    for win in tgsynth.CONFIGS["C2"]["windows"]:
-        _check_reach(tg, g, og, srcs, win)
-    g.close()
+    for bits in (1, 0):
+        g = _gpu_graph(tg, n, u, v, t, d, reach_bits=bits)
+        for win in tgsynth.CONFIGS["C2"]["windows"]:
+            _check_reach(tg, g, og, srcs, win)
+        g.close()
 
 
 # --------------------------------------------------------------------------- f4: LDS, top-K, summaries
@@ -632,7 +633,7 @@ def test_insert_edges_incremental(tg, seed):
     cols = lambda m, tmax: (rng.integers(0, n, m), rng.integers(0, n, m), rng.integers(0, tmax, m),
                             rng.integers(1, 7, m), rng.integers(0, 9, m))
     U, V, T, L, W = (np.asarray(c, np.uint32) for c in cols(m0, 200))
-    g = _gpu_graph(tg, n, U, V, T, L, W, dynamic=1)
+    g = _gpu_graph(tg, n, U, V, T, L, W, dynamic=1, reach_bits=1)
     for b, (k, tmax) in enumerate([(500, 200), (1200, 400), (1, 50), (800, 600)]):
         bu, bv, bt, bl, bw = (np.asarray(c, np.uint32) for c in cols(k, tmax))
         g.insert_edges(_t32(bu), _t32(bv), _t32(bt), _t32(bl), _t32(bw))
