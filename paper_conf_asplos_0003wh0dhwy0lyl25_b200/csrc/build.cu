@@ -487,17 +487,17 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
         // the virtualised GPU boxes (TG_TRACE_BUILD), so it is only the fallback
         size_t fr = 0, tot = 0;
         bool room = false;
-        {
-            int dev = 0;
-            cudaGetDevice(&dev);
-            cudaMemPool_t pool;
-            uint64_t reserved = 0, used = 0;
-            if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess &&
-                cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved) == cudaSuccess &&
-                cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used) == cudaSuccess)
-                room = reserved >= used && reserved - used >= m * 16 + (1ull << 20);
-            cudaGetLastError();
-        }
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaMemPool_t pool = nullptr;
+        uint64_t reserved = 0, used = 0;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess &&
+            cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved) == cudaSuccess &&
+            cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used) == cudaSuccess)
+            room = reserved >= used && reserved - used >= m * 16 + (1ull << 20);
+        else
+            pool = nullptr;
+        cudaGetLastError();
         if (!room) {
             cudaMemGetInfo(&fr, &tot);
             room = fr > m * 16 + (4ull << 30);
@@ -506,6 +506,19 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
             cudaGetLastError();
             srec = nullptr;
         }
+        // the pool's unused reserve may be fragmented: if the copy made the pool grow, keep
+        // the old 4 GB device headroom for the arrays this build still allocates, else fall
+        // back to the gather path
+        uint64_t reserved2 = 0;
+        if (srec && pool && cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved2) == cudaSuccess &&
+            reserved2 > reserved) {
+            cudaMemGetInfo(&fr, &tot);
+            if (fr < (4ull << 30)) {
+                cudaFreeAsync(srec, s);
+                srec = nullptr;
+            }
+        }
+        cudaGetLastError();
     }
     bmark(s, "memgetinfo");
     TG_LAUNCH(k_snap, blocks_for(m, 4 * TG_SNAP_ILP), BT, 0, s, sid, m, rec, cg->vnode_off, cg->node_t, tn, indeg, srec);
