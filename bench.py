@@ -38,7 +38,8 @@ import numpy as np  # noqa: E402
 HBM_FALLBACK_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
 METRIC = "temporal-path queries/s (EAT; plus LD/FP/SP where the config lists them)"
 UNIT = "queries/s"
-RELAX_KERNELS = ("k_eat_activate", "k_eat_big", "k_eat_chain", "k_reach_scan", "k_reach_big")
+RELAX_KERNELS = ("k_eat_activate", "k_eat_big", "k_eat_chain", "k_reach_scan", "k_reach_big", "k_spfp_activate",
+                 "k_spfp_wait", "k_spfp_big")
 
 
 def parse_args(argv=None):
@@ -294,12 +295,18 @@ def run_ours(a, rank, world, local_rank):
     # work counts (untimed): W per query from the engine's first-touch counter (== oracle W, tested)
     gstat = persistent or make_graph()
     gstat.set_option("stats", 1)
-    W_by_problem, Wu_by_problem = {}, {}
+    W_by_problem, Wu_by_problem, SPFP = {}, {}, {}
     for p in problems:
         if p == "reach" and a.reach_bits:
             # the bit-lane engine's usable edges are the EAT union of the same batch
             gstat.query("eat", mine, win, out=outs[p])
             Wu_by_problem[p] = int(gstat.last_stats(k)["slots_union"])
+            continue
+        if p in ("sp", "fp", "lds"):
+            # node-state engine: chain-slot relaxations and wait-edge steps
+            gstat.query(p, mine, win, out=outs[p])
+            st = gstat.last_stats(k)
+            SPFP[p] = (int(st["slots_relaxed"]), int(st["slots_union"]))
             continue
         if p not in ("eat", "ld", "reach"):
             continue  # the first-touch work counters cover the EAT-family engine
@@ -381,8 +388,12 @@ def run_ours(a, rank, world, local_rank):
         Wu_eat = sum(v for p, v in Wu_by_problem.items() if not (p == "reach" and bits)) * a.steps
         Wu_reach = Wu_by_problem.get("reach", 0) * a.steps if bits else 0
         reach_bytes = (32 * Wu_reach + 8 * n * (-(-k // 64)) * a.steps) if bits else 0
-        relax_bytes = 20 * Wu_eat + 4 * W_steps + reach_bytes
-        relax_bytes_pk = 20 * Wu_eat + 8 * W_steps + reach_bytes
+        # SP / FP / LDS: per chain-slot relaxation the 16-B slot, the 4-B tail
+        # node id and weight, the 4-B node state and the 4-B vertex output; per wait step the
+        # 4-B departure time and the 4-B node state
+        spfp_bytes = sum(32 * r + 8 * wst for r, wst in SPFP.values()) * a.steps
+        relax_bytes = 20 * Wu_eat + 4 * W_steps + reach_bytes + spfp_bytes
+        relax_bytes_pk = 20 * Wu_eat + 8 * W_steps + reach_bytes + spfp_bytes
         Wu_steps = Wu_eat + Wu_reach
         traffic = None
         tf = os.path.join(ROOT, "profiles", "round2", f"relax_traffic_{a.config}.json")
@@ -403,7 +414,9 @@ def run_ours(a, rank, world, local_rank):
             "algorithmic_bytes_formula": ("20 B x W_union + 4 B x sum_q W_q (SURVEY 8(d) batched source lanes, "
                                           "u32 state as timed)") if not ("reach" in problems and a.reach_bits) else
                                          "32 B x W_union + 8 B x n per 64-source word (bit-lane reach, DESIGN 5.5)",
+            "algorithmic_bytes_formula_spfp": "32 B x chain-slot relaxations + 8 B x wait steps (SP/FP/LDS)",
             "achieved_packed_8B_formula": relax_bytes_pk / (relax_ms / 1e3) / 1e9 if relax_ms else None,
+            "spfp_relax_and_wait_steps_per_step": {p: list(v) for p, v in SPFP.items()},
             "W_union_per_step": Wu_steps / a.steps,
             "W_sum_per_step": W_steps / a.steps,
             "relax_ms_per_step": relax_ms / a.steps,

@@ -236,7 +236,9 @@ typedef struct {
     uint64_t slots_relaxed;   /* relaxations performed (when stats are enabled)              */
     uint64_t kernel_launches; /* kernels launched by the last tg_query                       */
     uint64_t slots_union;     /* distinct slots relaxed by any query of a sub-batch, summed over
-                                 sub-batches (stats enabled; EAT/LD): W_union of SURVEY 8(d)  */
+                                 sub-batches (stats enabled; EAT/LD): W_union of SURVEY 8(d).
+                                 SP/FP/LD_SOURCE: slots_relaxed = chain-slot relaxations,
+                                 slots_union = wait-edge steps (node states updated by waiting) */
 } tg_query_stats;
 
 /* Statistics of the last tg_query on this handle.  If per_query_relax is not

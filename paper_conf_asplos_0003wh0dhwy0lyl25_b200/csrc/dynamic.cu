@@ -14,6 +14,9 @@
 // The mirror's order is unaffected by a larger C (C - a keeps its order), so its
 // kept order is merged the same way.
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 
 #include "tg_internal.cuh"
 
@@ -76,6 +79,18 @@ __global__ void k_mirror_times(const uint32_t *__restrict__ t, const uint32_t *_
         mt[i] = C - (t[i] + dur[i]);
 }
 
+// TG_TRACE_BUILD=1: synchronise at the insertion's section boundaries and print the
+// host time of each section (diagnostics)
+void dmark(const char *label) {
+    static const bool on = getenv("TG_TRACE_BUILD") != nullptr;
+    if (!on) return;
+    static std::chrono::steady_clock::time_point last;
+    cudaDeviceSynchronize();
+    const auto now = std::chrono::steady_clock::now();
+    if (label) fprintf(stderr, "insert-trace %s %.3f\n", label, std::chrono::duration<double, std::milli>(now - last).count());
+    last = now;
+}
+
 int bits_of(uint64_t x) {
     int b = 0;
     while (b < 64 && (x >> b) != 0) b++;
@@ -132,6 +147,7 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
     if (prev != g->device) cudaSetDevice(g->device);
     cudaStream_t s = 0;
     TG_TRY_CUDA(cudaDeviceSynchronize());
+    dmark(nullptr);
     const uint64_t m_old = g->m, m_new = g->m + k;
     // 1. the new edge arrays: the kept edges, then the batch (ids m_old .. m_new - 1)
     DevArena na;
@@ -147,6 +163,7 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
         TG_TRY_CUDA(cudaMemcpyAsync(*dst[i] + m_old, src[i], k * 4, cudaMemcpyDefault, s));
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
+    dmark("copy");
     // swap in; validation over all edges (updates max t / arrival / weight, the SP bound)
     std::swap(g->arena, na);
     g->d_u = nu; g->d_v = nv; g->d_t = nt; g->d_dur = nd; g->d_w = nw;
@@ -164,6 +181,7 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
         return vs;
     }
     na.free_all();  // the old edge arrays
+    dmark("validate");
     // query scratch is sized by m / nodes: rebuilt lazily by the next query
     TG_TRY_CUDA(cudaDeviceSynchronize());
     g->qs.arena.free_all();
@@ -172,6 +190,7 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);
     g->rs = ReachScratch{};
+    dmark("scratch");
     if (!g->built) return TG_OK;
     // 2./3. incremental re-transformation of each built direction
     uint32_t *ord = nullptr, *mt = nullptr;
@@ -179,10 +198,12 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
     {
         TG_TRY(merged_order(g->d_u, g->d_t, g->max_t, g->n, g->fwd.order, m_old, m_new, ord, s));
         TG_TRY_CUDA(cudaStreamSynchronize(s));
+        dmark("merge");
         g->fwd.arena.free_all();
         g->fwd = ChainGraph{};
         TG_TRY(tg_build_direction(g, &g->fwd, m_new, g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w, nullptr, g->max_t, s,
                                   ord));
+        dmark("rebuild");
     }
     if (g->mirror_built) {
         // reading A5's mirror with the (possibly larger) C = max(t + lambda)

@@ -56,6 +56,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_MLP
 #define TG_MLP 4                        // state reads in flight per lane in the pair loop
 #endif
+#ifndef TG_DEFER
+#define TG_DEFER 0                      // experiment (0 = off): defer units with fewer new queries one round
+#endif
 #ifndef TG_GAP_SKIP
 #define TG_GAP_SKIP 1                   // jump over union gaps no query lane's range covers
 #endif
@@ -75,6 +78,7 @@ struct EatP {
     void *st;  // [v * S + q]: packed u64 (arrival << 32 | pred) when PK, else u32 arrival
     uint32_t *act, *bits;
     uint32_t *touched;  // stats: slots relaxed by any query of the sub-batch
+    uint32_t *defer;    // TG_DEFER experiment: units deferred once (bit per unit)
     uint64_t bit_words;
     uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
     uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
@@ -354,6 +358,26 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         if (word) R.fin[ui] = 0u;  // consume
         uint32_t pending = __ballot_sync(0xffffffffu, word != 0);
         my_units += (lane == 0) ? __popc(pending) : 0u;
+#if TG_DEFER
+        // experiment: a unit with few new queries in a bulk round waits one round (its
+        // word moves to the next frontier) so that more of its group's queries share one
+        // scan of its edges; a unit is deferred at most once in a row
+        if (word && P.round >= 3 && P.defer) {
+            const uint32_t bit = 1u << (ui & 31);
+            uint32_t *dw = P.defer + (ui >> 5);
+            if (__popc(word) < TG_DEFER) {
+                if (!(atomicOr(dw, bit) & bit)) {
+                    atomicOr(R.fout + ui, word);
+                    word = 0;
+                } else {
+                    atomicAnd(dw, ~bit);
+                }
+            } else if (__ldcg(dw) & bit) {
+                atomicAnd(dw, ~bit);
+            }
+        }
+        pending = __ballot_sync(0xffffffffu, word != 0);
+#endif
         while (pending) {
             const int sl = __ffs(pending) - 1;
             pending &= pending - 1;
@@ -861,6 +885,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     Q.vwords = (uint32_t)((S + 31) / 32);  // query groups per vertex
     TG_TRY(A.alloc((void **)&Q.fb[0], n * Q.vwords * 4));
     TG_TRY(A.alloc((void **)&Q.fb[1], n * Q.vwords * 4));
+    if (TG_DEFER) TG_TRY(A.alloc((void **)&Q.defer, (n * Q.vwords + 31) / 32 * 4 + 4));
     if (nodes_state) {
         const uint64_t mark_len = S * nnodes;
         TG_TRY(A.alloc((void **)&Q.mark, std::max<uint64_t>(mark_len, 1) * 4));
@@ -946,6 +971,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     const uint32_t G = (S + 31) / 32;
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
+    if (TG_DEFER) TG_TRY_CUDA(cudaMemsetAsync(Q.defer, 0, (n * G + 31) / 32 * 4 + 4, s));
     if (g->opt_stats) {
         TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8 + 8 + 64, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, Q.bit_words * 4, s));
@@ -979,6 +1005,7 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         P.touched = Q.touched;
+        P.defer = Q.defer;
         P.diag = Q.relax_cnt + S + 1;
         const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;

@@ -62,6 +62,8 @@ struct SpP {
     uint64_t bigcap;
     uint4 *waitq;  // long wait-propagation walks {q, next node, vertex end, value}
     uint64_t waitcap;
+    unsigned long long *cnt;  // stats: [0] chain-slot relaxations [1] wait-edge steps
+    int stats;
 };
 
 struct RoundV {
@@ -113,6 +115,7 @@ __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s,
     uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
     uint32_t *vo = P.vout + (size_t)q * P.n;
     for (; s < s_end; s++) {
+        if (P.stats) atomicAdd(P.cnt + 0, 1ull);
         const int4 sl = tg_ld_slot(P.slots + s);
         const uint32_t arr = (uint32_t)sl.y;
         if (arr > P.omega) return;
@@ -203,6 +206,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             bool more = false;
             for (uint32_t steps = 0; jend < vend;) {
                 if (__ldg(P.node_t + jend) >= P.omega) break;  // no valid out-edge departs at >= omega
+                if (P.stats) atomicAdd(P.cnt + 1, 1ull);
                 const uint32_t old = atomicMin(dn + jend, d);
                 if (old <= d) break;
                 jend++;
@@ -283,6 +287,7 @@ __global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
             const uint32_t jj = j + lane;
             bool stop = true, improved = false;
             if (jj < vend && __ldg(P.node_t + jj) < P.omega) {
+                if (P.stats) atomicAdd(P.cnt + 1, 1ull);
                 const uint32_t old = atomicMin(dn + jj, d);
                 improved = old > d;
                 stop = !improved;
@@ -379,6 +384,7 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     P.ctl = Q.ctl; P.fr0 = Q.fr[0]; P.fr1 = Q.fr[1];
     P.bigq = Q.bigq; P.bigcap = Q.bigcap;
     P.waitq = Q.chq; P.waitcap = Q.chcap;
+    P.cnt = Q.relax_cnt; P.stats = (int)g->opt_stats;
     TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl);
     // rounds and dedupe stamps are host counters passed with each launch; stamps only
     // grow (marks of earlier rounds and loops never match)
@@ -401,11 +407,11 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
             P.round = r;
             P.stamp = ++Q.stamp;
             if (trace) cudaEventRecord(tev[0], s);
-            TG_LAUNCH(k_spfp_activate<MODE>, grid, QT, 0, s, P);
+            TG_LAUNCH_RELAX(k_spfp_activate<MODE>, grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[1], s);
-            TG_LAUNCH(k_spfp_wait<MODE>, grid, QT, 0, s, P);
+            TG_LAUNCH_RELAX(k_spfp_wait<MODE>, grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[2], s);
-            TG_LAUNCH(k_spfp_big<MODE>, grid, QT, 0, s, P);
+            TG_LAUNCH_RELAX(k_spfp_big<MODE>, grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[3], s);
         }
         TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
@@ -443,10 +449,18 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
         const uint32_t Sb = std::min(S, k - b0);
         TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
         uint32_t rounds = 0;
+        if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, 16, s));
         if (mode == 1) TG_TRY((spfp_rounds<1>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
         else if (mode == 2) TG_TRY((spfp_rounds<2>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
         else TG_TRY((spfp_rounds<0>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
         g->last.rounds = std::max(g->last.rounds, rounds);
+        if (g->opt_stats) {  // chain-slot relaxations and wait-edge steps (bench roofline)
+            unsigned long long h[2];
+            TG_TRY_CUDA(cudaMemcpyAsync(h, Q.relax_cnt, 16, cudaMemcpyDeviceToHost, s));
+            TG_TRY_CUDA(cudaStreamSynchronize(s));
+            g->last.slots_relaxed += h[0];
+            g->last.slots_union += h[1];
+        }
         g->last.sub_batches++;
         const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
         uint32_t *o = out_dev ? out + (size_t)b0 * n : nullptr, *no_pred = nullptr;

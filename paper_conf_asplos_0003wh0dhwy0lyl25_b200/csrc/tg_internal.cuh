@@ -139,6 +139,7 @@ struct QueryScratch {
     uint32_t *ctr = nullptr;   // counters [2][4] (SP/FP host-driven loop)
     struct RoundCtl *ctl = nullptr;  // device-side round control (EAT family), [TG_MAXP]
     uint32_t *lat = nullptr;         // partitioned mode: last activated arrival [v][q]
+    uint32_t *defer = nullptr;       // TG_DEFER experiment: units deferred once
     uint32_t *pcount = nullptr;      // partitioned mode: frontier bits of the next round
     uint32_t *h_ctr = nullptr; // pinned host mirror
     uint32_t *srcs = nullptr;  // [S] sources of the sub-batch (caller's vertex ids)

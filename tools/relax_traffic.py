@@ -1,31 +1,49 @@
-"""Relax-phase DRAM traffic per bench step from ncu launch lists of one EAT and one
-LD batch (tools/prof_query.py), written to profiles/<round>/relax_traffic_<cfg>.json
-for bench.py's roofline "traffic" field.
+"""Fold an ncu --csv launch log of the relax kernels (gpu__time_duration, dram bytes) of one
+64-source query into profiles/round2/relax_traffic_<CFG>.json, the `traffic` of bench.py's
+roofline: DRAM bytes per bench step = per-query bytes x queries per step / 64.
 
-    ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
-        -k regex:"k_eat_(activate|big|chain)" --csv --log-file eat.csv python tools/prof_query.py --problem eat
-    (same for ld) ; python tools/relax_traffic.py C2 eat.csv ld.csv profiles/round1
-"""
+usage: python tools/relax_traffic.py LOG.csv CFG SUBBATCHES_PER_STEP"""
+import collections
+import csv
 import json
 import os
 import sys
 
-sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
-from launches import load  # noqa: E402
-
-cfg, files, outdir = sys.argv[1], sys.argv[2:-1], sys.argv[-1]
-tot_b = tot_t = 0.0
-n = 0
-for f in files:
-    L = load(f)
-    for d in L.values():
-        tot_b += d.get("dram__bytes_read.sum", 0.0) + d.get("dram__bytes_write.sum", 0.0)
-        tot_t += d.get("gpu__time_duration.sum", 0.0)
-        n += 1
-res = {"config": cfg, "bytes_per_step": tot_b, "kernel_ns_per_step_under_ncu": tot_t, "launches": n,
-       "batches": [os.path.basename(f) for f in files],
-       "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum over k_eat_(activate|big|chain), "
-                 "one EAT and one LD batch of the bench step (cold-cache, serialised replay)"}
-os.makedirs(outdir, exist_ok=True)
-json.dump(res, open(os.path.join(outdir, f"relax_traffic_{cfg}.json"), "w"), indent=1)
-print(res)
+log, cfg, per_step = sys.argv[1], sys.argv[2], float(sys.argv[3])
+rows = [r for r in csv.reader(open(log)) if len(r) > 10]
+hdr = rows[0]
+ix = {k: i for i, k in enumerate(hdr)}
+acc = collections.defaultdict(lambda: collections.Counter())
+for r in rows[1:]:
+    if r[ix["Metric Name"]] not in ("gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum"):
+        continue
+    name = r[ix["Kernel Name"]].split("(")[0].replace("void ", "").replace("<unnamed>::", "")
+    unit = r[ix["Metric Unit"]]
+    v = float(r[ix["Metric Value"]].replace(",", ""))
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-6, "usecond": 1e-3, "ns": 1e-6, "us": 1e-3, "ms": 1.0,
+             "msecond": 1.0}.get(unit, 1.0)
+    key = r[ix["Metric Name"]]
+    acc[name][key] += v * scale
+    if key == "gpu__time_duration.sum":
+        acc[name]["launches"] += 1
+tot = collections.Counter()
+for k in acc.values():
+    tot.update(k)
+dram = tot["dram__bytes_read.sum"] + tot["dram__bytes_write.sum"]
+out = {
+    "config": cfg,
+    "dram_bytes_per_subbatch": dram,
+    "dram_bytes_per_step": dram * per_step,
+    "ncu_ms_per_subbatch": tot["gpu__time_duration.sum"],
+    "ncu_GBps": dram / (tot["gpu__time_duration.sum"] / 1e3) / 1e9 if tot["gpu__time_duration.sum"] else None,
+    "per_kernel": {k: {"launches": int(v["launches"]), "ms": round(v["gpu__time_duration.sum"], 3),
+                       "dram_GB": round((v["dram__bytes_read.sum"] + v["dram__bytes_write.sum"]) / 1e9, 3)}
+                   for k, v in acc.items()},
+    "source": (f"ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum over every "
+               f"k_eat_(activate|big|chain) launch of one 64-source EAT query (tools/prof_query.py --config {cfg}), "
+               f"serialised cold-cache replay; x{per_step:g} sub-batches per bench step"),
+}
+dst = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "round2",
+                   f"relax_traffic_{cfg}.json")
+json.dump(out, open(dst, "w"), indent=1)
+print(json.dumps(out, indent=1))
