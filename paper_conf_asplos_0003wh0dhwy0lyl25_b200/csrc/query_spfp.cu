@@ -134,9 +134,10 @@ __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s,
         if (vo[sl.x] > val) atomicMin(vo + sl.x, val);  // stale read is an upper bound
         const uint32_t tn = __ldg(P.slot_tn + s);
         if (tn == TG_NONE) return;  // sink
-        if (dn[tn] <= cand) return;  // not improved (stale read is an upper bound)
-        const uint32_t old = atomicMin(dn + tn, cand);
-        if (cand >= old) return;    // not improved: the improver pushed tn
+        if (__ldcg(dn + tn) <= cand) return;  // not improved (stale read is an upper bound)
+        // improved as far as this read knows: min (a reduction) and push; a concurrent
+        // better value only makes this walk redundant (push dedupes by stamp)
+        atomicMin(dn + tn, cand);
         push_node(P, R, q, tn);     // wait propagation + other out-edges next round
         cur = cand;
     }
@@ -171,9 +172,9 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_
                     cand = cur + (uint32_t)__ldg(P.sc_sumw + l);
                     atomicMin(P.vout + (size_t)q * P.n + scv.x, cand);
                 }
-                if (tn != TG_NONE) {
-                    const uint32_t old = atomicMin(P.dnode + (size_t)q * P.nnodes + tn, cand);
-                    if (cand < old) push_node(P, R, q, tn);
+                if (tn != TG_NONE && __ldcg(P.dnode + (size_t)q * P.nnodes + tn) > cand) {
+                    atomicMin(P.dnode + (size_t)q * P.nnodes + tn, cand);
+                    push_node(P, R, q, tn);
                 }
             }
         }
@@ -204,13 +205,34 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             // the first WAIT_INLINE nodes here, the rest by a warp in k_spfp_wait
             uint32_t jend = j + 1;
             bool more = false;
+            // plain (stale-safe) reads, 4 nodes in flight: a node already at <= d stops the
+            // walk (its own value is being propagated past it); a stale read that misses a
+            // concurrent improvement only costs a redundant min.  The mins are reductions.
             for (uint32_t steps = 0; jend < vend;) {
-                if (__ldg(P.node_t + jend) >= P.omega) break;  // no valid out-edge departs at >= omega
-                if (P.stats) atomicAdd(P.cnt + 1, 1ull);
-                const uint32_t old = atomicMin(dn + jend, d);
-                if (old <= d) break;
-                jend++;
-                if (++steps == WAIT_INLINE) { more = jend < vend; break; }
+                uint32_t tt[4], dd[4];
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    const uint32_t jj = jend + k;
+                    tt[k] = jj < vend ? __ldg(P.node_t + jj) : P.omega;
+                    dd[k] = jj < vend ? __ldcg(dn + jj) : 0u;
+                }
+                bool stop = false;
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    if (stop) continue;
+                    // no valid out-edge departs at >= omega; a node at <= d ends the walk
+                    if (tt[k] >= P.omega || dd[k] <= d || steps == WAIT_INLINE) { stop = true; continue; }
+                    if (P.stats) atomicAdd(P.cnt + 1, 1ull);
+                    atomicMin(dn + jend, d);
+                    jend++;
+                    steps++;
+                }
+                if (stop) break;
+            }
+            // the inline budget ran out with nodes left: the rest goes to k_spfp_wait
+            if (jend - (j + 1) == WAIT_INLINE && jend < vend) {
+                const uint32_t tt = __ldg(P.node_t + jend), dd = __ldcg(dn + jend);
+                more = tt < P.omega && dd > d;
             }
             if (more) {
                 // the rest of the walk as WAIT_SEG-node segments, walked by different warps in
@@ -288,8 +310,8 @@ __global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
             bool stop = true, improved = false;
             if (jj < vend && __ldg(P.node_t + jj) < P.omega) {
                 if (P.stats) atomicAdd(P.cnt + 1, 1ull);
-                const uint32_t old = atomicMin(dn + jj, d);
-                improved = old > d;
+                improved = __ldcg(dn + jj) > d;  // plain read: stale-safe (see the inline walk)
+                if (improved) atomicMin(dn + jj, d);
                 stop = !improved;
             }
             const uint32_t sm = __ballot_sync(0xffffffffu, stop);
