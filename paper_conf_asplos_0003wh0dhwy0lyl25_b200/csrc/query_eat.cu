@@ -355,6 +355,13 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+#if TG_DEFER
+    // deferral only in bulk rounds: the previous round consumed more than 1/8 of all units
+    // (in the tail it would only add rounds)
+    const bool bulk = P.defer && P.round >= TG_DEFER_FROM &&
+                      (uint64_t)*(volatile uint32_t *)&P.ctl->cnt[(P.round - 1) & (TG_RING - 1)][3] * 8 >
+                          (uint64_t)(P.ub1 - P.ub0);
+#endif
     for (uint32_t ub = P.ub0 + gw * 32; ub < NU; ub += nw * 32) {
         const uint32_t ui = ub + lane;
         uint32_t word = (ui < NU) ? R.fin[ui] : 0u;
@@ -365,7 +372,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         // experiment: a unit with few new queries in a bulk round waits one round (its
         // word moves to the next frontier) so that more of its group's queries share one
         // scan of its edges; a unit is deferred at most once in a row
-        if (word && P.round >= TG_DEFER_FROM && P.defer) {
+        if (word && bulk) {
             const uint32_t bit = 1u << (ui & 31);
             uint32_t *dw = P.defer + (ui >> 5);
             if (__popc(word) < TG_DEFER) {
