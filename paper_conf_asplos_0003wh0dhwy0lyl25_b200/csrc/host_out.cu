@@ -44,6 +44,25 @@ tg_status tg_sink_flush(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *h
     return TG_OK;
 }
 
+// as tg_sink_flush, with the staging buffer's row q going to the caller's row rows[q]
+tg_status tg_sink_flush_rows(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *host_pred, const uint32_t *rows,
+                             uint32_t nrows, uint64_t n, cudaStream_t s) {
+    if (!host_out && !host_pred) return TG_OK;
+    const int i = (int)(b & 1);
+    TG_TRY_CUDA(cudaEventRecord(g->ev_x[i], s));
+    TG_TRY_CUDA(cudaStreamWaitEvent(g->cstream, g->ev_x[i], 0));
+    for (uint32_t q = 0; q < nrows; q++) {
+        if (host_out)
+            TG_TRY_CUDA(cudaMemcpyAsync(host_out + (size_t)rows[q] * n, g->qs.out_stage[i] + (size_t)q * n, n * 4,
+                                        cudaMemcpyDeviceToHost, g->cstream));
+        if (host_pred)
+            TG_TRY_CUDA(cudaMemcpyAsync(host_pred + (size_t)rows[q] * n, g->qs.pred_stage[i] + (size_t)q * n, n * 4,
+                                        cudaMemcpyDeviceToHost, g->cstream));
+    }
+    TG_TRY_CUDA(cudaEventRecord(g->ev_c[i], g->cstream));
+    return TG_OK;
+}
+
 tg_status tg_sink_end(tg_graph *g) {
     if (g->cstream) TG_TRY_CUDA(cudaStreamSynchronize(g->cstream));
     return TG_OK;

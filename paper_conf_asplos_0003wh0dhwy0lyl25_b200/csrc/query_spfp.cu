@@ -45,6 +45,7 @@ constexpr uint32_t WAIT_SEG = TG_WAIT_SEG;  // nodes per queued wait segment (on
 
 struct SpP {
     const uint32_t *vnode_off, *node_t, *node_u, *node_eoff, *occ_slot, *occ_node;
+    const uint4 *occ_spr;
     const int4 *slots;
     const uint32_t *slot_w, *slot_tn;
     const uint2 *lc;
@@ -145,10 +146,31 @@ __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s,
 
 template <int MODE>
 __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_t q, uint32_t p) {
-    const uint32_t s = __ldg(P.occ_slot + p);
+    // occurrence-ordered record {v, arrival | walked flag, tail node, w}: an edge that is
+    // not on a walked chain needs nothing else (no slot, weight or tail-node gathers)
+    const uint4 rc = __ldg(P.occ_spr + p);
     const uint32_t j = __ldg(P.occ_node + p);
     const uint32_t cur = __ldcg(P.dnode + (size_t)q * P.nnodes + j);
     if (cur == TG_NONE) return;
+    if (!(rc.y >> 31)) {
+        const uint32_t arr = rc.y;
+        if (arr > P.omega) return;
+        if (P.stats) atomicAdd(P.cnt + 0, 1ull);
+        uint32_t cand, val;
+        if (MODE == 1) { cand = cur; val = arr - (0xFFFFFFFEu - cur); }
+        else if (MODE == 2) { cand = cur; val = cur; }
+        else { cand = cur + rc.w; val = cand; }
+        uint32_t *vo = P.vout + (size_t)q * P.n;
+        if (vo[rc.x] > val) atomicMin(vo + rc.x, val);
+        const uint32_t tn = rc.z;
+        if (tn == TG_NONE) return;
+        uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
+        if (__ldcg(dn + tn) <= cand) return;
+        atomicMin(dn + tn, cand);
+        push_node(P, R, q, tn);
+        return;
+    }
+    const uint32_t s = __ldg(P.occ_slot + p);
     const int4 sl = tg_ld_slot(P.slots + s);
     if ((uint32_t)sl.y > P.omega) return;
     uint32_t s_end = s + 1;
@@ -373,6 +395,17 @@ __global__ void k_spfp_init(SpP P, const uint32_t *srcs, uint32_t S) {
 }
 
 // SP / FP: the per-vertex minimum (source 0); LDS: latest start = ~key (source omega)
+// the node-state engines' occurrence records (built once per direction, on first use)
+__global__ void k_spfp_records(const uint2 *__restrict__ occ_rec, const uint32_t *__restrict__ occ_slot,
+                               const uint32_t *__restrict__ slot_tn, const uint32_t *__restrict__ slot_w, uint64_t m,
+                               uint4 *__restrict__ out) {
+    for (uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; p < m; p += (uint64_t)gridDim.x * blockDim.x) {
+        const uint2 r = occ_rec[p];
+        const uint32_t s = occ_slot[p];
+        out[p] = make_uint4(r.x, r.y, slot_tn[s], slot_w[s]);
+    }
+}
+
 __global__ void k_spfp_extract(const uint32_t *__restrict__ vout, uint32_t n, const uint32_t *__restrict__ srcs,
                                uint32_t *__restrict__ out, const uint32_t *__restrict__ perm, int lds,
                                uint32_t omega) {
@@ -392,14 +425,19 @@ template <int MODE>
 static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t omega, cudaStream_t s,
                              uint32_t *rounds_out) {
     QueryScratch &Q = g->qs;
-    const ChainGraph &c = g->fwd;
+    ChainGraph &c = g->fwd;
     const uint64_t n = g->n, nn = c.nnodes;
+    if (!c.occ_spr && g->m) {
+        TG_TRY(c.arena.alloc((void **)&c.occ_spr, g->m * 16));
+        TG_LAUNCH(k_spfp_records, (unsigned)std::min<uint64_t>((g->m + 255) / 256, 148ull * 32), 256, 0, s, c.occ_rec,
+                  c.occ_slot, c.slot_tn, c.slot_w, g->m, c.occ_spr);
+    }
     TG_TRY_CUDA(cudaMemsetAsync(Q.vout, 0xFF, Sb * n * 4, s));
     if (nn) TG_TRY_CUDA(cudaMemsetAsync(Q.dnode, 0xFF, Sb * nn * 4, s));
     if (g->m == 0 || alpha >= omega) { *rounds_out = 0; return TG_OK; }
     SpP P{};
     P.vnode_off = c.vnode_off; P.node_t = c.node_t; P.node_u = c.node_u; P.node_eoff = c.node_eoff;
-    P.occ_slot = c.occ_slot; P.occ_node = c.occ_node; P.slots = c.slots; P.slot_w = c.slot_w; P.slot_tn = c.slot_tn;
+    P.occ_slot = c.occ_slot; P.occ_node = c.occ_node; P.occ_spr = c.occ_spr; P.slots = c.slots; P.slot_w = c.slot_w; P.slot_tn = c.slot_tn;
     P.lc = c.lc; P.sc = c.sc; P.sc_sumw = c.sc_sumw;
     P.dnode = Q.dnode; P.vout = Q.vout; P.mark = Q.mark; P.n = g->n; P.nnodes = nn;
     P.alpha = alpha; P.omega = omega; P.use_sc = (int)g->opt_shortcuts;

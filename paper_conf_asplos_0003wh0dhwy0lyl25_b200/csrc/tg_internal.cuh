@@ -86,6 +86,7 @@ struct ChainGraph {
     uint32_t *occ_node = nullptr;  // sorted-edge position -> departure node (SP/FP entry state)
     uint2 *occ_rec = nullptr;      // sorted-edge position -> {head v, arrival | 1 << 31 if on a walked chain}
     uint4 *occ_rch = nullptr;      // bit-lane reach (built on first use): {v, arrival | walked flag, tail node, tail tau}
+    uint4 *occ_spr = nullptr;      // SP/FP/LDS (built on first use): {v, arrival | walked flag, tail node, w}
     int4 *slots = nullptr;
     uint32_t *slot_w = nullptr, *slot_tn = nullptr;
     uint2 *lc = nullptr;
@@ -144,6 +145,7 @@ struct QueryScratch {
     uint32_t *h_ctr = nullptr; // pinned host mirror
     uint32_t *srcs = nullptr;  // [S] sources of the sub-batch (caller's vertex ids)
     uint32_t *srcs_int = nullptr;  // [S] the same in the engine's internal vertex order
+    uint32_t *rows = nullptr;      // [S] the caller's output row of each query of the sub-batch
     unsigned long long *relax_cnt = nullptr;  // [S] + distinct-slot count
     uint32_t *touched = nullptr;              // stats: slots relaxed by any query of the sub-batch
     uint32_t *out_stage[2] = {nullptr, nullptr}, *pred_stage[2] = {nullptr, nullptr};  // [S][n] x 2 for host outputs
@@ -238,6 +240,7 @@ struct tg_graph {
     int opt_mirror = 1;
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
+    int64_t opt_order_sources = 1;  // schedule a call's sources by first departure time (query_eat.cu)
     int64_t opt_reach_bits = 0;  // 1 = TG_REACH without pred on the bit-lane engine (query_reach.cu)
     int64_t opt_dynamic = 0;   // 1 = keep each direction's sorted edge order for tg_graph_insert_edges
     int64_t opt_walk_min = 6;  // chains with fewer edges are not walked (RemoveChain threshold, build time)
@@ -300,6 +303,8 @@ tg_status tg_sink_begin(tg_graph *g, bool out_host, bool pred_host);
 tg_status tg_sink_target(tg_graph *g, uint32_t b, bool out_host, bool pred_host, uint32_t **o, uint32_t **pr,
                          cudaStream_t s);
 tg_status tg_sink_flush(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *host_pred, size_t bytes, cudaStream_t s);
+tg_status tg_sink_flush_rows(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *host_pred, const uint32_t *rows,
+                             uint32_t nrows, uint64_t n, cudaStream_t s);
 tg_status tg_sink_end(tg_graph *g);
 void tg_sink_destroy(tg_graph *g);
 

@@ -736,3 +736,35 @@ def test_streamed_c2_small_and_host_out(tg):
     for r, x in enumerate(srcs[:8]):
         np.testing.assert_array_equal(tg.as_u32(hout[r]), oracle.eat(og, x, 0, 10**9)[0])
     g.close()
+
+
+# --------------------------------------------------------------------------- sub-batch scheduling
+@pytest.mark.parametrize("seed", range(3))
+def test_source_scheduling_rows(tg, seed):
+    """Sources of a call are scheduled into sub-batches by first departure time; every
+    query's values, preds and first-touch W must land in the caller's row (device and host
+    outputs, ragged last sub-batch, sub-batch sizes 64 and 20, duplicate sources)."""
+    import torch
+    rng = np.random.default_rng(seed + 8800)
+    n, m = 500, 9000
+    u = rng.integers(0, n, m).astype(np.uint32); v = rng.integers(0, n, m).astype(np.uint32)
+    t = rng.integers(0, 400, m).astype(np.uint32); lam = rng.integers(1, 9, m).astype(np.uint32)
+    og = oracle.Graph(n, u, v, t, lam)
+    srcs = [int(x) for x in rng.choice(n, 150, replace=True)]
+    for sb in (0, 20):
+        g = _gpu_graph(tg, n, u, v, t, lam, stats=1, sub_batch=sb)
+        for win in [(0, 10**6), (50, 300)]:
+            for p in ("eat", "ld", "reach"):
+                _check_rows(tg, g, og, p, srcs, win, stats=(p == "eat"))
+                _check_values(tg, g, og, p, srcs, win)
+            hout = torch.empty((len(srcs), n), dtype=torch.int32)
+            hpred = torch.empty((len(srcs), n), dtype=torch.int32)
+            tg.tg_query(g.h, tg.TG_EAT, srcs, win, hout, hpred)
+            for r, x in enumerate(srcs):
+                A, P, _ = oracle.eat(og, x, *win)
+                np.testing.assert_array_equal(tg.as_u32(hout[r]), A)
+                np.testing.assert_array_equal(tg.as_u32(hpred[r]), P)
+            tg.tg_query(g.h, tg.TG_LD, srcs, win, hout)
+            for r, x in enumerate(srcs):
+                np.testing.assert_array_equal(tg.as_u32(hout[r]), oracle.ld(og, x, *win)[0])
+        g.close()
