@@ -57,7 +57,7 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #define TG_MLP 4                        // state reads in flight per lane in the pair loop
 #endif
 #ifndef TG_DEFER
-#define TG_DEFER 8                      // units with fewer new queries wait one round (0 = off; C4 -6 %)
+#define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
 #endif
 #ifndef TG_DEFER_FROM
 #define TG_DEFER_FROM 3                 // first round in which units may be deferred
