@@ -1075,6 +1075,25 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
     return TG_OK;
 }
 
+// The order in which a call's k sources are cut into sub-batches: by first departure time
+// >= alpha in direction cgr when `on` (stable), else the caller's order.
+tg_status tg_schedule_sources(tg_graph *g, const ChainGraph &cgr, const uint32_t *sources, uint32_t k, uint32_t alpha,
+                              bool on, std::vector<uint32_t> &order, cudaStream_t s) {
+    order.resize(k);
+    for (uint32_t i = 0; i < k; i++) order[i] = i;
+    if (!on) return TG_OK;
+    uint32_t *tmp = nullptr;
+    TG_TRY_CUDA(tg_malloc_async((void **)&tmp, (uint64_t)k * 12, s));
+    TG_TRY(tg_load_sources_to(g, sources, k, tmp, tmp + k, s));
+    TG_LAUNCH(k_source_keys, (k + 255) / 256, 256, 0, s, cgr.vnode_off, cgr.node_t, tmp + k, k, alpha, tmp + 2 * k);
+    std::vector<uint32_t> key(k);
+    TG_TRY_CUDA(cudaMemcpyAsync(key.data(), tmp + 2 * k, (uint64_t)k * 4, cudaMemcpyDeviceToHost, s));
+    TG_TRY_CUDA(cudaFreeAsync(tmp, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return key[a] < key[b]; });
+    return TG_OK;
+}
+
 tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
                             uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s) {
     const bool ld = (p == TG_LD);
@@ -1106,20 +1125,9 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     // >= alpha, so the queries sharing a sub-batch (and a 32-query frontier unit) start -- and
     // reach the graph's vertices -- at similar rounds; their activations share unit scans
     // (C4 1024-source job 3.17 -> 2.36 s).  Each query's row is written to the caller's row.
-    std::vector<uint32_t> order(k), srcs_sched(k);
-    for (uint32_t i = 0; i < k; i++) order[i] = i;
+    std::vector<uint32_t> order, srcs_sched(k);
     const bool sched = g->opt_order_sources && k > 32 && any_work && g->m > 0 && (!pred || out_dev == pred_dev);
-    if (sched) {
-        uint32_t *tmp = nullptr;
-        TG_TRY_CUDA(tg_malloc_async((void **)&tmp, (uint64_t)k * 12, s));
-        TG_TRY(tg_load_sources_to(g, sources, k, tmp, tmp + k, s));
-        TG_LAUNCH(k_source_keys, (k + 255) / 256, 256, 0, s, cgr.vnode_off, cgr.node_t, tmp + k, k, alpha, tmp + 2 * k);
-        std::vector<uint32_t> key(k);
-        TG_TRY_CUDA(cudaMemcpyAsync(key.data(), tmp + 2 * k, (uint64_t)k * 4, cudaMemcpyDeviceToHost, s));
-        TG_TRY_CUDA(cudaFreeAsync(tmp, s));
-        TG_TRY_CUDA(cudaStreamSynchronize(s));
-        std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return key[a] < key[b]; });
-    }
+    TG_TRY(tg_schedule_sources(g, cgr, sources, k, alpha, sched, order, s));
     for (uint32_t i = 0; i < k; i++) srcs_sched[i] = sources[order[i]];
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);

@@ -408,11 +408,12 @@ __global__ void k_spfp_records(const uint2 *__restrict__ occ_rec, const uint32_t
 
 __global__ void k_spfp_extract(const uint32_t *__restrict__ vout, uint32_t n, const uint32_t *__restrict__ srcs,
                                uint32_t *__restrict__ out, const uint32_t *__restrict__ perm, int lds,
-                               uint32_t omega) {
+                               uint32_t omega, const uint32_t *__restrict__ rows) {
     const uint32_t q = blockIdx.y;
     const uint32_t src = srcs[q];  // caller's vertex ids
+    const size_t row = rows ? rows[q] : q;  // the caller's row of this query
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-        const size_t i = (size_t)q * n + v;
+        const size_t i = row * n + v;
         const uint32_t x = vout[(size_t)q * n + (perm ? perm[v] : v)];
         if (lds) out[i] = (v == src) ? omega : (x == TG_NONE ? TG_NONE : 0xFFFFFFFEu - x);
         else out[i] = (v == src) ? 0u : x;
@@ -505,9 +506,21 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
     TG_TRY(tg_sink_begin(g, !out_dev, false));
     g->last = tg_query_stats{};
     const uint64_t launches0 = g_tg_launches;
+    // sub-batch scheduling by first departure time (query_eat.cu tg_schedule_sources)
+    std::vector<uint32_t> order, srcs_sched(k);
+    TG_TRY(tg_schedule_sources(g, g->fwd, sources, k, w.t_alpha,
+                               g->opt_order_sources && k > S && g->m > 0 && w.t_alpha < w.t_omega, order, s));
+    for (uint32_t i = 0; i < k; i++) srcs_sched[i] = sources[order[i]];
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
-        TG_TRY(tg_load_sources(g, sources + b0, Sb, s));
+        TG_TRY(tg_load_sources(g, srcs_sched.data() + b0, Sb, s));
+        bool consecutive = true;
+        for (uint32_t q = 0; q < Sb; q++) consecutive = consecutive && order[b0 + q] == b0 + q;
+        const uint32_t *rows = nullptr;
+        if (!consecutive && out_dev) {
+            TG_TRY_CUDA(cudaMemcpyAsync(Q.rows, order.data() + b0, Sb * 4, cudaMemcpyHostToDevice, s));
+            rows = Q.rows;
+        }
         uint32_t rounds = 0;
         if (g->opt_stats) TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, 16, s));
         if (mode == 1) TG_TRY((spfp_rounds<1>(g, Sb, w.t_alpha, w.t_omega, s, &rounds)));
@@ -523,12 +536,15 @@ tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32
         }
         g->last.sub_batches++;
         const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
-        uint32_t *o = out_dev ? out + (size_t)b0 * n : nullptr, *no_pred = nullptr;
+        uint32_t *o = out_dev ? (rows ? out : out + (size_t)b0 * n) : nullptr, *no_pred = nullptr;
         TG_TRY(tg_sink_target(g, bi, !out_dev, false, &o, &no_pred, s));
         dim3 grid((unsigned)std::min<uint64_t>((n + 255) / 256, 1024), Sb);
         TG_LAUNCH(k_spfp_extract, grid, 256, 0, s, Q.vout, g->n, Q.srcs, o, g->relabeled ? g->perm : (const uint32_t *)nullptr,
-                  mode == 2 ? 1 : 0, w.t_omega);
-        TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n, nullptr, (size_t)Sb * n * 4, s));
+                  mode == 2 ? 1 : 0, w.t_omega, rows);
+        if (consecutive || out_dev)
+            TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n, nullptr, (size_t)Sb * n * 4, s));
+        else
+            TG_TRY(tg_sink_flush_rows(g, bi, out, nullptr, order.data() + b0, Sb, n, s));
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     TG_TRY(tg_sink_end(g));

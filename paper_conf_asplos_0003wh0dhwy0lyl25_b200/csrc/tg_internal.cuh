@@ -306,6 +306,8 @@ tg_status tg_sink_flush(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *h
 tg_status tg_sink_flush_rows(tg_graph *g, uint32_t b, uint32_t *host_out, uint32_t *host_pred, const uint32_t *rows,
                              uint32_t nrows, uint64_t n, cudaStream_t s);
 tg_status tg_sink_end(tg_graph *g);
+tg_status tg_schedule_sources(tg_graph *g, const ChainGraph &cgr, const uint32_t *sources, uint32_t k, uint32_t alpha,
+                              bool on, std::vector<uint32_t> &order, cudaStream_t s);
 void tg_sink_destroy(tg_graph *g);
 
 // ----------------------------------------------------------------------------- device helpers

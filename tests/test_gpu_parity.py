@@ -767,4 +767,13 @@ def test_source_scheduling_rows(tg, seed):
             tg.tg_query(g.h, tg.TG_LD, srcs, win, hout)
             for r, x in enumerate(srcs):
                 np.testing.assert_array_equal(tg.as_u32(hout[r]), oracle.ld(og, x, *win)[0])
+            # node-state engines (sub-batches <= 32): scheduled rows, device and host outputs
+            few = srcs[:70]
+            for p, fn in (("sp", oracle.sp), ("fp", oracle.fp), ("lds", oracle.lds)):
+                dout = tg.as_u32(g.query(p, few, win))
+                tg.tg_query(g.h, tg.PROBLEMS[p], few, win, hout[:len(few)])
+                for r, x in enumerate(few):
+                    exp = fn(og, x, *win)
+                    np.testing.assert_array_equal(dout[r], exp, err_msg=f"{p} row {r}")
+                    np.testing.assert_array_equal(tg.as_u32(hout[r]), exp, err_msg=f"{p} host row {r}")
         g.close()
