@@ -365,7 +365,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         // experiment: a unit with few new queries in a bulk round waits one round (its
         // word moves to the next frontier) so that more of its group's queries share one
         // scan of its edges; a unit is deferred at most once in a row
-        if (word && P.defer && P.round >= TG_DEFER_FROM) {
+        if (word && P.defer && P.S >= 64 && P.round >= TG_DEFER_FROM) {  // full sub-batches only
             const uint32_t bit = 1u << (ui & 31);
             uint32_t *dw = P.defer + (ui >> 5);
             if (__popc(word) < TG_DEFER) {
