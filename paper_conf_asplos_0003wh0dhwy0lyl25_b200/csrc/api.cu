@@ -128,6 +128,7 @@ tg_status DevArena::alloc(void **p, size_t bytes) {
     size_t got = bytes;
     void *q = cache_take(bytes, dev, &got);
     if (!q) {
+        if (slack_pct) bytes = round_bytes(bytes + bytes / 100 * slack_pct);
         got = bytes;
         cudaError_t e = cudaMalloc(&q, bytes);
         if (e != cudaSuccess) {

@@ -401,6 +401,7 @@ tg_status tg_build_direction(tg_graph *g, ChainGraph *cg, uint64_t m, const uint
     cg->m = m;
     bmark(s, nullptr);
     DevArena &A = cg->arena;
+    if (g->opt_dynamic) A.slack_pct = 10;  // insertions re-transform into slightly larger arrays
     TG_TRY(A.alloc((void **)&cg->vnode_off, ((size_t)n + 1) * 4));
     if (m == 0) {
         TG_TRY_CUDA(cudaMemsetAsync(cg->vnode_off, 0, ((size_t)n + 1) * 4, s));

@@ -151,6 +151,7 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
     const uint64_t m_old = g->m, m_new = g->m + k;
     // 1. the new edge arrays: the kept edges, then the batch (ids m_old .. m_new - 1)
     DevArena na;
+    na.slack_pct = 10;  // the next insertion's edge arrays come from the cache
     uint32_t *nu = nullptr, *nv = nullptr, *nt = nullptr, *nd = nullptr, *nw = nullptr;
     uint32_t **dst[5] = {&nu, &nv, &nt, &nd, &nw};
     const uint32_t *oldp[5] = {g->d_u, g->d_v, g->d_t, g->d_dur, g->d_w};

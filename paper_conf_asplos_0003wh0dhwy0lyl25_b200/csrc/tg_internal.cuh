@@ -60,6 +60,8 @@ struct DevArena {
     struct Blk { void *p; size_t bytes; };
     std::vector<Blk> blks;
     size_t total = 0;
+    uint32_t slack_pct = 0;  // fresh blocks get this much extra room (dynamic graphs: the next,
+                             // slightly larger, re-transformation reuses them from the cache)
     tg_status alloc(void **p, size_t bytes);
     void free_all();
 };
