@@ -50,6 +50,8 @@ struct SpuP {
     uint4 *segq;       // {record, first node, end node, lane mask}
     uint32_t *segd;    // [record * 32 + lane] carried value
     uint64_t segcap;
+    uint2 *walkq;      // nodes improved by wait walks in this round: {node, lanes}
+    uint64_t walkcap;
     RoundCtl *ctl;
     uint32_t round, S;
     uint64_t nnodes;
@@ -135,25 +137,46 @@ __device__ __forceinline__ void relax_node(const SpuP &P, uint32_t j, uint32_t l
     for (uint32_t p = p0; p < p1; p++) relax_occ<MODE>(P, p, lanes, cur, fout);
 }
 
+// A node the wait walk improved: its out-edges are relaxed in the same round by
+// k_spu_expand (queue of {node, lanes}); a full queue falls back to the next frontier.
+__device__ __forceinline__ void walked_node(const SpuP &P, uint32_t j, uint32_t lanes, uint32_t *fout) {
+    const int lane = threadIdx.x & 31;
+    if (lane != 0) return;
+    const uint32_t k = atomicAdd(&P.ctl->cnt[P.round & (TG_RING - 1)][2], 1u);
+    if (k < P.walkcap) P.walkq[k] = make_uint2(j, lanes);
+    else atomicOr(fout + j, lanes);
+}
+
 // Wait walk over nodes [j, jend) of one vertex with per-lane carried values d: a lane stops
-// at its first node that is already as good; improved nodes are relaxed on the way.
-// Returns the node index the walk stopped at (jend if it reached the end).
-template <int MODE>
+// at its first node that is already as good (that node's value is being propagated past
+// it); every node it improves is queued for k_spu_expand.  Four node rows are read ahead
+// (independent loads; only the stop rule is sequential).  Returns the node the walk stopped
+// at (jend if it reached the end); `lanes` keeps the lanes still walking.
 __device__ __forceinline__ uint32_t wait_walk(const SpuP &P, uint32_t j, uint32_t jend, uint32_t &lanes, uint32_t d,
                                               uint32_t budget, uint32_t *fout) {
     const int lane = threadIdx.x & 31;
-    for (uint32_t steps = 0; j < jend && lanes; j++, steps++) {
-        if (steps == budget) return j;
-        if (__ldg(P.node_t + j) >= P.omega) return jend;  // nothing valid departs at >= omega
-        bool imp = false;
-        if ((lanes >> lane) & 1u) {
-            uint32_t *x = P.dn + (size_t)j * P.S + lane;
-            imp = __ldcg(x) > d;
-            if (imp) atomicMin(x, d);
+    uint32_t steps = 0;
+    while (j < jend && lanes) {
+        uint32_t tt[4], x[4];
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint32_t jj = j + k;
+            tt[k] = jj < jend ? __ldg(P.node_t + jj) : P.omega;
+            x[k] = (jj < jend && ((lanes >> lane) & 1u)) ? __ldcg(P.dn + (size_t)jj * P.S + lane) : 0u;
         }
-        if (P.stats && lane == 0) atomicAdd(P.cnt + 1, (unsigned long long)__popc(lanes));
-        lanes = __ballot_sync(0xffffffffu, imp);
-        if (lanes) relax_node<MODE>(P, j, lanes, d, fout);
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            if (!lanes || j >= jend) break;
+            if (steps == budget) return j;
+            if (tt[k] >= P.omega) return jend;  // nothing valid departs at >= omega
+            const bool imp = ((lanes >> lane) & 1u) && x[k] > d;
+            if (imp) atomicMin(P.dn + (size_t)j * P.S + lane, d);
+            if (P.stats && lane == 0) atomicAdd(P.cnt + 1, (unsigned long long)__popc(lanes));
+            lanes = __ballot_sync(0xffffffffu, imp);
+            if (lanes) walked_node(P, j, lanes, fout);
+            j++;
+            steps++;
+        }
     }
     return jend;
 }
@@ -186,7 +209,7 @@ __global__ void __launch_bounds__(UT) k_spu_activate(SpuP P) {
             relax_node<MODE>(P, j, lanes, d, fout);
             const uint32_t vend = __ldg(P.vnode_off + __ldg(P.node_u + j) + 1);
             uint32_t walking = lanes;  // lanes still carrying their value (the walk narrows it)
-            const uint32_t stop = wait_walk<MODE>(P, j + 1, vend, walking, d, WALK_INLINE, fout);
+            const uint32_t stop = wait_walk(P, j + 1, vend, walking, d, WALK_INLINE, fout);
             if (stop < vend && walking) {
                 // the rest of the vertex's nodes as segments walked by other warps
                 const uint32_t nseg = (vend - stop + WALK_SEG - 1) / WALK_SEG;
@@ -202,7 +225,7 @@ __global__ void __launch_bounds__(UT) k_spu_activate(SpuP P) {
                 } else {
                     // queue full: reserved entries empty, the walk finishes here
                     for (uint32_t c = lane; c < nseg && k + c < P.segcap; c += 32) P.segq[k + c] = make_uint4(0, 0, 0, 0);
-                    wait_walk<MODE>(P, stop, vend, walking, d, 0xFFFFFFFFu, fout);
+                    wait_walk(P, stop, vend, walking, d, 0xFFFFFFFFu, fout);
                 }
             }
         }
@@ -210,7 +233,6 @@ __global__ void __launch_bounds__(UT) k_spu_activate(SpuP P) {
     if (lane == 0 && my_units) atomicAdd(&P.ctl->cnt[r & (TG_RING - 1)][3], my_units);
 }
 
-template <int MODE>
 __global__ void __launch_bounds__(UT) k_spu_segments(SpuP P) {
     const uint32_t r = P.round;
     uint32_t *fout = P.fb[(r + 1) & 1];
@@ -223,7 +245,23 @@ __global__ void __launch_bounds__(UT) k_spu_segments(SpuP P) {
         if (c.y >= c.z) continue;
         const uint32_t d = P.segd[(size_t)c.x * 32 + lane];
         uint32_t walking = c.w;
-        wait_walk<MODE>(P, c.y, c.z, walking, d, 0xFFFFFFFFu, fout);
+        wait_walk(P, c.y, c.z, walking, d, 0xFFFFFFFFu, fout);
+    }
+}
+
+// Out-edges of the nodes the wait walks improved in this round, with their current values.
+template <int MODE>
+__global__ void __launch_bounds__(UT) k_spu_expand(SpuP P) {
+    const uint32_t r = P.round;
+    uint32_t *fout = P.fb[(r + 1) & 1];
+    const uint32_t B = (uint32_t)min((uint64_t)*(volatile uint32_t *)&P.ctl->cnt[r & (TG_RING - 1)][2], P.walkcap);
+    const int lane = threadIdx.x & 31;
+    const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t it = gw; it < B; it += nw) {
+        const uint2 c = P.walkq[it];
+        const uint32_t d = ((c.y >> lane) & 1u) ? __ldcg(P.dn + (size_t)c.x * P.S + lane) : TG_NONE;
+        relax_node<MODE>(P, c.x, c.y, d, fout);
     }
 }
 
@@ -251,13 +289,14 @@ __global__ void k_spu_ctl(RoundCtl *ctl) {
 }
 
 // rows of the caller: out[row(q)][v] from vout[v][q]; LDS un-keys, sources get 0 / omega
-__global__ void k_spu_extract(const uint32_t *__restrict__ vout, uint32_t n, uint32_t S, const uint32_t *__restrict__ srcs,
-                              uint32_t *__restrict__ out, const uint32_t *__restrict__ perm, int lds, uint32_t omega,
+__global__ void k_spu_extract(const uint32_t *__restrict__ vout, uint32_t n, uint32_t S, uint32_t stride,
+                              const uint32_t *__restrict__ srcs, uint32_t *__restrict__ out,
+                              const uint32_t *__restrict__ perm, int lds, uint32_t omega,
                               const uint32_t *__restrict__ rows) {
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
         const uint32_t vi = perm ? perm[v] : v;
         for (uint32_t q = 0; q < S; q++) {
-            const uint32_t x = vout[(size_t)vi * S + q];
+            const uint32_t x = vout[(size_t)vi * stride + q];
             const size_t row = rows ? rows[q] : q;
             uint32_t y;
             if (lds) y = (v == srcs[q]) ? omega : (x == TG_NONE ? TG_NONE : 0xFFFFFFFEu - x);
@@ -307,6 +346,8 @@ static tg_status spu_scratch(tg_graph *g, uint32_t S) {
     U.segcap = std::min<uint64_t>(nn / WALK_SEG + 65536, 1ull << 24);
     TG_TRY(A.alloc((void **)&U.segq, U.segcap * 16));
     TG_TRY(A.alloc((void **)&U.segd, U.segcap * 32 * 4));
+    U.walkcap = std::min<uint64_t>(nn + 65536, 1ull << 26);
+    TG_TRY(A.alloc((void **)&U.walkq, U.walkcap * 8));
     TG_TRY(A.alloc((void **)&U.ctl, sizeof(RoundCtl)));
     TG_TRY(A.alloc((void **)&U.cnt, 64));
     TG_TRY(A.alloc((void **)&U.srcs, 32 * 4));
@@ -336,6 +377,7 @@ static tg_status spu_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t o
     P.lc = c.lc; P.sc = c.sc; P.sc_sumw = c.sc_sumw;
     P.dn = U.dn; P.vout = U.vout; P.fb[0] = U.fb[0]; P.fb[1] = U.fb[1];
     P.segq = U.segq; P.segd = U.segd; P.segcap = U.segcap; P.ctl = U.ctl;
+    P.walkq = U.walkq; P.walkcap = U.walkcap;
     P.S = U.S; P.nnodes = nn; P.alpha = alpha; P.omega = omega;
     P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats; P.cnt = U.cnt;
     TG_LAUNCH(k_spu_ctl, 1, 1, 0, s, U.ctl);
@@ -350,7 +392,8 @@ static tg_status spu_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t o
         for (int k = 0; k < group; k++, r++) {
             P.round = r;
             TG_LAUNCH_RELAX(k_spu_activate<MODE>, grid, UT, 0, s, P);
-            TG_LAUNCH_RELAX(k_spu_segments<MODE>, grid, UT, 0, s, P);
+            TG_LAUNCH_RELAX(k_spu_segments, grid, UT, 0, s, P);
+            TG_LAUNCH_RELAX(k_spu_expand<MODE>, grid, UT, 0, s, P);
         }
         TG_TRY_CUDA(cudaMemcpyAsync(U.h_ctr, U.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
         TG_TRY_CUDA(cudaStreamSynchronize(s));
@@ -409,7 +452,7 @@ tg_status tg_run_spu(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_
         }
         // device outputs: rows straight to the caller's rows; host: staging rows 0.., then per row
         const unsigned xg = (unsigned)std::min<uint64_t>((n + 255) / 256, 148ull * 8);
-        TG_LAUNCH(k_spu_extract, xg, 256, 0, s, U.vout, g->n, Sb, U.srcs, out_dev ? out : U.stage,
+        TG_LAUNCH(k_spu_extract, xg, 256, 0, s, U.vout, g->n, Sb, U.S, U.srcs, out_dev ? out : U.stage,
                   g->relabeled ? g->perm : (const uint32_t *)nullptr, mode == 2 ? 1 : 0, w.t_omega,
                   out_dev ? (const uint32_t *)U.rows : (const uint32_t *)nullptr);
         if (!out_dev)

@@ -209,6 +209,8 @@ struct UnitScratch {
     uint4 *segq = nullptr;
     uint32_t *segd = nullptr;
     uint64_t segcap = 0;
+    uint2 *walkq = nullptr;
+    uint64_t walkcap = 0;
     struct RoundCtl *ctl = nullptr;
     unsigned long long *cnt = nullptr;
     uint32_t *srcs = nullptr, *srcs_int = nullptr, *rows = nullptr, *stage = nullptr;
