@@ -168,8 +168,6 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
                             uint32_t *out, uint32_t *pred, bool out_dev, bool pred_dev, cudaStream_t s);
 tg_status tg_run_reach_bits(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                             bool out_dev, cudaStream_t s);
-tg_status tg_run_spu(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
-                     bool out_dev, cudaStream_t s);
 tg_status tg_run_spfp(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                       bool out_dev, cudaStream_t s);
 tg_status tg_run_eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t k, tg_window w,
@@ -204,8 +202,7 @@ struct DeviceGuard {
 }  // namespace
 
 uint64_t tg_graph_bytes(const tg_graph *g) {
-    uint64_t b = g->arena.total + g->qs.arena.total + g->rs.arena.total + g->us.arena.total + g->fwd.arena.total +
-                 g->mir.arena.total;
+    uint64_t b = g->arena.total + g->qs.arena.total + g->rs.arena.total + g->fwd.arena.total + g->mir.arena.total;
     for (int p = 0; p < TG_MAXP; p++) b += g->pf[p].arena.total + g->pm[p].arena.total;
     if (g->stream) b += g->stream->slot_arena.total;
     return b;
@@ -420,7 +417,6 @@ tg_status tg_query(tg_graph *g, tg_problem p, const uint32_t *sources, uint32_t 
     if (p == TG_EAT || p == TG_LD || p == TG_REACH) {
         return tg_run_eat_family(g, p, sources, n_sources, w, out, pred, out_dev, pred_dev, s);
     }
-    if (g->opt_spfp_engine == 0) return tg_run_spu(g, p, sources, n_sources, w, out, out_dev, s);
     return tg_run_spfp(g, p, sources, n_sources, w, out, out_dev, s);
 }
 
@@ -434,8 +430,6 @@ void tg_graph_destroy(tg_graph *g) {
     tg_pinned_put(g->qs.h_ctr);
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);
-    g->us.arena.free_all();
-    tg_pinned_put(g->us.h_ctr);
     g->fwd.arena.free_all();
     g->mir.arena.free_all();
     for (int p = 0; p < TG_MAXP; p++) { g->pf[p].arena.free_all(); g->pm[p].arena.free_all(); }
@@ -587,7 +581,6 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     else if (k == "packed_state") g->opt_packed_state = value ? 1 : 0;
     else if (k == "reach_bits") g->opt_reach_bits = value ? 1 : 0;
     else if (k == "order_sources") g->opt_order_sources = value ? 1 : 0;
-    else if (k == "spfp_engine") g->opt_spfp_engine = value ? 1 : 0;
     else if (k == "dynamic") {
         if (g->built) { tg_set_error("set dynamic before tg_build_chains"); return TG_ERR_STATE; }
         g->opt_dynamic = value ? 1 : 0;

@@ -191,9 +191,6 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);
     g->rs = ReachScratch{};
-    g->us.arena.free_all();
-    tg_pinned_put(g->us.h_ctr);
-    g->us = UnitScratch{};
     dmark("scratch");
     if (!g->built) return TG_OK;
     // 2./3. incremental re-transformation of each built direction

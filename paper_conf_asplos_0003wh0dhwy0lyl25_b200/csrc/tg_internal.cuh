@@ -201,24 +201,6 @@ struct ReachScratch {
     DevArena arena;
 };
 
-// Unit engine for SP / FP / LDS (query_spu.cu): node state interleaved over <= 32 queries.
-struct UnitScratch {
-    uint32_t S = 0;
-    uint64_t nn = 0, n = 0;
-    uint32_t *dn = nullptr, *vout = nullptr, *fb[2] = {nullptr, nullptr};
-    uint4 *segq = nullptr;
-    uint32_t *segd = nullptr;
-    uint64_t segcap = 0;
-    uint2 *walkq = nullptr;
-    uint64_t walkcap = 0;
-    struct RoundCtl *ctl = nullptr;
-    unsigned long long *cnt = nullptr;
-    uint32_t *srcs = nullptr, *srcs_int = nullptr, *rows = nullptr, *stage = nullptr;
-    uint32_t *h_ctr = nullptr;
-    uint64_t bytes = 0;
-    DevArena arena;
-};
-
 #define TG_MAXP 16  // logical vertex-range partitions per process (tests / one rank's share)
 
 struct tg_comm;  // comm.cu: NCCL communicator (loaded with dlopen)
@@ -250,8 +232,6 @@ struct tg_graph {
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
     ReachScratch rs;
-    UnitScratch us;
-    int64_t opt_spfp_engine = 0;  // 0 = unit engine (query_spu.cu), 1 = per-(query, node) queue engine
     StreamGraph *stream = nullptr;  // out-of-memory graph (tg_graph_create_streamed)
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
     // options
