@@ -777,3 +777,22 @@ def test_source_scheduling_rows(tg, seed):
                     np.testing.assert_array_equal(dout[r], exp, err_msg=f"{p} row {r}")
                     np.testing.assert_array_equal(tg.as_u32(hout[r]), exp, err_msg=f"{p} host row {r}")
         g.close()
+
+
+def test_streamed_edge_cases(tg):
+    """Out-of-memory graphs: no edges; every edge at one departure time (one block larger
+    than block_edges); a window that excludes every block."""
+    n = 40
+    g = _streamed(tg, n, *(np.zeros(0, np.uint32) for _ in range(4)), block_edges=4)
+    out = tg.as_u32(g.query("eat", [0, 3], (5, 9)))
+    assert out[0, 0] == 5 and out[1, 3] == 5 and (out[0, 1:] == NONE).all()
+    g.close()
+    rng = np.random.default_rng(12)
+    m = 500
+    u = rng.integers(0, n, m).astype(np.uint32); v = rng.integers(0, n, m).astype(np.uint32)
+    t = np.full(m, 7, np.uint32); lam = rng.integers(1, 4, m).astype(np.uint32)
+    og = oracle.Graph(n, u, v, t, lam)
+    g = _streamed(tg, n, u, v, t, lam, block_edges=16)
+    for win in [(0, 100), (8, 100), (0, 7)]:
+        _check_rows(tg, g, og, "eat", list(range(n)), win)
+    g.close()
