@@ -44,14 +44,18 @@ namespace cg = cooperative_groups;
 namespace {
 
 constexpr int QT = 256;                 // threads per block
-#ifndef TG_BIG_T
-#define TG_BIG_T 128
-#endif
-#ifndef TG_CHUNK
-#define TG_CHUNK 128
-#endif
-constexpr uint32_t BIG_T = TG_BIG_T;    // unions longer than this are split into chunks
-constexpr uint32_t CHUNK = TG_CHUNK;    // edges per chunk (one warp)
+// Unions longer than big_t edges are cut into big_t-edge chunks for k_eat_big, big_t =
+// 8 x the mean out-degree within [BIG_T_MIN, BIG_T_MAX]: denser graphs amortise a chunk's
+// record over more edges (C4, degree 32: 256 -> job -1.8 %; C2, degree 16: 128, 512 would
+// cost +16 %).  Queue capacities are sized for the smallest chunk.
+constexpr uint32_t BIG_T_MIN = 128, BIG_T_MAX = 512;
+constexpr uint32_t BIG_T = BIG_T_MIN;   // capacity sizing
+constexpr uint32_t CHUNK = BIG_T_MIN;
+
+static uint32_t pick_big_t(const tg_graph *g) {
+    const uint64_t deg = g->n ? g->m / g->n : 0;
+    return (uint32_t)std::min<uint64_t>(BIG_T_MAX, std::max<uint64_t>(BIG_T_MIN, 8 * deg));
+}
 constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in the activating thread
 #ifndef TG_MLP
 #define TG_MLP 4                        // state reads in flight per lane in the pair loop
@@ -88,6 +92,7 @@ struct EatP {
     uint32_t alpha, omega;
     int use_sc, stats;
     int omega_all;  // omega > every departure time: a vertex's window end is its last edge (no search)
+    uint32_t big_t;   // unions longer than this are cut into chunks of this many edges for k_eat_big
     RoundCtl *ctl;
     uint32_t round;       // GAC round of this launch (host loop counter; parity picks the bitmaps)
     uint32_t *fb0, *fb1;  // frontier masks [n][G] (bit = query within the group), by round parity
@@ -437,10 +442,10 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
                 uhi = max(uhi, __shfl_xor_sync(0xffffffffu, uhi, o));
             }
             if (ulo >= uhi) continue;
-            if (uhi - ulo > BIG_T) {
-                // long union: record the 32 ranges once, queue chunks of CHUNK edges
+            if (uhi - ulo > P.big_t) {
+                // long union: record the 32 ranges once, queue chunks of P.big_t edges
                 uint32_t rec = 0, k0 = 0;
-                const uint32_t nch = (uhi - ulo + CHUNK - 1) / CHUNK;
+                const uint32_t nch = (uhi - ulo + P.big_t - 1) / P.big_t;
                 if (lane == 0) {
                     rec = atomicAdd(R.rec_cnt, 1u);
                     k0 = atomicAdd(R.big_cnt, nch);
@@ -454,12 +459,12 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
                 uint32_t queued = 0;
                 if (k0 < P.bigcap) queued = min(nch, (uint32_t)(P.bigcap - k0));
                 for (uint32_t c = lane; c < queued; c += 32) {
-                    const uint32_t b0 = ulo + c * CHUNK;
-                    P.bigq[k0 + c] = rec_ok ? make_uint4(rec, b0, min(uhi, b0 + CHUNK), g) : make_uint4(0, 0, 0, g);
+                    const uint32_t b0 = ulo + c * P.big_t;
+                    P.bigq[k0 + c] = rec_ok ? make_uint4(rec, b0, min(uhi, b0 + P.big_t), g) : make_uint4(0, 0, 0, g);
                 }
                 if (rec_ok) {
                     if (queued == nch) continue;
-                    ulo = ulo + queued * CHUNK;  // the rest, in place
+                    ulo = ulo + queued * P.big_t;  // the rest, in place
                 }
             }
             unit_range<PK>(P, R, g, lo, hi, ulo, uhi, ws);
@@ -536,13 +541,13 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
             }
         }
         // long ranges: chunks for k_eat_big (query 0's range in lane 0 of the record)
-        const bool big = lo < hi && hi - lo > BIG_T;
+        const bool big = lo < hi && hi - lo > P.big_t;
         uint32_t bm = __ballot_sync(0xffffffffu, big);
         while (bm) {
             const int o = __ffs(bm) - 1;
             bm &= bm - 1;
             const uint32_t olo = __shfl_sync(0xffffffffu, lo, o), ohi = __shfl_sync(0xffffffffu, hi, o);
-            const uint32_t nch = (ohi - olo + CHUNK - 1) / CHUNK;
+            const uint32_t nch = (ohi - olo + P.big_t - 1) / P.big_t;
             uint32_t rec = 0, k0 = 0;
             if (lane == 0) {
                 rec = atomicAdd(R.rec_cnt, 1u);
@@ -555,13 +560,13 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
             uint32_t queued = 0;
             if (k0 < P.bigcap) queued = min(nch, (uint32_t)(P.bigcap - k0));
             for (uint32_t c = lane; c < queued; c += 32) {
-                const uint32_t b0 = olo + c * CHUNK;
-                P.bigq[k0 + c] = rec_ok ? make_uint4(rec, b0, min(ohi, b0 + CHUNK), 0) : make_uint4(0, 0, 0, 0);
+                const uint32_t b0 = olo + c * P.big_t;
+                P.bigq[k0 + c] = rec_ok ? make_uint4(rec, b0, min(ohi, b0 + P.big_t), 0) : make_uint4(0, 0, 0, 0);
             }
             // whatever is not queued stays with the owner lane for the shared pass below
             if (lane == o) {
                 if (rec_ok && queued == nch) { lo = 0; hi = 0; }
-                else if (rec_ok) lo = olo + queued * CHUNK;
+                else if (rec_ok) lo = olo + queued * P.big_t;
             }
         }
         // the remaining ranges, concatenated: lane takes edge t of the concatenation
@@ -1022,6 +1027,7 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.ub0 = 0; P.ub1 = g->n * G;
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
         P.omega_all = omega > dir_max_t(g, cgr) ? 1 : 0;
+        P.big_t = pick_big_t(g);
         P.ctl = Q.ctl; P.fb0 = Q.fb[0]; P.fb1 = Q.fb[1]; P.recs = Q.recs; P.reccap = Q.reccap;
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         P.touched = Q.touched;
@@ -1260,6 +1266,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
             base.n = g->n; base.S = Sb; base.G = G; base.alpha = alpha; base.omega = omega;
             base.use_sc = (int)g->opt_shortcuts; base.stats = (int)g->opt_stats;
             base.omega_all = 0;  // (per partition below)
+            base.big_t = pick_big_t(g);
             base.fb0 = Q.fb[0]; base.fb1 = Q.fb[1]; base.recs = Q.recs; base.reccap = Q.reccap;
             base.bigq = Q.bigq; base.bigcap = Q.bigcap; base.chq = Q.chq; base.chcap = Q.chcap;
             base.relax_cnt = Q.relax_cnt;
