@@ -63,9 +63,6 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_DEFER
 #define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
 #endif
-#ifndef TG_DENSE_ROW
-#define TG_DENSE_ROW 12                 // edges with at least this many new queries of the group: row mode (33 = off)
-#endif
 #ifndef TG_DEFER_FROM
 #define TG_DEFER_FROM 3                 // first round in which units may be deferred
 #endif
@@ -289,49 +286,6 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         // each query lane's range as a row of block bits, transposed across the warp
         uint32_t mask = tg_warp_transpose32(lo < hi ? tg_block_bits(lo, hi, pb) : 0u);
         if (p >= pend || (uint32_t)sl.y > P.omega) mask = 0;  // past the window end: never usable
-#if TG_DENSE_ROW < 33
-        {
-            // Dense edges (many of the group's queries new at once -- the common case once a
-            // sub-batch's queries are scheduled by start time): row mode, lanes = queries, one
-            // coalesced read of the edge's head row; two edges in flight.  The rest go through
-            // the pair list below.
-            uint32_t dm = __ballot_sync(0xffffffffu, __popc(mask) >= TG_DENSE_ROW);
-            const uint32_t q = g * 32 + lane;
-            while (dm) {
-                const int k1 = __ffs(dm) - 1;
-                dm &= dm - 1;
-                const int k2 = dm ? __ffs(dm) - 1 : k1;
-                if (dm) dm &= dm - 1;
-                const uint32_t m1 = __shfl_sync(0xffffffffu, mask, k1), m2 = __shfl_sync(0xffffffffu, mask, k2);
-                const int4 s1 = make_int4(__shfl_sync(0xffffffffu, sl.x, k1), __shfl_sync(0xffffffffu, sl.y, k1),
-                                          __shfl_sync(0xffffffffu, sl.z, k1), __shfl_sync(0xffffffffu, sl.w, k1));
-                const int4 s2 = make_int4(__shfl_sync(0xffffffffu, sl.x, k2), __shfl_sync(0xffffffffu, sl.y, k2),
-                                          __shfl_sync(0xffffffffu, sl.z, k2), __shfl_sync(0xffffffffu, sl.w, k2));
-                const uint32_t x1 = __shfl_sync(0xffffffffu, s, k1), x2 = __shfl_sync(0xffffffffu, s, k2);
-                const bool on1 = (m1 >> lane) & 1u, on2 = k2 != k1 && ((m2 >> lane) & 1u);
-                typename StW<PK>::T c1 = 0, c2 = 0;
-                if (on1 && (uint32_t)s1.w == TG_SINGLE) c1 = st_load<PK>(P, (size_t)(uint32_t)s1.x * P.S + q);
-                if (on2 && (uint32_t)s2.w == TG_SINGLE) c2 = st_load<PK>(P, (size_t)(uint32_t)s2.x * P.S + q);
-                if (on1) {
-                    if ((uint32_t)s1.w == TG_SINGLE)
-                        eat_relax_cur<PK>(P, R, q, x1, (uint32_t)s1.x, (uint32_t)s1.y, (uint32_t)s1.z, c1);
-                    else
-                        eat_long<PK>(P, R, q, x1, s1);
-                }
-                if (on2) {
-                    if ((uint32_t)s2.w == TG_SINGLE)
-                        eat_relax_cur<PK>(P, R, q, x2, (uint32_t)s2.x, (uint32_t)s2.y, (uint32_t)s2.z, c2);
-                    else
-                        eat_long<PK>(P, R, q, x2, s2);
-                }
-            }
-            if (P.stats) {
-                const uint32_t dp = __reduce_add_sync(0xffffffffu, __popc(mask) >= TG_DENSE_ROW ? __popc(mask) : 0u);
-                if (lane == 0 && dp) atomicAdd(P.diag + 2, (unsigned long long)dp);
-            }
-            if (__popc(mask) >= TG_DENSE_ROW) mask = 0;  // handled
-        }
-#endif
         const uint32_t cnt = __popc(mask);
         uint32_t incl = cnt;
 #pragma unroll
