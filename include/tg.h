@@ -293,6 +293,9 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *                engine, which is faster on the measured configs
  *   "dynamic"    1 = keep each direction's sorted edge order (before build; 4 B per edge
  *                and direction) so tg_graph_insert_edges re-transforms incrementally
+ *   "order_sources" 1 (default) = a call's sources are cut into sub-batches in order of
+ *                their first departure time >= t_alpha (results still go to the caller's
+ *                rows); 0 = in the caller's order
  *   "packed_state" 1 = EAT/LD/REACH keep the packed u64 (arrival << 32 | pred) state even
  *                when pred == NULL (default 0: without pred the state is the u32 arrival
  *                alone -- half the state bytes; values are identical) */
