@@ -7,5 +7,5 @@ timeout 1500 ncu --metrics gpu__time_duration.sum --clock-control none --kernel-
 for sb in 32 96 128; do timeout 300 python tools/variant_bench.py paper_conf_asplos_0003wh0dhwy0lyl25_b200/libtempgraph.so C4 $sb --problems=eat --opt=mirror:0 --opt=sub_batch:$sb >> gpurun_out/r2b/subbatch.log 2>&1; done
 timeout 600 python bench.py --config C5 --partitions 8 --query-only --k 1 --steps 5 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/r2b/bench_C5_k1.json 2> gpurun_out/r2b/bench_C5_k1.err; echo c5=$?
 timeout 600 python tools/dynamic_bench.py C2 100000 5 > gpurun_out/r2b/dynamic_C2.json 2> gpurun_out/r2b/dynamic_C2.err; echo dyn=$?
-timeout 3000 python -m pytest tests/test_gpu_fullsize.py -x -q > gpurun_out/r2b/pytest_fullsize.log 2>&1; echo full=$?
+timeout 3000 python -m pytest tests/test_gpu_parity_fullsize.py -x -q > gpurun_out/r2b/pytest_fullsize.log 2>&1; echo full=$?
 tail -3 gpurun_out/r2b/pytest_fullsize.log; grep median gpurun_out/r2b/subbatch.log; cat gpurun_out/r2b/dynamic_C2.json
