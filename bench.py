@@ -409,6 +409,8 @@ def run_ours(a, rank, world, local_rank):
             "frac": ach / peak if ach else None,
             "traffic": (traffic["dram_bytes_per_step"] if traffic else None),
             "traffic_source": (os.path.relpath(tf, ROOT) + ": " + traffic["source"]) if traffic else None,
+            "traffic_vs_algorithmic": (traffic["dram_bytes_per_step"] / (relax_bytes / a.steps)) if traffic else None,
+            "ncu_dram_GBps": traffic.get("ncu_GBps") if traffic else None,
             "peak_source": peak_src,
             "algorithmic_bytes_per_step": relax_bytes / a.steps,
             "algorithmic_bytes_formula": ("20 B x W_union + 4 B x sum_q W_q (SURVEY 8(d) batched source lanes, "
