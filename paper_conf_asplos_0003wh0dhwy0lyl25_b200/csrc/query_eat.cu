@@ -63,6 +63,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_DEFER
 #define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
 #endif
+#ifndef TG_PAIR_REGS
+#define TG_PAIR_REGS 1                  // pair entries and edge records kept in registers across the pair loop
+#endif
 #ifndef TG_DEFER_FROM
 #define TG_DEFER_FROM 3                 // first round in which units may be deferred
 #endif
@@ -162,17 +165,17 @@ __device__ __forceinline__ typename StW<PK>::T st_load(const EatP &P, size_t i) 
 // Relax (v, q) with (arr, id) given a value `cur` read earlier from the state (any
 // earlier read: states only decrease, so a stale value is an upper bound and when it
 // is already <= the candidate the atomic cannot change anything -- most relaxations).
-template <bool PK>
+template <bool PK, bool ST>
 __device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, uint32_t q, uint32_t slot, uint32_t v,
                                               uint32_t arr, uint32_t id, typename StW<PK>::T cur) {
     using W = StW<PK>;
-    if (P.stats) {  // work counters: relaxations per query, distinct slots of the sub-batch
+    if (ST) {  // work counters: relaxations per query, distinct slots of the sub-batch
         atomicAdd(P.relax_cnt + q, 1ull);
         atomicOr(P.touched + (slot >> 5), 1u << (slot & 31));
     }
     const typename W::T pk = W::make(arr, id);
     if (cur <= pk) return;
-    if (P.stats) atomicAdd(P.diag + 5, 1ull);  // relaxations past the filter read
+    if (ST) atomicAdd(P.diag + 5, 1ull);  // relaxations past the filter read
     const size_t i = (size_t)v * P.S + q;
     // fire-and-forget min (RED): nobody waits on the old value.  The frontier bit is set
     // whenever the (possibly stale) read says the arrival improves: if a concurrent
@@ -184,10 +187,10 @@ __device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, ui
     if (arr < W::time(cur)) atomicOr(R.fout + (size_t)v * P.G + (q >> 5), 1u << (q & 31));
 }
 
-template <bool PK>
+template <bool PK, bool ST>
 __device__ __forceinline__ void eat_relax(const EatP &P, const RoundV &R, uint32_t q, uint32_t slot, uint32_t v,
                                           uint32_t arr, uint32_t id) {
-    eat_relax_cur<PK>(P, R, q, slot, v, arr, id, st_load<PK>(P, (size_t)v * P.S + q));
+    eat_relax_cur<PK, ST>(P, R, q, slot, v, arr, id, st_load<PK>(P, (size_t)v * P.S + q));
 }
 
 // test-and-set of slot s's claim bit for query q; true if this caller claimed it
@@ -198,30 +201,30 @@ __device__ __forceinline__ bool claim(const EatP &P, uint32_t q, uint32_t s) {
 
 // sequential walk over slots [s, s_end): claim, relax, continue; stop at a slot
 // somebody else claimed (they continue) or past omega.
-template <bool PK>
+template <bool PK, bool ST>
 __device__ __forceinline__ void eat_walk(const EatP &P, const RoundV &R, uint32_t q, uint32_t s, uint32_t s_end) {
     for (; s < s_end; s++) {
         const int4 sl = tg_ld_slot(P.slots + s);
         if ((uint32_t)sl.y > P.omega) return;  // arrivals increase strictly along a chain
         if (!claim(P, q, s)) return;
-        eat_relax<PK>(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+        eat_relax<PK, ST>(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     }
 }
 
 // A newly usable occurrence at slot s (already loaded) of a long chain.
-template <bool PK>
+template <bool PK, bool ST>
 __device__ __forceinline__ void eat_long(const EatP &P, const RoundV &R, uint32_t q, uint32_t s, int4 sl) {
     const uint32_t l = (uint32_t)sl.w;
     const uint2 info = __ldg(P.lc + l);  // {first slot, length}
     if (s != info.x && !claim(P, q, s)) return;  // a walker from an earlier entry got here first
-    eat_relax<PK>(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+    eat_relax<PK, ST>(P, R, q, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
     uint32_t s_end = info.x + info.y;
     if (s + 1 >= s_end) return;
     if (P.use_sc) {
         // skeleton: Propagate along the shortcut head -> tail (Alg. 2 / Alg. 3 line 6)
         const int4 scv = __ldg(P.sc + l);
         if ((uint32_t)scv.y <= P.omega && claim(P, q, s_end - 1)) {
-            eat_relax<PK>(P, R, q, s_end - 1, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
+            eat_relax<PK, ST>(P, R, q, s_end - 1, (uint32_t)scv.x, (uint32_t)scv.y, (uint32_t)scv.z);
             s_end -= 1;
         }
     }
@@ -232,7 +235,7 @@ __device__ __forceinline__ void eat_long(const EatP &P, const RoundV &R, uint32_
             return;
         }
     }
-    eat_walk<PK>(P, R, q, s + 1, s_end);
+    eat_walk<PK, ST>(P, R, q, s + 1, s_end);
 }
 
 // Per-warp shared-memory staging of one 32-edge block: the (edge, query) pairs
@@ -243,11 +246,11 @@ struct WarpStage {
     uint32_t sidx[32];
 };
 
-template <bool PK>
+template <bool PK, bool ST>
 __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint32_t g, uint32_t lo, uint32_t hi,
                                            uint32_t pbeg, uint32_t pend, WarpStage &ws) {
     const int lane = threadIdx.x & 31;
-    if (P.stats && lane == 0) {
+    if (ST && lane == 0) {
         atomicAdd(P.diag + 0, (unsigned long long)(pend - pbeg));
         atomicAdd(P.diag + 1, 1ull);
     }
@@ -278,7 +281,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
                     sl = tg_ld_slot(P.slots + s);
                 } else {
                     sl = make_int4((int)r.x, (int)r.y, 0, (int)TG_SINGLE);
-                    if (P.stats) s = __ldg(P.occ_slot + p);  // distinct-slot counter
+                    if (ST) s = __ldg(P.occ_slot + p);  // distinct-slot counter
                 }
             }
         }
@@ -295,7 +298,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         }
         const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
         if (total == 0) { pb += 32; continue; }
-        if (P.stats && lane == 0) atomicAdd(P.diag + 2, (unsigned long long)total);
+        if (ST && lane == 0) atomicAdd(P.diag + 2, (unsigned long long)total);
         // expand: edge lane k writes its pairs at [incl - cnt, incl) in edge-major order
         ws.slot[lane] = sl;
         ws.sidx[lane] = s;
@@ -311,6 +314,35 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         // latency the relax phase waits on), then each is filtered / relaxed.
         for (uint32_t t0 = 0; t0 < total; t0 += 32 * TG_MLP) {
             typename StW<PK>::T cur[TG_MLP];
+#if TG_PAIR_REGS
+            // each pair's entry and its edge's {head, arrival} read from shared memory once,
+            // kept in registers between the state reads and the relaxations
+            uint32_t pe[TG_MLP], pv[TG_MLP], pa[TG_MLP];
+#pragma unroll
+            for (int j = 0; j < TG_MLP; j++) {
+                const uint32_t t = t0 + j * 32 + lane;
+                pe[j] = 0xFFFFFFFFu;
+                if (t < total) {
+                    const uint32_t e = ws.pairs[t];
+                    const int4 osl = ws.slot[e >> 5];
+                    pe[j] = e;
+                    pv[j] = (uint32_t)osl.x;
+                    pa[j] = (uint32_t)osl.w == TG_SINGLE ? (uint32_t)osl.y : 0xFFFFFFFFu;  // NONE: walked chain
+                    if (pa[j] != 0xFFFFFFFFu) cur[j] = st_load<PK>(P, (size_t)pv[j] * P.S + g * 32 + (e & 31));
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < TG_MLP; j++) {
+                if (pe[j] == 0xFFFFFFFFu) continue;
+                const uint32_t k = pe[j] >> 5;
+                const uint32_t q = g * 32 + (pe[j] & 31);
+                if (pa[j] != 0xFFFFFFFFu)
+                    eat_relax_cur<PK, ST>(P, R, q, ST ? ws.sidx[k] : 0u, pv[j], pa[j],
+                                          PK ? (uint32_t)ws.slot[k].z : 0u, cur[j]);
+                else
+                    eat_long<PK, ST>(P, R, q, ws.sidx[k], ws.slot[k]);
+            }
+#else
 #pragma unroll
             for (int j = 0; j < TG_MLP; j++) {
                 const uint32_t t = t0 + j * 32 + lane;
@@ -330,12 +362,13 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
                     const uint32_t q = g * 32 + (e & 31);
                     const int4 osl = ws.slot[k];
                     if ((uint32_t)osl.w == TG_SINGLE)
-                        eat_relax_cur<PK>(P, R, q, ws.sidx[k], (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z,
+                        eat_relax_cur<PK, ST>(P, R, q, ws.sidx[k], (uint32_t)osl.x, (uint32_t)osl.y, (uint32_t)osl.z,
                                           cur[j]);
                     else
-                        eat_long<PK>(P, R, q, ws.sidx[k], osl);
+                        eat_long<PK, ST>(P, R, q, ws.sidx[k], osl);
                 }
             }
+#endif
         }
         __syncwarp();
         pb += 32;
@@ -349,7 +382,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
 // an edge index (atomicMin makes concurrent activations disjoint).  The union of
 // the lanes' ranges is relaxed edge-major (unit_range); long unions are split into
 // chunks for k_eat_big.
-template <bool PK>
+template <bool PK, bool ST>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
     clear_next_round(P);
@@ -429,10 +462,10 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
                 if (hi == TG_NONE) hi = ehi;
             }
             if (lo >= hi) { lo = 0; hi = 0; }
-            if (P.stats && lane == 0) {
+            if (ST && lane == 0) {
                 atomicAdd(P.diag + 3, (unsigned long long)__popc(__ballot_sync(0xffffffffu, lo < hi)));
                 atomicAdd(P.diag + 4, (unsigned long long)__popc(qm));
-            } else if (P.stats) {
+            } else if (ST) {
                 __ballot_sync(0xffffffffu, lo < hi);
             }
             uint32_t ulo = (lo < hi) ? lo : 0xFFFFFFFFu, uhi = hi;
@@ -467,7 +500,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
                     ulo = ulo + queued * P.big_t;  // the rest, in place
                 }
             }
-            unit_range<PK>(P, R, g, lo, hi, ulo, uhi, ws);
+            unit_range<PK, ST>(P, R, g, lo, hi, ulo, uhi, ws);
         }
     }
     if (lane == 0 && my_units) atomicAdd(R.words_cnt, my_units);  // per warp: no block barrier
@@ -481,7 +514,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
 // lane 0); the rest are relaxed by the warp together: each lane takes one edge of the
 // concatenated ranges (owner found by a shuffle search over the prefix sums).
 constexpr uint32_t LANE_SEARCH_MAX = 64;  // departure nodes a lane searches alone
-template <bool PK>
+template <bool PK, bool ST>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
     const RoundV R = round_view(P);
     clear_next_round(P);
@@ -533,7 +566,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
                 hi = 0;
             }
         }
-        if (P.stats) {
+        if (ST) {
             const uint32_t act_n = __popc(__ballot_sync(0xffffffffu, lo < hi));
             if (lane == 0) {
                 atomicAdd(P.diag + 3, (unsigned long long)act_n);
@@ -578,7 +611,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
             if (lane >= o) incl += y;
         }
         const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-        if (P.stats && lane == 0 && total) atomicAdd(P.diag + 0, (unsigned long long)total);
+        if (ST && lane == 0 && total) atomicAdd(P.diag + 0, (unsigned long long)total);
         for (uint32_t t0 = 0; t0 < total; t0 += 32) {
             const uint32_t t = t0 + lane;
             uint32_t k = 0;  // owner: first lane with incl > t
@@ -604,19 +637,19 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
                     sl = tg_ld_slot(P.slots + s);
                 } else {
                     sl = make_int4((int)r.x, (int)r.y, 0, (int)TG_SINGLE);
-                    if (P.stats) s = __ldg(P.occ_slot + p);
+                    if (ST) s = __ldg(P.occ_slot + p);
                 }
             }
             if ((uint32_t)sl.y > P.omega) continue;  // past the window end: never usable
-            if ((uint32_t)sl.w == TG_SINGLE) eat_relax<PK>(P, R, 0, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
-            else eat_long<PK>(P, R, 0, s, sl);
+            if ((uint32_t)sl.w == TG_SINGLE) eat_relax<PK, ST>(P, R, 0, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+            else eat_long<PK, ST>(P, R, 0, s, sl);
         }
     }
     if (lane == 0 && my_units) atomicAdd(R.words_cnt, my_units);
 }
 
 // Chunks of long unions: one warp per chunk, the unit's 32 query ranges from its record.
-template <bool PK>
+template <bool PK, bool ST>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_big(EatP P) {
     const RoundV R = round_view(P);
     __shared__ WarpStage stage[QT / 32];
@@ -628,14 +661,14 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_big(EatP P) {
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
         const uint2 r = P.recs[(size_t)c.x * 32 + lane];
-        unit_range<PK>(P, R, c.w, r.x, r.y, c.y, c.z, ws);
+        unit_range<PK, ST>(P, R, c.w, r.x, r.y, c.y, c.z, ws);
     }
 }
 
 // ChainEngine: warp per queued walk, lanes over consecutive slots; the warp
 // continues iff its last lane claimed its slot (otherwise that slot's claimer
 // continues the chain).
-template <bool PK>
+template <bool PK, bool ST>
 __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
     const RoundV R = round_view(P);
     const uint32_t C = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.ch_cnt, P.chcap);
@@ -652,7 +685,7 @@ __global__ void __launch_bounds__(QT) k_eat_chain(EatP P) {
                 if ((uint32_t)sl.y > P.omega) {
                     past = true;
                 } else if (claim(P, c.x, s)) {
-                    eat_relax<PK>(P, R, c.x, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
+                    eat_relax<PK, ST>(P, R, c.x, s, (uint32_t)sl.x, (uint32_t)sl.y, (uint32_t)sl.z);
                     cont = true;
                 }
             }
@@ -978,6 +1011,26 @@ template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
                           cudaStream_t s, uint32_t *rounds_out);
 
+// One GAC round's relax kernels; the stats counters are a template argument so that the
+// timed path carries no per-pair stats branch.
+template <bool PK, bool ST>
+static tg_status launch_round(const EatP &P, uint32_t S, uint32_t grid, cudaStream_t s, cudaEvent_t *tev) {
+    if (tev) cudaEventRecord(tev[0], s);
+    if (S == 1) TG_LAUNCH_RELAX((k_eat_activate1<PK, ST>), grid, QT, 0, s, P);
+    else TG_LAUNCH_RELAX((k_eat_activate<PK, ST>), grid, QT, 0, s, P);
+    if (tev) cudaEventRecord(tev[1], s);
+    TG_LAUNCH_RELAX((k_eat_big<PK, ST>), grid, QT, 0, s, P);
+    if (tev) cudaEventRecord(tev[2], s);
+    TG_LAUNCH_RELAX((k_eat_chain<PK, ST>), 148, QT, 0, s, P);  // at most a few hundred walks per round
+    if (tev) cudaEventRecord(tev[3], s);
+    return TG_OK;
+}
+
+template <bool PK>
+static tg_status relax_round(const EatP &P, uint32_t S, uint32_t grid, cudaStream_t s, cudaEvent_t *tev) {
+    return P.stats ? launch_round<PK, true>(P, S, grid, s, tev) : launch_round<PK, false>(P, S, grid, s, tev);
+}
+
 // largest departure time of a direction: forward max t; the LD mirror's departures are
 // C - (t + lambda) <= C - min t - 1 (a bound is enough: it only enables a shortcut)
 static uint32_t dir_max_t(const tg_graph *g, const ChainGraph &cg) {
@@ -1043,14 +1096,7 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         for (;;) {
             for (int k = 0; k < group; k++, r++) {
                 P.round = r;
-                if (trace) cudaEventRecord(tev[0], s);
-                if (S == 1) TG_LAUNCH_RELAX(k_eat_activate1<PK>, grid, QT, 0, s, P);
-                else TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, P);
-                if (trace) cudaEventRecord(tev[1], s);
-                TG_LAUNCH_RELAX(k_eat_big<PK>, grid, QT, 0, s, P);
-                if (trace) cudaEventRecord(tev[2], s);
-                TG_LAUNCH_RELAX(k_eat_chain<PK>, 148, QT, 0, s, P);  // at most a few hundred walks per round
-                if (trace) cudaEventRecord(tev[3], s);
+                TG_TRY(relax_round<PK>(P, S, grid, s, trace ? tev : nullptr));
             }
             TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
@@ -1307,10 +1353,7 @@ static tg_status eat_partitioned(tg_graph *g, tg_problem p, const uint32_t *sour
                 for (int pi = 0; pi < g->nparts; pi++) {
                     if (parts[pi].ub0 == parts[pi].ub1) continue;  // no vertices: never any work
                     parts[pi].round = r;
-                    if (Sb == 1) TG_LAUNCH_RELAX(k_eat_activate1<PK>, grid, QT, 0, s, parts[pi]);
-                    else TG_LAUNCH_RELAX(k_eat_activate<PK>, grid, QT, 0, s, parts[pi]);
-                    TG_LAUNCH_RELAX(k_eat_big<PK>, grid, QT, 0, s, parts[pi]);
-                    TG_LAUNCH_RELAX(k_eat_chain<PK>, 148, QT, 0, s, parts[pi]);
+                    TG_TRY(relax_round<PK>(parts[pi], Sb, grid, s, nullptr));
                 }
                 if (local) {
                     // a round in which no partition consumed a frontier word did no work
