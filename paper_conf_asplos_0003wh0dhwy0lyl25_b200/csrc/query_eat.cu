@@ -63,9 +63,6 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_DEFER
 #define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
 #endif
-#ifndef TG_PAIR_REGS
-#define TG_PAIR_REGS 1                  // pair entries and edge records kept in registers across the pair loop
-#endif
 #ifndef TG_DEFER_FROM
 #define TG_DEFER_FROM 3                 // first round in which units may be deferred
 #endif
@@ -314,35 +311,6 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         // latency the relax phase waits on), then each is filtered / relaxed.
         for (uint32_t t0 = 0; t0 < total; t0 += 32 * TG_MLP) {
             typename StW<PK>::T cur[TG_MLP];
-#if TG_PAIR_REGS
-            // each pair's entry and its edge's {head, arrival} read from shared memory once,
-            // kept in registers between the state reads and the relaxations
-            uint32_t pe[TG_MLP], pv[TG_MLP], pa[TG_MLP];
-#pragma unroll
-            for (int j = 0; j < TG_MLP; j++) {
-                const uint32_t t = t0 + j * 32 + lane;
-                pe[j] = 0xFFFFFFFFu;
-                if (t < total) {
-                    const uint32_t e = ws.pairs[t];
-                    const int4 osl = ws.slot[e >> 5];
-                    pe[j] = e;
-                    pv[j] = (uint32_t)osl.x;
-                    pa[j] = (uint32_t)osl.w == TG_SINGLE ? (uint32_t)osl.y : 0xFFFFFFFFu;  // NONE: walked chain
-                    if (pa[j] != 0xFFFFFFFFu) cur[j] = st_load<PK>(P, (size_t)pv[j] * P.S + g * 32 + (e & 31));
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < TG_MLP; j++) {
-                if (pe[j] == 0xFFFFFFFFu) continue;
-                const uint32_t k = pe[j] >> 5;
-                const uint32_t q = g * 32 + (pe[j] & 31);
-                if (pa[j] != 0xFFFFFFFFu)
-                    eat_relax_cur<PK, ST>(P, R, q, ST ? ws.sidx[k] : 0u, pv[j], pa[j],
-                                          PK ? (uint32_t)ws.slot[k].z : 0u, cur[j]);
-                else
-                    eat_long<PK, ST>(P, R, q, ws.sidx[k], ws.slot[k]);
-            }
-#else
 #pragma unroll
             for (int j = 0; j < TG_MLP; j++) {
                 const uint32_t t = t0 + j * 32 + lane;
@@ -368,7 +336,6 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
                         eat_long<PK, ST>(P, R, q, ws.sidx[k], osl);
                 }
             }
-#endif
         }
         __syncwarp();
         pb += 32;
