@@ -111,12 +111,12 @@ __device__ __forceinline__ void push_node(const SpP &P, const RoundV &R, uint32_
 }
 
 // Walk the chain from slot s (entered with head-node value cur).
-template <int MODE>
+template <int MODE, bool ST>
 __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s, uint32_t s_end, uint32_t cur) {
     uint32_t *dn = P.dnode + (size_t)q * P.nnodes;
     uint32_t *vo = P.vout + (size_t)q * P.n;
     for (; s < s_end; s++) {
-        if (P.stats) atomicAdd(P.cnt + 0, 1ull);
+        if (ST) atomicAdd(P.cnt + 0, 1ull);
         const int4 sl = tg_ld_slot(P.slots + s);
         const uint32_t arr = (uint32_t)sl.y;
         if (arr > P.omega) return;
@@ -144,7 +144,7 @@ __device__ void spfp_walk(const SpP &P, const RoundV &R, uint32_t q, uint32_t s,
     }
 }
 
-template <int MODE>
+template <int MODE, bool ST>
 __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_t q, uint32_t p) {
     // occurrence-ordered record {v, arrival | walked flag, tail node, w}: an edge that is
     // not on a walked chain needs nothing else (no slot, weight or tail-node gathers)
@@ -155,7 +155,7 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_
     if (!(rc.y >> 31)) {
         const uint32_t arr = rc.y;
         if (arr > P.omega) return;
-        if (P.stats) atomicAdd(P.cnt + 0, 1ull);
+        if (ST) atomicAdd(P.cnt + 0, 1ull);
         uint32_t cand, val;
         if (MODE == 1) { cand = cur; val = arr - (0xFFFFFFFEu - cur); }
         else if (MODE == 2) { cand = cur; val = cur; }
@@ -201,10 +201,10 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_
             }
         }
     }
-    spfp_walk<MODE>(P, R, q, s, s_end, cur);
+    spfp_walk<MODE, ST>(P, R, q, s, s_end, cur);
 }
 
-template <int MODE>
+template <int MODE, bool ST>
 __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
     const RoundV R = round_view(P);
     clear_later_rounds(P);
@@ -244,7 +244,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
                     if (stop) continue;
                     // no valid out-edge departs at >= omega; a node at <= d ends the walk
                     if (tt[k] >= P.omega || dd[k] <= d || steps == WAIT_INLINE) { stop = true; continue; }
-                    if (P.stats) atomicAdd(P.cnt + 1, 1ull);
+                    if (ST) atomicAdd(P.cnt + 1, 1ull);
                     atomicMin(dn + jend, d);
                     jend++;
                     steps++;
@@ -280,7 +280,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             for (uint32_t c = 0; c < nch; c++) {
                 const uint32_t b0 = e0 + c * CHUNK, b1 = min(e0 + cnt, b0 + CHUNK);
                 if (k + c < P.bigcap) P.bigq[k + c] = make_uint4(q, b0, b1, 0);
-                else for (uint32_t p = b0; p < b1; p++) spfp_edge<MODE>(P, R, q, p);
+                else for (uint32_t p = b0; p < b1; p++) spfp_edge<MODE, ST>(P, R, q, p);
             }
             cnt = 0;
         }
@@ -304,7 +304,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
             const uint32_t oe0 = __shfl_sync(0xffffffffu, e0, own);
             const uint32_t oex = __shfl_sync(0xffffffffu, excl, own);
             const uint32_t oq = __shfl_sync(0xffffffffu, q, own);
-            if (g < total) spfp_edge<MODE>(P, R, oq, oe0 + (g - oex));
+            if (g < total) spfp_edge<MODE, ST>(P, R, oq, oe0 + (g - oex));
         }
     }
 }
@@ -314,7 +314,7 @@ __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
 // out-edges are queued as chunks for k_spfp_big of the same round.  Nodes past the
 // first non-improving one that still improved (legal: waiting is transitive) are
 // pushed to the next frontier.
-template <int MODE>
+template <int MODE, bool ST>
 __global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
     const RoundV R = round_view(P);
     const uint32_t NW = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.wait_cnt, P.waitcap);
@@ -331,7 +331,7 @@ __global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
             const uint32_t jj = j + lane;
             bool stop = true, improved = false;
             if (jj < vend && __ldg(P.node_t + jj) < P.omega) {
-                if (P.stats) atomicAdd(P.cnt + 1, 1ull);
+                if (ST) atomicAdd(P.cnt + 1, 1ull);
                 improved = __ldcg(dn + jj) > d;  // plain read: stale-safe (see the inline walk)
                 if (improved) atomicMin(dn + jj, d);
                 stop = !improved;
@@ -352,13 +352,13 @@ __global__ void __launch_bounds__(QT) k_spfp_wait(SpP P) {
             for (uint32_t cc = lane; cc < nch; cc += 32) {
                 const uint32_t b0 = e0 + cc * CHUNK, b1 = min(e1, b0 + CHUNK);
                 if (k + cc < P.bigcap) P.bigq[k + cc] = make_uint4(q, b0, b1, 0);
-                else for (uint32_t pp = b0; pp < b1; pp++) spfp_edge<MODE>(P, R, q, pp);
+                else for (uint32_t pp = b0; pp < b1; pp++) spfp_edge<MODE, ST>(P, R, q, pp);
             }
         }
     }
 }
 
-template <int MODE>
+template <int MODE, bool ST>
 __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
     const RoundV R = round_view(P);
     const uint32_t B = (uint32_t)min((uint64_t)*(volatile uint32_t *)R.big_cnt, P.bigcap);
@@ -367,7 +367,7 @@ __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
-        for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<MODE>(P, R, c.x, p);
+        for (uint32_t p = c.y + lane; p < c.z; p += 32) spfp_edge<MODE, ST>(P, R, c.x, p);
     }
 }
 
@@ -468,11 +468,14 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
             P.round = r;
             P.stamp = ++Q.stamp;
             if (trace) cudaEventRecord(tev[0], s);
-            TG_LAUNCH_RELAX(k_spfp_activate<MODE>, grid, QT, 0, s, P);
+            if (P.stats) TG_LAUNCH_RELAX((k_spfp_activate<MODE, true>), grid, QT, 0, s, P);
+            else TG_LAUNCH_RELAX((k_spfp_activate<MODE, false>), grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[1], s);
-            TG_LAUNCH_RELAX(k_spfp_wait<MODE>, grid, QT, 0, s, P);
+            if (P.stats) TG_LAUNCH_RELAX((k_spfp_wait<MODE, true>), grid, QT, 0, s, P);
+            else TG_LAUNCH_RELAX((k_spfp_wait<MODE, false>), grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[2], s);
-            TG_LAUNCH_RELAX(k_spfp_big<MODE>, grid, QT, 0, s, P);
+            if (P.stats) TG_LAUNCH_RELAX((k_spfp_big<MODE, true>), grid, QT, 0, s, P);
+            else TG_LAUNCH_RELAX((k_spfp_big<MODE, false>), grid, QT, 0, s, P);
             if (trace) cudaEventRecord(tev[3], s);
         }
         TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
