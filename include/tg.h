@@ -298,7 +298,12 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *                rows); 0 = in the caller's order
  *   "packed_state" 1 = EAT/LD/REACH keep the packed u64 (arrival << 32 | pred) state even
  *                when pred == NULL (default 0: without pred the state is the u32 arrival
- *                alone -- half the state bytes; values are identical) */
+ *                alone -- half the state bytes; values are identical)
+ *   "ub_filter"  EAT/LD/REACH batches of 2..64 queries: per (vertex, 8 queries) an 8-bit
+ *                code of an upper bound of their arrivals, refreshed at activation, lets
+ *                an edge skip the queries it cannot improve before any state read.
+ *                0 = off, 1 (default) = on when the sub-batch state is >= 1 GiB, 2 = on.
+ *                Results are identical either way. */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
 
 /* Total kernels this library has launched in this process (all handles). */

@@ -72,6 +72,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_COOP_SEARCH
 #define TG_COOP_SEARCH 1                // warp-cooperative departure-time search in the activation
 #endif
+#ifndef TG_UB
+#define TG_UB 1                         // per-(vertex, 8 queries) arrival bounds prune (edge, query) pairs
+#endif
 #ifndef TG_ACT_MINB
 #define TG_ACT_MINB 6                   // resident blocks per SM requested for the relax kernels (8, 7, 5, 4 measured slower)
 #endif
@@ -83,6 +86,9 @@ struct EatP {
     const uint2 *lc;
     const int4 *sc;
     void *st;  // [v * S + q]: packed u64 (arrival << 32 | pred) when PK, else u32 arrival
+    unsigned long long *ub;  // [v]: byte j = code of an upper bound of the arrivals of queries
+                             // 8j .. 8j+7 at v (255 = none); NULL = off (TG_UB)
+    uint32_t ub_sh;          // code c <-> bound alpha + (c << ub_sh)
     uint32_t *act, *bits;
     uint32_t *touched;  // stats: slots relaxed by any query of the sub-batch
     uint32_t *defer;    // TG_DEFER experiment: units deferred once (bit per unit)
@@ -243,7 +249,7 @@ struct WarpStage {
     uint32_t sidx[32];
 };
 
-template <bool PK, bool ST>
+template <bool PK, bool ST, bool UB>
 __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint32_t g, uint32_t lo, uint32_t hi,
                                            uint32_t pbeg, uint32_t pend, WarpStage &ws) {
     const int lane = threadIdx.x & 31;
@@ -265,6 +271,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         const uint32_t p = pb + lane;
         uint32_t s = 0;
         int4 sl = make_int4(0, -1, 0, 0);
+        unsigned long long ubw = ~0ull;
         if (p < pend) {
             if (PK) {  // the pred needs the edge id: the full slot
                 s = __ldg(P.occ_slot + p);
@@ -279,6 +286,9 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
                 } else {
                     sl = make_int4((int)r.x, (int)r.y, 0, (int)TG_SINGLE);
                     if (ST) s = __ldg(P.occ_slot + p);  // distinct-slot counter
+#if TG_UB
+                    if (UB) ubw = __ldcg(P.ub + r.x);
+#endif
                 }
             }
         }
@@ -286,6 +296,15 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         // each query lane's range as a row of block bits, transposed across the warp
         uint32_t mask = tg_warp_transpose32(lo < hi ? tg_block_bits(lo, hi, pb) : 0u);
         if (p >= pend || (uint32_t)sl.y > P.omega) mask = 0;  // past the window end: never usable
+#if TG_UB
+        // one-edge chains: the queries of an 8-query block whose arrival bound at the head
+        // is already <= the candidate (packed states: <) cannot improve -- no pair at all.
+        // code <= d  <=>  alpha + (code << sh) <= arrival - (PK ? 1 : 0); code 255 never is.
+        if (UB && ubw != ~0ull) {
+            const uint32_t d = min(254u, ((uint32_t)sl.y - P.alpha - (PK ? 1u : 0u)) >> P.ub_sh);
+            mask &= ~__vcmpleu4((uint32_t)(ubw >> (g * 32)), d * 0x01010101u);
+        }
+#endif
         const uint32_t cnt = __popc(mask);
         uint32_t incl = cnt;
 #pragma unroll
@@ -349,7 +368,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
 // an edge index (atomicMin makes concurrent activations disjoint).  The union of
 // the lanes' ranges is relaxed edge-major (unit_range); long unions are split into
 // chunks for k_eat_big.
-template <bool PK, bool ST>
+template <bool PK, bool ST, bool UB>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
     clear_next_round(P);
@@ -402,6 +421,23 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
             // consumed once), so the boundary needs no atomic: plain load, issued with the
             // state load, and a plain store
             uint32_t prev = 0, now = 0;
+#if TG_UB
+            if (UB) {
+                // refresh the group's arrival bounds at v from every query's state (one
+                // coalesced row; states only decrease, so any refresh stays a bound)
+                uint32_t code = 0;  // lanes past S hold no query
+                if (q < P.S) {
+                    const uint32_t x = StW<PK>::time(__ldcg((const typename StW<PK>::T *)P.st + si));
+                    if (on) now = x;
+                    code = x == 0xFFFFFFFFu ? 255u : (x - P.alpha + (1u << P.ub_sh) - 1) >> P.ub_sh;
+                }
+                code = max(code, __shfl_xor_sync(0xffffffffu, code, 1));
+                code = max(code, __shfl_xor_sync(0xffffffffu, code, 2));
+                code = max(code, __shfl_xor_sync(0xffffffffu, code, 4));
+                if ((lane & 7) == 0) ((uint8_t *)(P.ub + v))[g * 4 + (lane >> 3)] = (uint8_t)code;
+                if (on) prev = __ldcg(P.act + si);
+            } else
+#endif
             if (on) {
                 prev = __ldcg(P.act + si);
                 now = StW<PK>::time(__ldcg((const typename StW<PK>::T *)P.st + si));
@@ -467,7 +503,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
                     ulo = ulo + queued * P.big_t;  // the rest, in place
                 }
             }
-            unit_range<PK, ST>(P, R, g, lo, hi, ulo, uhi, ws);
+            unit_range<PK, ST, UB>(P, R, g, lo, hi, ulo, uhi, ws);
         }
     }
     if (lane == 0 && my_units) atomicAdd(R.words_cnt, my_units);  // per warp: no block barrier
@@ -616,7 +652,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
 }
 
 // Chunks of long unions: one warp per chunk, the unit's 32 query ranges from its record.
-template <bool PK, bool ST>
+template <bool PK, bool ST, bool UB>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_big(EatP P) {
     const RoundV R = round_view(P);
     __shared__ WarpStage stage[QT / 32];
@@ -628,7 +664,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_big(EatP P) {
     for (uint32_t it = gw; it < B; it += nw) {
         const uint4 c = P.bigq[it];
         const uint2 r = P.recs[(size_t)c.x * 32 + lane];
-        unit_range<PK, ST>(P, R, c.w, r.x, r.y, c.y, c.z, ws);
+        unit_range<PK, ST, UB>(P, R, c.w, r.x, r.y, c.y, c.z, ws);
     }
 }
 
@@ -906,6 +942,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     Q.st_copies = copies;
     TG_TRY(A.alloc((void **)&Q.st, S * n * 8 * copies));
     TG_TRY(A.alloc((void **)&Q.act, S * n * 4));
+    if (TG_UB) TG_TRY(A.alloc((void **)&Q.ub, n * 8));
     Q.vwords = (uint32_t)((S + 31) / 32);  // query groups per vertex
     TG_TRY(A.alloc((void **)&Q.fb[0], n * Q.vwords * 4));
     TG_TRY(A.alloc((void **)&Q.fb[1], n * Q.vwords * 4));
@@ -976,7 +1013,7 @@ tg_status tg_ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) { return 
 
 template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
-                          cudaStream_t s, uint32_t *rounds_out);
+                          cudaStream_t s, uint32_t *rounds_out, bool ub = false);
 
 // One GAC round's relax kernels; the stats counters are a template argument so that the
 // timed path carries no per-pair stats branch.
@@ -984,9 +1021,11 @@ template <bool PK, bool ST>
 static tg_status launch_round(const EatP &P, uint32_t S, uint32_t grid, cudaStream_t s, cudaEvent_t *tev) {
     if (tev) cudaEventRecord(tev[0], s);
     if (S == 1) TG_LAUNCH_RELAX((k_eat_activate1<PK, ST>), grid, QT, 0, s, P);
-    else TG_LAUNCH_RELAX((k_eat_activate<PK, ST>), grid, QT, 0, s, P);
+    else if (P.ub) TG_LAUNCH_RELAX((k_eat_activate<PK, ST, true>), grid, QT, 0, s, P);
+    else TG_LAUNCH_RELAX((k_eat_activate<PK, ST, false>), grid, QT, 0, s, P);
     if (tev) cudaEventRecord(tev[1], s);
-    TG_LAUNCH_RELAX((k_eat_big<PK, ST>), grid, QT, 0, s, P);
+    if (P.ub) TG_LAUNCH_RELAX((k_eat_big<PK, ST, true>), grid, QT, 0, s, P);
+    else TG_LAUNCH_RELAX((k_eat_big<PK, ST, false>), grid, QT, 0, s, P);
     if (tev) cudaEventRecord(tev[2], s);
     TG_LAUNCH_RELAX((k_eat_chain<PK, ST>), 148, QT, 0, s, P);  // at most a few hundred walks per round
     if (tev) cudaEventRecord(tev[3], s);
@@ -1022,10 +1061,15 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
         TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, Q.bit_words * 4, s));
     }
     const bool work = any_work && g->m > 0 && alpha < omega;
+    // arrival bounds: batches of 2 .. 64 queries (one u64 of 8 codes per vertex) whose
+    // state is far larger than the L2 (C4: 4.3 GB, job -3.4 %; C2's 256 MB: +3 %)
+    const bool ub = TG_UB && work && S > 1 && S <= 64 && !g->opt_stats &&
+                    (g->opt_ub == 1 ? (uint64_t)S * n * 4 >= (1ull << 30) : g->opt_ub == 2);
+    if (ub) TG_TRY_CUDA(cudaMemsetAsync(Q.ub, 0xFF, n * 8, s));
     TG_LAUNCH(k_eat_init<PK>, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
     *rounds_out = 0;
-    if (work) TG_TRY(eat_loop<PK>(g, cgr, S, alpha, omega, s, rounds_out));
+    if (work) TG_TRY(eat_loop<PK>(g, cgr, S, alpha, omega, s, rounds_out, ub));
     return TG_OK;
 }
 
@@ -1033,7 +1077,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
 // round control reset; stops at the first round whose frontier was empty.
 template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
-                          cudaStream_t s, uint32_t *rounds_out) {
+                          cudaStream_t s, uint32_t *rounds_out, bool ub) {
     QueryScratch &Q = g->qs;
     const uint32_t G = (S + 31) / 32;
     uint32_t rounds = 0;
@@ -1045,6 +1089,14 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
         P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
         P.ub0 = 0; P.ub1 = g->n * G;
+        if (ub) {
+            // codes over [alpha, min(omega, largest arrival)], where every state but INF
+            // lies: the smallest shift that maps the far end to <= 254
+            P.ub = Q.ub;
+            const uint32_t far = std::min(omega, g->max_arr);
+            const uint64_t span = far > alpha ? far - alpha : 0;
+            while (((span + (1ull << P.ub_sh) - 1) >> P.ub_sh) > 254) P.ub_sh++;
+        }
         P.use_sc = (int)g->opt_shortcuts; P.stats = (int)g->opt_stats;
         P.omega_all = omega > dir_max_t(g, cgr) ? 1 : 0;
         P.big_t = pick_big_t(g);

@@ -123,6 +123,7 @@ struct QueryScratch {
     void *st = nullptr;  // [n][S] packed u64 (time << 32 | pred), or u32 time when no pred is requested
     uint32_t st_copies = 1;  // option "exchange" with logical partitions: one private state copy each
     uint32_t *act = nullptr;           // [S][n] last activated time
+    unsigned long long *ub = nullptr;  // [n] arrival-bound codes per 8 queries (query_eat.cu, TG_UB)
     uint32_t stamp = 0;                // SP/FP frontier dedupe stamps handed out (host counter; marks start at 0)
     uint32_t *mark = nullptr;          // [S][n] (EAT) or [S][nnodes] (SP/FP) frontier dedupe stamp
     uint32_t *bits = nullptr;          // [S][ceil(m/32)] "slot relaxed" bits (interior slots of long chains)
@@ -241,6 +242,7 @@ struct tg_graph {
     int64_t opt_round_group = 8;  // GAC rounds launched per host convergence check
     int opt_mirror = 1;
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
+    int64_t opt_ub = 1;  // arrival bounds per (vertex, 8 queries) prune pairs: 0 off, 1 auto, 2 on (query_eat.cu)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
     int64_t opt_order_sources = 1;  // schedule a call's sources by first departure time (query_eat.cu)
     int64_t opt_reach_bits = 0;  // 1 = TG_REACH without pred on the bit-lane engine (query_reach.cu)

@@ -492,6 +492,34 @@ def test_unpacked_state_c2_small(tg):
         _check_values(tg, g, og, "ld", srcs[:16], win)
 
 
+@pytest.mark.parametrize("seed,sub_batch", [(0, 64), (1, 40), (2, 9), (3, 33)])
+def test_arrival_bound_filter_random(tg, seed, sub_batch):
+    """Option ub_filter=2 forces the per-(vertex, 8 queries) arrival bounds that prune
+    (edge, query) pairs (auto-enabled only for states >= 1 GiB): values and preds stay
+    equal to the oracle, with full and ragged 8-query blocks and one or two groups."""
+    n, u, v, t, lam, w = tgsynth.tiny_random(seed + 4100, n_max=120, m_max=3000, t_max=300, lam_max=9)
+    g = _gpu_graph(tg, n, u, v, t, lam, w, sub_batch=sub_batch, ub_filter=2)
+    og = oracle.Graph(n, u, v, t, lam, w)
+    srcs = [i % n for i in range(70)]
+    for win in [(0, 10**6), (20, 200), (7, 7)]:
+        _check_rows(tg, g, og, "eat", srcs, win)
+        _check_rows(tg, g, og, "ld", srcs[:24], win)
+        for p in ("eat", "ld", "reach"):
+            _check_values(tg, g, og, p, srcs, win)
+
+
+def test_arrival_bound_filter_c2_small(tg):
+    ge = tgsynth.make_graph("C2", scale_shift=-4)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, w, ub_filter=2)
+    og = oracle.Graph(n, u, v, t, d, w)
+    srcs = tgsynth.config_sources("C2", ge)
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        _check_values(tg, g, og, "eat", srcs, win)
+        _check_rows(tg, g, og, "eat", srcs[:8], win)
+        _check_values(tg, g, og, "ld", srcs[:16], win)
+
+
 # --------------------------------------------------------------------------- bit-lane reachability (f2)
 def _check_reach(tg, g, og, sources, win, host=False):
     import torch
