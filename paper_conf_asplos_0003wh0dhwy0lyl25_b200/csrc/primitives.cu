@@ -270,10 +270,10 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const unsigned lon
 template <int DB>
 tg_status radix_passes(unsigned long long *&ka, uint32_t *&va, unsigned long long *&kb, uint32_t *&vb, uint64_t m,
                        int key_bits, uint64_t ntiles, uint32_t *counts, cudaStream_t s, int snap_bits,
-                       uint32_t *snap_vals) {
+                       uint32_t *snap_vals, int begin_bit = 0) {
     TG_TRY_CUDA(cudaFuncSetAttribute(k_radix_scatter<DB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)rs_smem<DB>()));
-    for (int shift = 0; shift < key_bits; shift += DB) {
+    for (int shift = begin_bit; shift < begin_bit + key_bits; shift += DB) {
         TG_LAUNCH(k_radix_hist<DB>, (unsigned)ntiles, RS_THREADS, 0, s, ka, m, shift, counts, (uint32_t)ntiles);
         TG_TRY(tg_exclusive_scan_u32(counts, counts, ntiles << DB, nullptr, s, nullptr));
         TG_LAUNCH(k_radix_scatter<DB>, (unsigned)ntiles, RS_THREADS, rs_smem<DB>(), s, ka, va, kb, vb, m, shift,
@@ -296,9 +296,26 @@ tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t
 // As above; additionally, after the first `snap_bits` key bits have been sorted
 // (snap_bits a multiple of 8), the payload order of that intermediate state (stable
 // by the low snap_bits bits) is copied to snap_vals.
+static tg_status radix_sort_impl(unsigned long long *keys, uint32_t *vals, uint64_t m, int begin_bit, int key_bits,
+                                 unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s,
+                                 int snap_bits, uint32_t *snap_vals);
+
+tg_status tg_radix_sort_pairs_bits(unsigned long long *keys, uint32_t *vals, uint64_t m, int begin_bit, int key_bits,
+                                   cudaStream_t s) {
+    unsigned long long *sk;
+    uint32_t *sv;
+    return radix_sort_impl(keys, vals, m, begin_bit, key_bits, &sk, &sv, s, 0, nullptr);
+}
+
 tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
                                    unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s,
                                    int snap_bits, uint32_t *snap_vals) {
+    return radix_sort_impl(keys, vals, m, 0, key_bits, sorted_keys, sorted_vals, s, snap_bits, snap_vals);
+}
+
+static tg_status radix_sort_impl(unsigned long long *keys, uint32_t *vals, uint64_t m, int begin_bit, int key_bits,
+                                 unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s,
+                                 int snap_bits, uint32_t *snap_vals) {
     if (snap_vals && m >= 1 && (snap_bits <= 0 || m == 1 || key_bits <= 0))
         TG_TRY_CUDA(cudaMemcpyAsync(snap_vals, vals, m * 4, cudaMemcpyDeviceToDevice, s));
     *sorted_keys = keys;
@@ -326,9 +343,9 @@ tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uin
     TG_TRY_CUDA(tg_malloc_async((void **)&counts, (ntiles << db) * 4, s));
     unsigned long long *ka = keys, *kb = k2;
     uint32_t *va = vals, *vb = v2;
-    if (db == 10) TG_TRY((radix_passes<10>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals)));
-    else if (db == 9) TG_TRY((radix_passes<9>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals)));
-    else TG_TRY((radix_passes<8>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals)));
+    if (db == 10) TG_TRY((radix_passes<10>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals, begin_bit)));
+    else if (db == 9) TG_TRY((radix_passes<9>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals, begin_bit)));
+    else TG_TRY((radix_passes<8>(ka, va, kb, vb, m, key_bits, ntiles, counts, s, snap_bits, snap_vals, begin_bit)));
     TG_TRY_CUDA(cudaFreeAsync(counts, s));
     if (ka != keys) {
         // result lives in the scratch buffers: copy back so the caller's buffers hold it

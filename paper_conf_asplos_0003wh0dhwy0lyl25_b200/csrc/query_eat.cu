@@ -73,8 +73,12 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #define TG_COOP_SEARCH 1                // warp-cooperative departure-time search in the activation
 #endif
 #ifndef TG_UB
-#define TG_UB 1                         // per-(vertex, 8 queries) arrival bounds prune (edge, query) pairs
+#define TG_UB 1                         // per-(vertex, TG_UBQ queries) arrival bounds prune (edge, query) pairs
 #endif
+#ifndef TG_UBQ
+#define TG_UBQ 8                        // queries per arrival-bound code (8 or 4)
+#endif
+constexpr uint32_t UB_WORDS = TG_UBQ == 4 ? 2 : 1;  // u64 code words per vertex
 #ifndef TG_ACT_MINB
 #define TG_ACT_MINB 6                   // resident blocks per SM requested for the relax kernels (8, 7, 5, 4 measured slower)
 #endif
@@ -86,8 +90,8 @@ struct EatP {
     const uint2 *lc;
     const int4 *sc;
     void *st;  // [v * S + q]: packed u64 (arrival << 32 | pred) when PK, else u32 arrival
-    unsigned long long *ub;  // [v]: byte j = code of an upper bound of the arrivals of queries
-                             // 8j .. 8j+7 at v (255 = none); NULL = off (TG_UB)
+    unsigned long long *ub;  // [v * UB_WORDS]: byte j = code of an upper bound of the arrivals of
+                             // queries TG_UBQ j .. TG_UBQ (j + 1) - 1 at v (255 = none); NULL = off
     uint32_t ub_sh;          // code c <-> bound alpha + (c << ub_sh)
     uint32_t *act, *bits;
     uint32_t *touched;  // stats: slots relaxed by any query of the sub-batch
@@ -165,6 +169,15 @@ __device__ __forceinline__ typename StW<PK>::T st_load(const EatP &P, size_t i) 
     return ((const typename StW<PK>::T *)P.st)[i];
 }
 
+// work counters (stats only): relaxations per query, distinct slots of the sub-batch
+template <bool ST>
+__device__ __forceinline__ void eat_count(const EatP &P, uint32_t q, uint32_t slot) {
+    if (ST) {
+        atomicAdd(P.relax_cnt + q, 1ull);
+        atomicOr(P.touched + (slot >> 5), 1u << (slot & 31));
+    }
+}
+
 // Relax (v, q) with (arr, id) given a value `cur` read earlier from the state (any
 // earlier read: states only decrease, so a stale value is an upper bound and when it
 // is already <= the candidate the atomic cannot change anything -- most relaxations).
@@ -172,10 +185,7 @@ template <bool PK, bool ST>
 __device__ __forceinline__ void eat_relax_cur(const EatP &P, const RoundV &R, uint32_t q, uint32_t slot, uint32_t v,
                                               uint32_t arr, uint32_t id, typename StW<PK>::T cur) {
     using W = StW<PK>;
-    if (ST) {  // work counters: relaxations per query, distinct slots of the sub-batch
-        atomicAdd(P.relax_cnt + q, 1ull);
-        atomicOr(P.touched + (slot >> 5), 1u << (slot & 31));
-    }
+    eat_count<ST>(P, q, slot);
     const typename W::T pk = W::make(arr, id);
     if (cur <= pk) return;
     if (ST) atomicAdd(P.diag + 5, 1ull);  // relaxations past the filter read
@@ -287,7 +297,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
                     sl = make_int4((int)r.x, (int)r.y, 0, (int)TG_SINGLE);
                     if (ST) s = __ldg(P.occ_slot + p);  // distinct-slot counter
 #if TG_UB
-                    if (UB) ubw = __ldcg(P.ub + r.x);
+                    if (UB) ubw = __ldcg(P.ub + (size_t)r.x * UB_WORDS + (UB_WORDS == 2 ? g : 0));
 #endif
                 }
             }
@@ -302,7 +312,23 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         // code <= d  <=>  alpha + (code << sh) <= arrival - (PK ? 1 : 0); code 255 never is.
         if (UB && ubw != ~0ull) {
             const uint32_t d = min(254u, ((uint32_t)sl.y - P.alpha - (PK ? 1u : 0u)) >> P.ub_sh);
-            mask &= ~__vcmpleu4((uint32_t)(ubw >> (g * 32)), d * 0x01010101u);
+            uint32_t cut;
+            if (TG_UBQ == 8) {
+                cut = mask & __vcmpleu4((uint32_t)(ubw >> (g * 32)), d * 0x01010101u);
+            } else {  // 8 codes of 4 queries: byte flags -> nibbles
+                auto nib = [](uint32_t r) {
+                    r &= 0x0F0F0F0Fu;
+                    r = (r | (r >> 4)) & 0x00FF00FFu;
+                    return (r | (r >> 8)) & 0xFFFFu;
+                };
+                cut = mask & (nib(__vcmpleu4((uint32_t)ubw, d * 0x01010101u)) |
+                              nib(__vcmpleu4((uint32_t)(ubw >> 32), d * 0x01010101u)) << 16);
+            }
+            mask &= ~cut;
+            if (ST && cut) {  // the pruned pairs are relaxations too (first touch): count them
+                atomicAdd(P.diag + 6, (unsigned long long)__popc(cut));
+                for (uint32_t c = cut; c; c &= c - 1) eat_count<ST>(P, g * 32 + __ffs(c) - 1, s);
+            }
         }
 #endif
         const uint32_t cnt = __popc(mask);
@@ -433,8 +459,9 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
                 }
                 code = max(code, __shfl_xor_sync(0xffffffffu, code, 1));
                 code = max(code, __shfl_xor_sync(0xffffffffu, code, 2));
-                code = max(code, __shfl_xor_sync(0xffffffffu, code, 4));
-                if ((lane & 7) == 0) ((uint8_t *)(P.ub + v))[g * 4 + (lane >> 3)] = (uint8_t)code;
+                if (TG_UBQ == 8) code = max(code, __shfl_xor_sync(0xffffffffu, code, 4));
+                if ((lane & (TG_UBQ - 1)) == 0)
+                    ((uint8_t *)(P.ub + (size_t)v * UB_WORDS))[g * (32 / TG_UBQ) + lane / TG_UBQ] = (uint8_t)code;
                 if (on) prev = __ldcg(P.act + si);
             } else
 #endif
@@ -942,7 +969,7 @@ static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     Q.st_copies = copies;
     TG_TRY(A.alloc((void **)&Q.st, S * n * 8 * copies));
     TG_TRY(A.alloc((void **)&Q.act, S * n * 4));
-    if (TG_UB) TG_TRY(A.alloc((void **)&Q.ub, n * 8));
+    if (TG_UB) TG_TRY(A.alloc((void **)&Q.ub, n * 8 * UB_WORDS));
     Q.vwords = (uint32_t)((S + 31) / 32);  // query groups per vertex
     TG_TRY(A.alloc((void **)&Q.fb[0], n * Q.vwords * 4));
     TG_TRY(A.alloc((void **)&Q.fb[1], n * Q.vwords * 4));
@@ -1063,9 +1090,9 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     const bool work = any_work && g->m > 0 && alpha < omega;
     // arrival bounds: batches of 2 .. 64 queries (one u64 of 8 codes per vertex) whose
     // state is far larger than the L2 (C4: 4.3 GB, job -3.4 %; C2's 256 MB: +3 %)
-    const bool ub = TG_UB && work && S > 1 && S <= 64 && !g->opt_stats &&
+    const bool ub = TG_UB && work && S > 1 && S <= 64 &&
                     (g->opt_ub == 1 ? (uint64_t)S * n * 4 >= (1ull << 30) : g->opt_ub == 2);
-    if (ub) TG_TRY_CUDA(cudaMemsetAsync(Q.ub, 0xFF, n * 8, s));
+    if (ub) TG_TRY_CUDA(cudaMemsetAsync(Q.ub, 0xFF, n * 8 * UB_WORDS, s));
     TG_LAUNCH(k_eat_init<PK>, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
     *rounds_out = 0;
@@ -1248,8 +1275,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
             static const bool trace = getenv("TG_TRACE") != nullptr;
             if (trace)
                 fprintf(stderr, "[tg] diag S=%u: union edges %llu, unit ranges %llu, pairs %llu, activations %llu, "
-                        "frontier bits %llu, past filter %llu\n", Sb, h[Sb + 1], h[Sb + 2], h[Sb + 3], h[Sb + 4],
-                        h[Sb + 5], h[Sb + 6]);
+                        "frontier bits %llu, past filter %llu, pruned by bounds %llu\n", Sb, h[Sb + 1], h[Sb + 2], h[Sb + 3],
+                        h[Sb + 4], h[Sb + 5], h[Sb + 6], h[Sb + 7]);
         }
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));

@@ -273,6 +273,9 @@ tg_status tg_exclusive_scan_u32(const uint32_t *in, uint32_t *out, uint64_t coun
 // Stable LSD radix sort of (key, val) pairs on the low `key_bits` bits.
 tg_status tg_radix_sort_pairs(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
                               unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s);
+// Stable LSD radix sort in place on key bits [begin_bit, begin_bit + key_bits).
+tg_status tg_radix_sort_pairs_bits(unsigned long long *keys, uint32_t *vals, uint64_t m, int begin_bit, int key_bits,
+                                   cudaStream_t s);
 // ... and after the first snap_bits (multiple of 8) bits, a copy of the payload order to snap_vals.
 tg_status tg_radix_sort_pairs_snap(unsigned long long *keys, uint32_t *vals, uint64_t m, int key_bits,
                                    unsigned long long **sorted_keys, uint32_t **sorted_vals, cudaStream_t s,

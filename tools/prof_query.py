@@ -24,7 +24,12 @@ ap.add_argument("--shortcuts", type=int, default=1)
 ap.add_argument("--walk-min", type=int, default=0)
 ap.add_argument("--relabel", type=int, default=0)
 ap.add_argument("--stats", type=int, default=0)
+ap.add_argument("--lib", default="")
+ap.add_argument("--opt", action="append", default=[], help="key=value library option")
 a = ap.parse_args()
+if a.lib:
+    from paper_conf_asplos_0003wh0dhwy0lyl25_b200 import tempgraph as _T
+    _T.load_library(a.lib)
 
 ge = tgsynth.make_graph(a.config, device="cuda")
 cfg = tgsynth.CONFIGS[a.config]
@@ -40,6 +45,8 @@ if a.sub_batch:
     g.set_option("sub_batch", a.sub_batch)
 g.set_option("shortcuts", a.shortcuts)
 g.set_option("stats", a.stats)
+for kv in a.opt:
+    g.set_option(kv.split("=")[0], int(kv.split("=")[1]))
 src = tgsynth.config_sources(a.config, ge, k=a.k)
 win = cfg["windows"][0]
 out = torch.empty((len(src), ge.n), dtype=torch.int32, device="cuda")
