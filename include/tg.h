@@ -303,7 +303,10 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *                code of an upper bound of their arrivals, refreshed at activation, lets
  *                an edge skip the queries it cannot improve before any state read.
  *                0 = off, 1 (default) = on when the sub-batch state is >= 1 GiB, 2 = on.
- *                Results are identical either way. */
+ *                Results are identical either way.
+ *   "graph_loop" 1 (default) = EAT/LD/REACH GAC rounds run as one CUDA graph with a
+ *                conditional WHILE node (round number and stop test on the device);
+ *                0 = host-driven rounds checked every "round_group" rounds */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
 
 /* Total kernels this library has launched in this process (all handles). */

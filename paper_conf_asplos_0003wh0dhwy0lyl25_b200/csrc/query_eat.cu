@@ -35,6 +35,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 #include <vector>
 
 #include "tg_internal.cuh"
@@ -123,11 +124,14 @@ struct RoundV {
     uint32_t fin_n;
     uint32_t *fout;  // next round's frontier bitmap
     uint32_t *rec_cnt, *big_cnt, *ch_cnt, *words_cnt;
+    uint32_t r;      // this round
 };
 
 __device__ __forceinline__ RoundV round_view(const EatP &P) {
     RoundV R;
-    const uint32_t r = P.round;
+    // host-driven loops pass the round; the graph loop (P.round == 0) keeps it on the device
+    const uint32_t r = P.round ? P.round : *(volatile const uint32_t *)&P.ctl->round;
+    R.r = r;
     R.fin = (r & 1) ? P.fb1 : P.fb0;
     R.fout = (r & 1) ? P.fb0 : P.fb1;
     R.fin_n = 0;
@@ -141,8 +145,8 @@ __device__ __forceinline__ RoundV round_view(const EatP &P) {
 // Round r's counters were cleared during round r - 1: the first kernel of a round
 // clears the next round's (nobody touches them before that round; the host reads
 // only the last round of a group, which is cleared again three rounds later).
-__device__ __forceinline__ void clear_next_round(const EatP &P) {
-    if (blockIdx.x == 0 && threadIdx.x < 4) P.ctl->cnt[(P.round + 1) & (TG_RING - 1)][threadIdx.x] = 0;
+__device__ __forceinline__ void clear_next_round(const EatP &P, const RoundV &R) {
+    if (blockIdx.x == 0 && threadIdx.x < 4) P.ctl->cnt[(R.r + 1) & (TG_RING - 1)][threadIdx.x] = 0;
 }
 
 // Layouts interleave the S queries of a sub-batch (query index fastest):
@@ -397,7 +401,7 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
 template <bool PK, bool ST, bool UB>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
     const RoundV R = round_view(P);
-    clear_next_round(P);
+    clear_next_round(P, R);
     __shared__ WarpStage stage[QT / 32];
     WarpStage &ws = stage[threadIdx.x >> 5];
     uint32_t my_units = 0;
@@ -415,7 +419,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         // experiment: a unit with few new queries in a bulk round waits one round (its
         // word moves to the next frontier) so that more of its group's queries share one
         // scan of its edges; a unit is deferred at most once in a row
-        if (word && P.defer && P.S >= 64 && P.round >= TG_DEFER_FROM) {  // full sub-batches only
+        if (word && P.defer && P.S >= 64 && R.r >= TG_DEFER_FROM) {  // full sub-batches only
             const uint32_t bit = 1u << (ui & 31);
             uint32_t *dw = P.defer + (ui >> 5);
             if (__popc(word) < TG_DEFER) {
@@ -547,7 +551,7 @@ constexpr uint32_t LANE_SEARCH_MAX = 64;  // departure nodes a lane searches alo
 template <bool PK, bool ST>
 __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate1(EatP P) {
     const RoundV R = round_view(P);
-    clear_next_round(P);
+    clear_next_round(P, R);
     uint32_t my_units = 0;
     const uint32_t NU = P.ub1;
     const int lane = threadIdx.x & 31;
@@ -946,7 +950,27 @@ __global__ void k_ctl_reset(RoundCtl *ctl) {
     ctl->stamp = ctl->stamp + 1;
 }
 
+// Graph loop: ends a round.  The loop's WHILE condition drops to 0 after the first round
+// whose activation consumed no frontier word (it did no work), or at the round limit.
+__global__ void k_round_next(RoundCtl *ctl, cudaGraphConditionalHandle h, uint32_t limit) {
+    if (threadIdx.x != 0) return;
+    const uint32_t r = ctl->round;
+    if (ctl->cnt[r & (TG_RING - 1)][3] == 0 || r >= limit) {
+        ctl->last = r;
+        cudaGraphSetConditional(h, 0);
+    } else {
+        ctl->round = r + 1;
+    }
+}
+
 }  // namespace
+
+void tg_round_graph_free(tg_graph *g) {
+    auto &G = g->rgraph;
+    if (G.exec) cudaGraphExecDestroy(G.exec);
+    if (G.graph) cudaGraphDestroy(G.graph);
+    G = tg_graph::RoundGraph{};
+}
 
 static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
     QueryScratch &Q = g->qs;
@@ -1070,6 +1094,78 @@ static uint32_t dir_max_t(const tg_graph *g, const ChainGraph &cg) {
     return (&cg == &g->mir || (g->nparts && &cg >= g->pm && &cg < g->pm + TG_MAXP)) ? g->max_arr - g->min_t : g->max_t;
 }
 
+// The GAC rounds as one CUDA graph: a conditional WHILE node whose body is one round
+// (activate, big, chain) plus k_round_next, which keeps the round number on the device
+// and ends the loop at the first empty round -- no host check every few rounds, no
+// rounds launched past convergence.  The instantiation is cached on the handle, keyed
+// by the kernel parameters (one per sub-batch shape; a job's sub-batches share it).
+template <bool PK>
+static tg_status graph_rounds(tg_graph *g, EatP P, uint32_t S, uint32_t grid, cudaStream_t s, uint32_t *rounds) {
+    QueryScratch &Q = g->qs;
+    constexpr uint32_t LIMIT = 1000000;
+    P.round = 0;  // device-side round (RoundCtl::round, reset by k_eat_init / k_ctl_reset)
+    auto &RG = g->rgraph;
+    // the key: everything the captured launches depend on (parameters, shape, state width)
+    unsigned char key[sizeof(EatP) + 9];
+    static_assert(sizeof(key) <= sizeof(RG.key), "round-graph key");
+    std::memcpy(key, &P, sizeof(EatP));
+    std::memcpy(key + sizeof(EatP), &S, 4);
+    std::memcpy(key + sizeof(EatP) + 4, &grid, 4);
+    key[sizeof(EatP) + 8] = PK ? 1 : 0;
+    if (!RG.exec || RG.key_len != sizeof(key) || std::memcmp(RG.key, key, sizeof(key)) != 0) {
+        tg_round_graph_free(g);
+        TG_TRY_CUDA(cudaGraphCreate(&RG.graph, 0));
+        cudaGraphConditionalHandle h;
+        TG_TRY_CUDA(cudaGraphConditionalHandleCreate(&h, RG.graph, 1, cudaGraphCondAssignDefault));
+        cudaGraphNodeParams cp = {};
+        cp.type = cudaGraphNodeTypeConditional;
+        cp.conditional.handle = h;
+        cp.conditional.type = cudaGraphCondTypeWhile;
+        cp.conditional.size = 1;
+        cudaGraphNode_t node;
+        TG_TRY_CUDA(cudaGraphAddNode(&node, RG.graph, nullptr, 0, &cp));
+        cudaGraph_t body = cp.conditional.phGraph_out[0];
+        cudaStream_t cs;  // capture needs a non-legacy stream
+        TG_TRY_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+        cudaError_t e = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
+        tg_status st = TG_OK;
+        if (e == cudaSuccess) {
+            const int prof = g_tg_profile;
+            const uint64_t l0 = g_tg_launches;
+            g_tg_profile = 0;  // no event records inside the body
+            st = launch_round<PK, false>(P, S, grid, cs, nullptr);
+            if (st == TG_OK) k_round_next<<<1, 32, 0, cs>>>(Q.ctl, h, LIMIT);
+            g_tg_profile = prof;
+            g_tg_launches = l0;  // counted per executed round below
+            cudaGraph_t out = nullptr;
+            const cudaError_t e2 = cudaStreamEndCapture(cs, &out);
+            if (e == cudaSuccess) e = e2;
+            if (e == cudaSuccess) e = cudaGetLastError();
+        }
+        cudaStreamDestroy(cs);
+        if (st != TG_OK) { tg_round_graph_free(g); return st; }
+        if (e == cudaSuccess) e = cudaGraphInstantiate(&RG.exec, RG.graph, 0);
+        if (e != cudaSuccess) {
+            tg_round_graph_free(g);
+            tg_set_error(std::string("round graph: ") + cudaGetErrorString(e));
+            return TG_ERR_CUDA;
+        }
+        std::memcpy(RG.key, key, sizeof(key));
+        RG.key_len = sizeof(key);
+    }
+    cudaEvent_t ev0 = (g_tg_profile && g_tg_profile <= 2) ? tg_prof_begin(s) : nullptr;
+    TG_TRY_CUDA(cudaGraphLaunch(RG.exec, s));
+    if (ev0) tg_prof_end("k_eat_rounds (graph loop: k_eat_activate + k_eat_big + k_eat_chain per round)", s, ev0);
+    TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    const RoundCtl *hc = (const RoundCtl *)Q.h_ctr;
+    const uint32_t last = hc->last;
+    g_tg_launches += 4ull * last;  // activate, big, chain, k_round_next per executed round
+    if (hc->cnt[last & (TG_RING - 1)][3] != 0) { tg_set_error("GAC rounds did not converge"); return TG_ERR_CUDA; }
+    *rounds = last - 1;  // the last round had an empty frontier
+    return TG_OK;
+}
+
 // Run the GAC rounds of one sub-batch on direction cg; returns rounds used.
 template <bool PK>
 static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
@@ -1134,6 +1230,10 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.diag = Q.relax_cnt + S + 1;
         const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;
+        if (g->opt_graph_loop && !trace && !P.stats) {
+            TG_TRY(graph_rounds<PK>(g, P, S, grid, s, rounds_out));
+            return TG_OK;
+        }
         const int group = trace ? 1 : (int)std::max<int64_t>(1, g->opt_round_group);
         cudaEvent_t tev[4] = {};
         if (trace)

@@ -110,7 +110,7 @@ struct RoundCtl {
     uint32_t round;
     uint32_t stamp;
     uint32_t done_blocks;
-    uint32_t pad;
+    uint32_t last;  // graph loop: the round that ended it (its frontier was empty, or the limit)
     uint32_t cnt[TG_RING][4];
 };
 
@@ -232,6 +232,14 @@ struct tg_graph {
     int comm_mode = 0;              // 0 replicated (source sharding), 1 vertex range
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
+    // EAT-family round loop captured as a CUDA graph with a conditional WHILE node
+    // (query_eat.cu): the last instantiation, keyed by its kernel parameters
+    struct RoundGraph {
+        cudaGraphExec_t exec = nullptr;
+        cudaGraph_t graph = nullptr;
+        unsigned char key[512] = {};
+        size_t key_len = 0;
+    } rgraph;
     ReachScratch rs;
     StreamGraph *stream = nullptr;  // out-of-memory graph (tg_graph_create_streamed)
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
@@ -243,6 +251,7 @@ struct tg_graph {
     int opt_mirror = 1;
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
     int64_t opt_ub = 1;  // arrival bounds per (vertex, 8 queries) prune pairs: 0 off, 1 auto, 2 on (query_eat.cu)
+    int64_t opt_graph_loop = 1;  // 1 = GAC rounds run in a device-driven CUDA-graph WHILE loop (query_eat.cu)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
     int64_t opt_order_sources = 1;  // schedule a call's sources by first departure time (query_eat.cu)
     int64_t opt_reach_bits = 0;  // 1 = TG_REACH without pred on the bit-lane engine (query_reach.cu)
@@ -296,6 +305,7 @@ tg_status tg_validate_launch(const uint32_t *u, const uint32_t *v, const uint32_
 tg_status tg_validate_finish(tg_graph *g, const uint32_t *h);  // h: the 5 accumulated words
 tg_status tg_build_streamed(tg_graph *g);
 void tg_stream_free(tg_graph *g);
+void tg_round_graph_free(tg_graph *g);  // query_eat.cu: the cached round-loop graph
 tg_status tg_run_eat_streamed(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                               uint32_t *pred, bool out_dev, bool pred_dev, int mode, cudaStream_t s);
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,

@@ -520,6 +520,29 @@ def test_arrival_bound_filter_c2_small(tg):
         _check_values(tg, g, og, "ld", srcs[:16], win)
 
 
+@pytest.mark.parametrize("graph_loop", [0, 1])
+def test_round_loop_modes(tg, graph_loop):
+    """GAC rounds driven by the host (checks every round_group rounds) or by the device in
+    a CUDA-graph WHILE loop (the default): same rows, preds, and round counts; packed and
+    u32 states alternate on one handle (the cached loop graph is keyed by the state width)."""
+    ge = tgsynth.make_graph("C2", scale_shift=-5)
+    n, u, v, t, d, w = ge.numpy()
+    g = _gpu_graph(tg, n, u, v, t, d, graph_loop=graph_loop)
+    og = oracle.Graph(n, u, v, t, d)
+    srcs = tgsynth.config_sources("C2", ge, k=40)
+    rounds = []
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        for p in ("eat", "ld"):
+            _check_rows(tg, g, og, p, srcs, win)
+            rounds.append(g.last_stats()["rounds"])
+            _check_values(tg, g, og, p, srcs, win)
+    g2 = _gpu_graph(tg, n, u, v, t, d, graph_loop=1 - graph_loop)
+    for i, win in enumerate(tgsynth.CONFIGS["C2"]["windows"]):
+        for j, p in enumerate(("eat", "ld")):
+            g2.query(p, srcs, win, with_pred=True)
+            assert g2.last_stats()["rounds"] == rounds[2 * i + j]
+
+
 # --------------------------------------------------------------------------- bit-lane reachability (f2)
 def _check_reach(tg, g, og, sources, win, host=False):
     import torch
