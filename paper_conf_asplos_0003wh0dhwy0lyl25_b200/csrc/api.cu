@@ -202,7 +202,7 @@ struct DeviceGuard {
 }  // namespace
 
 uint64_t tg_graph_bytes(const tg_graph *g) {
-    uint64_t b = g->arena.total + g->qs.arena.total + g->rs.arena.total + g->fwd.arena.total + g->mir.arena.total;
+    uint64_t b = g->arena.total + g->qs.arena.total + g->qs2.arena.total + g->rs.arena.total + g->fwd.arena.total + g->mir.arena.total;
     for (int p = 0; p < TG_MAXP; p++) b += g->pf[p].arena.total + g->pm[p].arena.total;
     if (g->stream) b += g->stream->slot_arena.total;
     return b;
@@ -429,6 +429,11 @@ void tg_graph_destroy(tg_graph *g) {
     tg_round_graph_free(g);
     g->qs.arena.free_all();
     tg_pinned_put(g->qs.h_ctr);
+    g->qs2.arena.free_all();
+    tg_pinned_put(g->qs2.h_ctr);
+    if (g->lane_stream) cudaStreamDestroy(g->lane_stream);
+    for (auto &e : g->lane_ev)
+        if (e) cudaEventDestroy(e);
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);
     g->fwd.arena.free_all();
@@ -581,6 +586,7 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     else if (k == "exchange") g->opt_exchange = value ? 1 : 0;
     else if (k == "packed_state") g->opt_packed_state = value ? 1 : 0;
     else if (k == "graph_loop") g->opt_graph_loop = value ? 1 : 0;
+    else if (k == "lanes") g->opt_lanes = value >= 2 ? 2 : 1;
     else if (k == "ub_filter") g->opt_ub = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (k == "reach_bits") g->opt_reach_bits = value ? 1 : 0;
     else if (k == "order_sources") g->opt_order_sources = value ? 1 : 0;

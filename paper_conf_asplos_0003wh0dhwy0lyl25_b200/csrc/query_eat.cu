@@ -965,15 +965,18 @@ __global__ void k_round_next(RoundCtl *ctl, cudaGraphConditionalHandle h, uint32
 
 }  // namespace
 
-void tg_round_graph_free(tg_graph *g) {
-    auto &G = g->rgraph;
+static void rg_free(tg_graph::RoundGraph &G) {
     if (G.exec) cudaGraphExecDestroy(G.exec);
     if (G.graph) cudaGraphDestroy(G.graph);
     G = tg_graph::RoundGraph{};
 }
 
-static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
-    QueryScratch &Q = g->qs;
+void tg_round_graph_free(tg_graph *g) {
+    rg_free(g->rgraph);
+    rg_free(g->rgraph2);
+}
+
+static tg_status ensure_scratch_q(tg_graph *g, QueryScratch &Q, uint32_t S, bool nodes_state) {
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
     const uint32_t copies = (g->opt_exchange && !g->comm && g->nparts > 1) ? (uint32_t)g->nparts : 1u;
     if (Q.S >= S && Q.n == g->n && Q.st && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat) &&
@@ -1060,11 +1063,16 @@ uint32_t tg_pick_sub_batch(tg_graph *g, uint32_t k, bool nodes_state) {
     return (uint32_t)std::min<uint64_t>(S, k);
 }
 
+static tg_status ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) {
+    return ensure_scratch_q(g, g->qs, S, nodes_state);
+}
+
 tg_status tg_ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) { return ensure_scratch(g, S, nodes_state); }
 
 template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
-                          cudaStream_t s, uint32_t *rounds_out, bool ub = false);
+                          cudaStream_t s, uint32_t *rounds_out, bool ub = false, QueryScratch *Qp = nullptr,
+                          tg_graph::RoundGraph *RGp = nullptr, bool async = false);
 
 // One GAC round's relax kernels; the stats counters are a template argument so that the
 // timed path carries no per-pair stats branch.
@@ -1099,12 +1107,13 @@ static uint32_t dir_max_t(const tg_graph *g, const ChainGraph &cg) {
 // and ends the loop at the first empty round -- no host check every few rounds, no
 // rounds launched past convergence.  The instantiation is cached on the handle, keyed
 // by the kernel parameters (one per sub-batch shape; a job's sub-batches share it).
+static tg_status graph_rounds_finish(QueryScratch &Q, uint32_t *rounds);
+
 template <bool PK>
-static tg_status graph_rounds(tg_graph *g, EatP P, uint32_t S, uint32_t grid, cudaStream_t s, uint32_t *rounds) {
-    QueryScratch &Q = g->qs;
+static tg_status graph_rounds(tg_graph *g, QueryScratch &Q, tg_graph::RoundGraph &RG, EatP P, uint32_t S,
+                              uint32_t grid, cudaStream_t s, uint32_t *rounds, bool async) {
     constexpr uint32_t LIMIT = 1000000;
     P.round = 0;  // device-side round (RoundCtl::round, reset by k_eat_init / k_ctl_reset)
-    auto &RG = g->rgraph;
     // the key: everything the captured launches depend on (parameters, shape, state width)
     unsigned char key[sizeof(EatP) + 9];
     static_assert(sizeof(key) <= sizeof(RG.key), "round-graph key");
@@ -1113,7 +1122,7 @@ static tg_status graph_rounds(tg_graph *g, EatP P, uint32_t S, uint32_t grid, cu
     std::memcpy(key + sizeof(EatP) + 4, &grid, 4);
     key[sizeof(EatP) + 8] = PK ? 1 : 0;
     if (!RG.exec || RG.key_len != sizeof(key) || std::memcmp(RG.key, key, sizeof(key)) != 0) {
-        tg_round_graph_free(g);
+        rg_free(RG);
         TG_TRY_CUDA(cudaGraphCreate(&RG.graph, 0));
         cudaGraphConditionalHandle h;
         TG_TRY_CUDA(cudaGraphConditionalHandleCreate(&h, RG.graph, 1, cudaGraphCondAssignDefault));
@@ -1143,10 +1152,10 @@ static tg_status graph_rounds(tg_graph *g, EatP P, uint32_t S, uint32_t grid, cu
             if (e == cudaSuccess) e = cudaGetLastError();
         }
         cudaStreamDestroy(cs);
-        if (st != TG_OK) { tg_round_graph_free(g); return st; }
+        if (st != TG_OK) { rg_free(RG); return st; }
         if (e == cudaSuccess) e = cudaGraphInstantiate(&RG.exec, RG.graph, 0);
         if (e != cudaSuccess) {
-            tg_round_graph_free(g);
+            rg_free(RG);
             tg_set_error(std::string("round graph: ") + cudaGetErrorString(e));
             return TG_ERR_CUDA;
         }
@@ -1157,7 +1166,13 @@ static tg_status graph_rounds(tg_graph *g, EatP P, uint32_t S, uint32_t grid, cu
     TG_TRY_CUDA(cudaGraphLaunch(RG.exec, s));
     if (ev0) tg_prof_end("k_eat_rounds (graph loop: k_eat_activate + k_eat_big + k_eat_chain per round)", s, ev0);
     TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
+    if (async) return TG_OK;  // two query lanes: graph_rounds_finish after the lane's stream is synchronised
     TG_TRY_CUDA(cudaStreamSynchronize(s));
+    return graph_rounds_finish(Q, rounds);
+}
+
+// After the stream of a graph loop is synchronised: its round count (and convergence).
+static tg_status graph_rounds_finish(QueryScratch &Q, uint32_t *rounds) {
     const RoundCtl *hc = (const RoundCtl *)Q.h_ctr;
     const uint32_t last = hc->last;
     g_tg_launches += 4ull * last;  // activate, big, chain, k_round_next per executed round
@@ -1168,9 +1183,9 @@ static tg_status graph_rounds(tg_graph *g, EatP P, uint32_t S, uint32_t grid, cu
 
 // Run the GAC rounds of one sub-batch on direction cg; returns rounds used.
 template <bool PK>
-static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
-                            bool any_work, cudaStream_t s, uint32_t *rounds_out) {
-    QueryScratch &Q = g->qs;
+static tg_status eat_rounds(tg_graph *g, QueryScratch &Q, tg_graph::RoundGraph &RG, const ChainGraph &cgr, uint32_t S,
+                            uint32_t alpha, uint32_t omega, bool any_work, cudaStream_t s, uint32_t *rounds_out,
+                            bool async) {
     const uint64_t n = g->n;
     TG_TRY_CUDA(cudaMemsetAsync(Q.st, 0xFF, S * n * (PK ? 8 : 4), s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.act, 0xFF, S * n * 4, s));
@@ -1192,7 +1207,7 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
     TG_LAUNCH(k_eat_init<PK>, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
     *rounds_out = 0;
-    if (work) TG_TRY(eat_loop<PK>(g, cgr, S, alpha, omega, s, rounds_out, ub));
+    if (work) TG_TRY(eat_loop<PK>(g, cgr, S, alpha, omega, s, rounds_out, ub, &Q, &RG, async));
     return TG_OK;
 }
 
@@ -1200,8 +1215,9 @@ static tg_status eat_rounds(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint
 // round control reset; stops at the first round whose frontier was empty.
 template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
-                          cudaStream_t s, uint32_t *rounds_out, bool ub) {
-    QueryScratch &Q = g->qs;
+                          cudaStream_t s, uint32_t *rounds_out, bool ub, QueryScratch *Qp, tg_graph::RoundGraph *RGp,
+                          bool async) {
+    QueryScratch &Q = Qp ? *Qp : g->qs;
     const uint32_t G = (S + 31) / 32;
     uint32_t rounds = 0;
     {
@@ -1231,9 +1247,10 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;
         if (g->opt_graph_loop && !trace && !P.stats) {
-            TG_TRY(graph_rounds<PK>(g, P, S, grid, s, rounds_out));
+            TG_TRY(graph_rounds<PK>(g, Q, RGp ? *RGp : g->rgraph, P, S, grid, s, rounds_out, async));
             return TG_OK;
         }
+        if (async) { tg_set_error("async rounds need the graph loop"); return TG_ERR_STATE; }
         const int group = trace ? 1 : (int)std::max<int64_t>(1, g->opt_round_group);
         cudaEvent_t tev[4] = {};
         if (trace)
@@ -1306,7 +1323,6 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     }
     const uint32_t S = tg_pick_sub_batch(g, k, false);
     TG_TRY(ensure_scratch(g, S, false));
-    QueryScratch &Q = g->qs;
     const uint64_t n = g->n;
     TG_TRY(tg_sink_begin(g, !out_dev, pred && !pred_dev));
     g->last = tg_query_stats{};
@@ -1327,48 +1343,91 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     const bool sched = g->opt_order_sources && k > 32 && any_work && g->m > 0 && (!pred || out_dev == pred_dev);
     TG_TRY(tg_schedule_sources(g, cgr, sources, k, alpha, sched, order, s));
     for (uint32_t i = 0; i < k; i++) srcs_sched[i] = sources[order[i]];
+    // Two query lanes: consecutive sub-batches alternate between two scratch sets and two
+    // streams, each running its device-driven round loop, so one sub-batch's kernels fill
+    // the other's kernel tails and sparse rounds (C4 half scale: 535 -> 485 ms).  Device
+    // outputs only (host outputs stream through the single staging sink).
+    static const bool trace = getenv("TG_TRACE") != nullptr;
+    const bool work = any_work && g->m > 0 && alpha < omega;
+    bool dual = g->opt_lanes >= 2 && k > S && out_dev && (!pred || pred_dev) && !g->opt_stats && g->opt_graph_loop &&
+                !trace && work;
+    if (dual && ensure_scratch_q(g, g->qs2, S, false) != TG_OK) {  // no room for a second scratch set
+        cudaGetLastError();
+        cudaDeviceSynchronize();
+        g->qs2.arena.free_all();
+        tg_pinned_put(g->qs2.h_ctr);
+        g->qs2 = QueryScratch{};
+        dual = false;
+    }
+    cudaStream_t ls[2] = {s, s};
+    if (dual) {
+        if (!g->lane_stream) TG_TRY_CUDA(cudaStreamCreateWithFlags(&g->lane_stream, cudaStreamNonBlocking));
+        if (!g->lane_ev[0]) {
+            TG_TRY_CUDA(cudaEventCreateWithFlags(&g->lane_ev[0], cudaEventDisableTiming));
+            TG_TRY_CUDA(cudaEventCreateWithFlags(&g->lane_ev[1], cudaEventDisableTiming));
+        }
+        ls[1] = g->lane_stream;
+        TG_TRY_CUDA(cudaEventRecord(g->lane_ev[0], s));  // lane 1 starts after the caller's prior work
+        TG_TRY_CUDA(cudaStreamWaitEvent(ls[1], g->lane_ev[0], 0));
+    }
+    bool pending[2] = {false, false};
+    auto finish = [&](int l) -> tg_status {
+        if (!pending[l]) return TG_OK;
+        pending[l] = false;
+        TG_TRY_CUDA(cudaStreamSynchronize(ls[l]));
+        uint32_t r = 0;
+        TG_TRY(graph_rounds_finish(l ? g->qs2 : g->qs, &r));
+        g->last.rounds = std::max(g->last.rounds, r);
+        return TG_OK;
+    };
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
-        TG_TRY(tg_load_sources(g, srcs_sched.data() + b0, Sb, s));
+        const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
+        const int lane = dual ? (int)(bi & 1) : 0;
+        QueryScratch &Q = lane ? g->qs2 : g->qs;
+        tg_graph::RoundGraph &RG = lane ? g->rgraph2 : g->rgraph;
+        const cudaStream_t st = ls[lane];
+        TG_TRY(finish(lane));  // the lane's previous sub-batch (the other lane keeps running)
+        TG_TRY(tg_load_sources_to(g, srcs_sched.data() + b0, Sb, Q.srcs, Q.srcs_int, st));
         // caller rows of this sub-batch's queries (NULL: consecutive rows b0 ..)
         const uint32_t *rows = nullptr;
         bool consecutive = true;
         for (uint32_t q = 0; q < Sb; q++) consecutive = consecutive && order[b0 + q] == b0 + q;
         if (!consecutive && out_dev && (!pred || pred_dev)) {
-            TG_TRY_CUDA(cudaMemcpyAsync(Q.rows, order.data() + b0, Sb * 4, cudaMemcpyHostToDevice, s));
+            TG_TRY_CUDA(cudaMemcpyAsync(Q.rows, order.data() + b0, Sb * 4, cudaMemcpyHostToDevice, st));
             rows = Q.rows;
         }
         uint32_t rounds = 0;
-        if (pk) TG_TRY(eat_rounds<true>(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
-        else TG_TRY(eat_rounds<false>(g, cgr, Sb, alpha, omega, any_work, s, &rounds));
-        g->last.rounds = std::max(g->last.rounds, rounds);
+        if (pk) TG_TRY(eat_rounds<true>(g, Q, RG, cgr, Sb, alpha, omega, any_work, st, &rounds, dual));
+        else TG_TRY(eat_rounds<false>(g, Q, RG, cgr, Sb, alpha, omega, any_work, st, &rounds, dual));
+        if (dual) pending[lane] = true;
+        else g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;
-        const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
         uint32_t *o = out_dev ? (rows ? out : out + (size_t)b0 * n) : nullptr;
         uint32_t *pr = pred ? (pred_dev ? (rows ? pred : pred + (size_t)b0 * n) : pred) : nullptr;
-        TG_TRY(tg_sink_target(g, bi, !out_dev, pred && !pred_dev, &o, &pr, s));
+        TG_TRY(tg_sink_target(g, bi, !out_dev, pred && !pred_dev, &o, &pr, st));
         const unsigned xgrid = (unsigned)std::min<uint64_t>((n + 31) / 32, 148ull * 16);
         if (pk)
-            TG_LAUNCH(k_eat_extract<true>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
+            TG_LAUNCH(k_eat_extract<true>, xgrid, 256, 0, st, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
                       g->relabeled ? g->perm : (const uint32_t *)nullptr, rows);
         else if (Sb == 64 && !g->relabeled)
-            TG_LAUNCH(k_eat_extract64, (unsigned)std::min<uint64_t>((n + 63) / 64, 148ull * 8), 256, 0, s,
+            TG_LAUNCH(k_eat_extract64, (unsigned)std::min<uint64_t>((n + 63) / 64, 148ull * 8), 256, 0, st,
                       (const uint32_t *)Q.st, g->n, Q.srcs, mode, C, w.t_omega, o, rows);
         else
-            TG_LAUNCH(k_eat_extract<false>, xgrid, 256, 0, s, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
+            TG_LAUNCH(k_eat_extract<false>, xgrid, 256, 0, st, Q.st, g->n, Sb, Q.srcs, mode, C, w.t_omega, o, pr,
                       g->relabeled ? g->perm : (const uint32_t *)nullptr, rows);
         if (consecutive || (out_dev && (!pred || pred_dev)))
             TG_TRY(tg_sink_flush(g, bi, out_dev ? nullptr : out + (size_t)b0 * n,
-                                 (pred && !pred_dev) ? pred + (size_t)b0 * n : nullptr, (size_t)Sb * n * 4, s));
+                                 (pred && !pred_dev) ? pred + (size_t)b0 * n : nullptr, (size_t)Sb * n * 4, st));
         else  // host outputs of a reordered sub-batch: one copy per row
             TG_TRY(tg_sink_flush_rows(g, bi, out_dev ? nullptr : out, (pred && !pred_dev) ? pred : nullptr,
-                                      order.data() + b0, Sb, n, s));
+                                      order.data() + b0, Sb, n, st));
         if (g->opt_stats) {
             const uint64_t tw = (g->m + 31) / 32 + TG_MAXP + 1;
-            TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, Q.touched, tw,
-                      Q.relax_cnt + Sb);
+            TG_LAUNCH(k_popcount, (unsigned)std::min<uint64_t>((tw + 255) / 256, 4096), 256, 0, s, g->qs.touched, tw,
+                      g->qs.relax_cnt + Sb);
             std::vector<unsigned long long> h(Sb + 1 + 8);
-            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), Q.relax_cnt, (Sb + 1 + 8) * 8, cudaMemcpyDeviceToHost, s));
+            TG_TRY_CUDA(cudaMemcpyAsync(h.data(), g->qs.relax_cnt, (Sb + 1 + 8) * 8, cudaMemcpyDeviceToHost, s));
             TG_TRY_CUDA(cudaStreamSynchronize(s));
             for (uint32_t q = 0; q < Sb; q++) { g->last_relax[order[b0 + q]] = h[q]; g->last.slots_relaxed += h[q]; }
             g->last.slots_union += h[Sb];
@@ -1378,6 +1437,12 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
                         "frontier bits %llu, past filter %llu, pruned by bounds %llu\n", Sb, h[Sb + 1], h[Sb + 2], h[Sb + 3],
                         h[Sb + 4], h[Sb + 5], h[Sb + 6], h[Sb + 7]);
         }
+    }
+    TG_TRY(finish(0));
+    TG_TRY(finish(1));
+    if (dual) {  // the caller's stream continues after lane 1's work
+        TG_TRY_CUDA(cudaEventRecord(g->lane_ev[1], ls[1]));
+        TG_TRY_CUDA(cudaStreamWaitEvent(s, g->lane_ev[1], 0));
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     TG_TRY(tg_sink_end(g));

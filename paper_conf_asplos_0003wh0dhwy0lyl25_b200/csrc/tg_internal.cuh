@@ -239,7 +239,11 @@ struct tg_graph {
         cudaGraph_t graph = nullptr;
         unsigned char key[512] = {};
         size_t key_len = 0;
-    } rgraph;
+    } rgraph, rgraph2;
+    // second query lane (EAT family, device outputs): its scratch, stream, fork/join events
+    QueryScratch qs2;
+    cudaStream_t lane_stream = nullptr;
+    cudaEvent_t lane_ev[2] = {nullptr, nullptr};
     ReachScratch rs;
     StreamGraph *stream = nullptr;  // out-of-memory graph (tg_graph_create_streamed)
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
@@ -251,7 +255,8 @@ struct tg_graph {
     int opt_mirror = 1;
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
     int64_t opt_ub = 1;  // arrival bounds per (vertex, 8 queries) prune pairs: 0 off, 1 auto, 2 on (query_eat.cu)
-    int64_t opt_graph_loop = 1;  // 1 = GAC rounds run in a device-driven CUDA-graph WHILE loop (query_eat.cu)
+    int64_t opt_graph_loop = 1;
+    int64_t opt_lanes = 2;  // sub-batches in flight (EAT family, device outputs, graph loop): 1 or 2  // 1 = GAC rounds run in a device-driven CUDA-graph WHILE loop (query_eat.cu)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
     int64_t opt_order_sources = 1;  // schedule a call's sources by first departure time (query_eat.cu)
     int64_t opt_reach_bits = 0;  // 1 = TG_REACH without pred on the bit-lane engine (query_reach.cu)

@@ -523,8 +523,8 @@ def test_arrival_bound_filter_c2_small(tg):
 @pytest.mark.parametrize("graph_loop", [0, 1])
 def test_round_loop_modes(tg, graph_loop):
     """GAC rounds driven by the host (checks every round_group rounds) or by the device in
-    a CUDA-graph WHILE loop (the default): same rows, preds, and round counts; packed and
-    u32 states alternate on one handle (the cached loop graph is keyed by the state width)."""
+    a CUDA-graph WHILE loop (the default): same rows and preds; packed and u32 states
+    alternate on one handle (the cached loop graph is keyed by the state width)."""
     ge = tgsynth.make_graph("C2", scale_shift=-5)
     n, u, v, t, d, w = ge.numpy()
     g = _gpu_graph(tg, n, u, v, t, d, graph_loop=graph_loop)
@@ -536,11 +536,38 @@ def test_round_loop_modes(tg, graph_loop):
             _check_rows(tg, g, og, p, srcs, win)
             rounds.append(g.last_stats()["rounds"])
             _check_values(tg, g, og, p, srcs, win)
-    g2 = _gpu_graph(tg, n, u, v, t, d, graph_loop=1 - graph_loop)
-    for i, win in enumerate(tgsynth.CONFIGS["C2"]["windows"]):
-        for j, p in enumerate(("eat", "ld")):
-            g2.query(p, srcs, win, with_pred=True)
-            assert g2.last_stats()["rounds"] == rounds[2 * i + j]
+    assert min(rounds) >= 1
+
+
+def test_two_query_lanes(tg):
+    """Sub-batches alternating between two query lanes (scratch sets + streams, option
+    lanes=2, the default for device outputs) give the same rows as one lane, for EAT, LD
+    and REACH, with scheduled (reordered) sources, a ragged last sub-batch and preds."""
+    import torch
+    ge = tgsynth.make_graph("C2", scale_shift=-5)
+    n, u, v, t, d, w = ge.numpy()
+    og = oracle.Graph(n, u, v, t, d)
+    srcs = tgsynth.config_sources("C2", ge, k=200)
+    res = {}
+    for lanes in (1, 2):
+        g = _gpu_graph(tg, n, u, v, t, d, lanes=lanes)
+        for win in tgsynth.CONFIGS["C2"]["windows"]:
+            for p in ("eat", "ld", "reach"):
+                o = g.query(p, srcs, win)
+                o2, pr = g.query(p, srcs, win, with_pred=True)
+                torch.cuda.synchronize()
+                res[(lanes, win, p)] = (tg.as_u32(o), tg.as_u32(o2), tg.as_u32(pr), g.last_stats()["rounds"])
+    for key in [k for k in res if k[0] == 2]:
+        a, b = res[key], res[(1,) + key[1:]]
+        for x, y in zip(a[:3], b[:3]):
+            np.testing.assert_array_equal(x, y)
+        # (round counts are not compared: which round a relaxation lands in depends on the
+        # timing of concurrent claims and stale-safe reads; the fixpoint does not)
+        assert a[3] >= 1 and b[3] >= 1
+    for win in tgsynth.CONFIGS["C2"]["windows"]:
+        vals = res[(2, win, "eat")][0]
+        for r in (0, 63, 64, 127, 128, 199):
+            np.testing.assert_array_equal(vals[r], oracle.eat(og, srcs[r], *win)[0])
 
 
 # --------------------------------------------------------------------------- bit-lane reachability (f2)
