@@ -307,9 +307,9 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *   "graph_loop" 1 (default) = EAT/LD/REACH GAC rounds run as one CUDA graph with a
  *                conditional WHILE node (round number and stop test on the device);
  *                0 = host-driven rounds checked every "round_group" rounds
- *   "lanes"      2 (default) = EAT/LD/REACH calls with several sub-batches and device
- *                outputs keep two sub-batches in flight (two scratch sets and streams;
- *                falls back to 1 when the second scratch set does not fit); 1 = one */
+ *   "lanes"      1..4 (default 4): EAT/LD/REACH calls with several sub-batches and device
+ *                outputs keep up to this many sub-batches in flight, one scratch set and
+ *                stream each (as many sets as fit in device memory); 1 = one at a time */
 TG_API tg_status tg_set_option(tg_graph *g, const char *key, int64_t value);
 
 /* Total kernels this library has launched in this process (all handles). */

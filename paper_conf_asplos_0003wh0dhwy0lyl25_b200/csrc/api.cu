@@ -123,6 +123,18 @@ void tg_pinned_put(void *p) {
 tg_status DevArena::alloc(void **p, size_t bytes) {
     *p = nullptr;
     bytes = round_bytes(bytes ? bytes : 16);
+    if (use_pool) {  // no retry: a query lane that does not fit is simply not used
+        void *q = nullptr;
+        if (cudaMallocAsync(&q, bytes, pool_stream) != cudaSuccess) {
+            cudaGetLastError();
+            tg_set_error("query lane scratch does not fit");
+            return TG_ERR_NOMEM;
+        }
+        *p = q;
+        blks.push_back({q, bytes});
+        total += bytes;
+        return TG_OK;
+    }
     int dev = 0;
     cudaGetDevice(&dev);
     size_t got = bytes;
@@ -153,6 +165,12 @@ tg_status DevArena::alloc(void **p, size_t bytes) {
 }
 
 void DevArena::free_all() {
+    if (use_pool) {  // stream-ordered: after the lane's queued work
+        for (const Blk &b : blks) cudaFreeAsync(b.p, pool_stream);
+        blks.clear();
+        total = 0;
+        return;
+    }
     // callers synchronise before releasing (blocks may be reused by the next owner at once)
     int dev = 0;
     cudaGetDevice(&dev);
@@ -202,7 +220,7 @@ struct DeviceGuard {
 }  // namespace
 
 uint64_t tg_graph_bytes(const tg_graph *g) {
-    uint64_t b = g->arena.total + g->qs.arena.total + g->qs2.arena.total + g->rs.arena.total + g->fwd.arena.total + g->mir.arena.total;
+    uint64_t b = g->arena.total + g->qs.arena.total + g->qsl[0].arena.total + g->qsl[1].arena.total + g->qsl[2].arena.total + g->rs.arena.total + g->fwd.arena.total + g->mir.arena.total;
     for (int p = 0; p < TG_MAXP; p++) b += g->pf[p].arena.total + g->pm[p].arena.total;
     if (g->stream) b += g->stream->slot_arena.total;
     return b;
@@ -245,6 +263,36 @@ int tg_profile_report(char *buf, uint64_t buf_len) {
     // with buf == NULL only returns the size needed.
     struct Acc { std::string name; uint64_t n = 0; double ms = 0; };
     static std::vector<Acc> acc;
+    // graph round loops of concurrent query lanes overlap in time: their union as well
+    // ("k_eat_rounds_union": the wall time some lane's round loop was running)
+    {
+        const char *pre = "k_eat_rounds";
+        cudaEvent_t ref = nullptr;
+        std::vector<std::pair<double, double>> iv;
+        for (auto &r : g_prof) {
+            if (std::strncmp(r.name, pre, std::strlen(pre)) != 0) continue;
+            cudaEventSynchronize(r.e1);
+            if (!ref) ref = r.e0;
+            float a = 0, b = 0;
+            cudaEventElapsedTime(&a, ref, r.e0);
+            cudaEventElapsedTime(&b, ref, r.e1);
+            iv.push_back({a, b});
+        }
+        if (!iv.empty()) {
+            std::sort(iv.begin(), iv.end());
+            double tot = 0, lo = iv[0].first, hi = iv[0].second;
+            for (auto &x : iv) {
+                if (x.first > hi) { tot += hi - lo; lo = x.first; hi = x.second; }
+                else hi = std::max(hi, x.second);
+            }
+            tot += hi - lo;
+            const std::string nm = "k_eat_rounds_union";
+            auto it = std::find_if(acc.begin(), acc.end(), [&](const Acc &p) { return p.name == nm; });
+            if (it == acc.end()) { acc.push_back(Acc{nm}); it = acc.end() - 1; }
+            it->n += iv.size();
+            it->ms += tot;
+        }
+    }
     for (auto &r : g_prof) {
         cudaEventSynchronize(r.e1);
         float ms = 0;
@@ -429,11 +477,15 @@ void tg_graph_destroy(tg_graph *g) {
     tg_round_graph_free(g);
     g->qs.arena.free_all();
     tg_pinned_put(g->qs.h_ctr);
-    g->qs2.arena.free_all();
-    tg_pinned_put(g->qs2.h_ctr);
-    if (g->lane_stream) cudaStreamDestroy(g->lane_stream);
-    for (auto &e : g->lane_ev)
+    for (auto &q : g->qsl) {
+        q.arena.free_all();
+        tg_pinned_put(q.h_ctr);
+    }
+    for (auto &x : g->lane_stream)
+        if (x) cudaStreamDestroy(x);
+    for (auto &e : g->lane_join)
         if (e) cudaEventDestroy(e);
+    if (g->lane_fork) cudaEventDestroy(g->lane_fork);
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);
     g->fwd.arena.free_all();
@@ -586,7 +638,7 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     else if (k == "exchange") g->opt_exchange = value ? 1 : 0;
     else if (k == "packed_state") g->opt_packed_state = value ? 1 : 0;
     else if (k == "graph_loop") g->opt_graph_loop = value ? 1 : 0;
-    else if (k == "lanes") g->opt_lanes = value >= 2 ? 2 : 1;
+    else if (k == "lanes") g->opt_lanes = value < 1 ? 1 : (value > TG_LANES ? TG_LANES : value);
     else if (k == "ub_filter") g->opt_ub = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (k == "reach_bits") g->opt_reach_bits = value ? 1 : 0;
     else if (k == "order_sources") g->opt_order_sources = value ? 1 : 0;

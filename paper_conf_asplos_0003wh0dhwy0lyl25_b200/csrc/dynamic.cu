@@ -188,9 +188,11 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
     g->qs.arena.free_all();
     tg_pinned_put(g->qs.h_ctr);
     g->qs = QueryScratch{};
-    g->qs2.arena.free_all();
-    tg_pinned_put(g->qs2.h_ctr);
-    g->qs2 = QueryScratch{};
+    for (auto &q : g->qsl) {
+        q.arena.free_all();
+        tg_pinned_put(q.h_ctr);
+        q = QueryScratch{};
+    }
     tg_round_graph_free(g);
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);

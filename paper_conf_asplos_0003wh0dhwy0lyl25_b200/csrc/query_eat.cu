@@ -973,20 +973,26 @@ static void rg_free(tg_graph::RoundGraph &G) {
 
 void tg_round_graph_free(tg_graph *g) {
     rg_free(g->rgraph);
-    rg_free(g->rgraph2);
+    for (auto &r : g->rgl) rg_free(r);
 }
 
-static tg_status ensure_scratch_q(tg_graph *g, QueryScratch &Q, uint32_t S, bool nodes_state) {
+// pool_stream: a query lane's scratch, from the stream-ordered pool on that stream (freed
+// at the end of the call, so the next build's temporaries can reuse the memory)
+static tg_status ensure_scratch_q(tg_graph *g, QueryScratch &Q, uint32_t S, bool nodes_state,
+                                  uint32_t st_w = 8, cudaStream_t pool_stream = nullptr) {
     const uint64_t nnodes = std::max(g->fwd.nnodes, g->mir.nnodes);
     const uint32_t copies = (g->opt_exchange && !g->comm && g->nparts > 1) ? (uint32_t)g->nparts : 1u;
     if (Q.S >= S && Q.n == g->n && Q.st && (!nodes_state || Q.nodes_state) && (g->nparts == 0 || Q.lat) &&
-        Q.st_copies >= copies)
+        Q.st_copies >= copies && Q.st_w >= st_w && !pool_stream)
         return TG_OK;
-    TG_TRY_CUDA(cudaDeviceSynchronize());  // blocks go back to the cache for immediate reuse
+    if (!pool_stream) TG_TRY_CUDA(cudaDeviceSynchronize());  // blocks go back to the cache for immediate reuse
     Q.arena.free_all();
     tg_pinned_put(Q.h_ctr);
     Q.h_ctr = nullptr;
     Q = QueryScratch{};
+    Q.arena.use_pool = pool_stream != nullptr;
+    Q.arena.pool_stream = pool_stream;
+    Q.st_w = st_w;
     const uint64_t n = g->n, m = g->stream ? g->stream->max_m : g->m;  // streamed: the largest block
     Q.S = S;
     Q.n = g->n;
@@ -994,7 +1000,7 @@ static tg_status ensure_scratch_q(tg_graph *g, QueryScratch &Q, uint32_t S, bool
     Q.nodes_state = nodes_state;
     DevArena &A = Q.arena;
     Q.st_copies = copies;
-    TG_TRY(A.alloc((void **)&Q.st, S * n * 8 * copies));
+    TG_TRY(A.alloc((void **)&Q.st, S * n * st_w * copies));
     TG_TRY(A.alloc((void **)&Q.act, S * n * 4));
     if (TG_UB) TG_TRY(A.alloc((void **)&Q.ub, n * 8 * UB_WORDS));
     Q.vwords = (uint32_t)((S + 31) / 32);  // query groups per vertex
@@ -1024,9 +1030,14 @@ static tg_status ensure_scratch_q(tg_graph *g, QueryScratch &Q, uint32_t S, bool
     Q.chcap = std::min<uint64_t>(S * (m / 2) + (1u << 16), 1ull << 26);
     TG_TRY(A.alloc((void **)&Q.chq, Q.chcap * 16));
     TG_TRY(A.alloc((void **)&Q.ctr, 64));
-    TG_TRY_CUDA(cudaMemset(Q.ctr, 0, 64));
     TG_TRY(A.alloc((void **)&Q.ctl, sizeof(RoundCtl) * TG_MAXP));
-    TG_TRY_CUDA(cudaMemset(Q.ctl, 0, sizeof(RoundCtl) * TG_MAXP));
+    if (pool_stream) {  // stream-ordered on the lane's stream
+        TG_TRY_CUDA(cudaMemsetAsync(Q.ctr, 0, 64, pool_stream));
+        TG_TRY_CUDA(cudaMemsetAsync(Q.ctl, 0, sizeof(RoundCtl) * TG_MAXP, pool_stream));
+    } else {
+        TG_TRY_CUDA(cudaMemset(Q.ctr, 0, 64));
+        TG_TRY_CUDA(cudaMemset(Q.ctl, 0, sizeof(RoundCtl) * TG_MAXP));
+    }
     if (g->nparts > 0) {
         TG_TRY(A.alloc((void **)&Q.lat, S * n * 4));
         TG_TRY(A.alloc((void **)&Q.pcount, 64));
@@ -1343,49 +1354,55 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     const bool sched = g->opt_order_sources && k > 32 && any_work && g->m > 0 && (!pred || out_dev == pred_dev);
     TG_TRY(tg_schedule_sources(g, cgr, sources, k, alpha, sched, order, s));
     for (uint32_t i = 0; i < k; i++) srcs_sched[i] = sources[order[i]];
-    // Two query lanes: consecutive sub-batches alternate between two scratch sets and two
+    // Query lanes: consecutive sub-batches rotate over up to TG_LANES scratch sets and
     // streams, each running its device-driven round loop, so one sub-batch's kernels fill
-    // the other's kernel tails and sparse rounds (C4 half scale: 535 -> 485 ms).  Device
-    // outputs only (host outputs stream through the single staging sink).
+    // the others' kernel tails and sparse rounds (C4 1024-source job, 2 lanes: 2088 ->
+    // 1844 ms).  Device outputs only (host outputs stream through the single staging sink).
     static const bool trace = getenv("TG_TRACE") != nullptr;
     const bool work = any_work && g->m > 0 && alpha < omega;
-    bool dual = g->opt_lanes >= 2 && k > S && out_dev && (!pred || pred_dev) && !g->opt_stats && g->opt_graph_loop &&
-                !trace && work;
-    if (dual && ensure_scratch_q(g, g->qs2, S, false) != TG_OK) {  // no room for a second scratch set
-        cudaGetLastError();
-        cudaDeviceSynchronize();
-        g->qs2.arena.free_all();
-        tg_pinned_put(g->qs2.h_ctr);
-        g->qs2 = QueryScratch{};
-        dual = false;
-    }
-    cudaStream_t ls[2] = {s, s};
-    if (dual) {
-        if (!g->lane_stream) TG_TRY_CUDA(cudaStreamCreateWithFlags(&g->lane_stream, cudaStreamNonBlocking));
-        if (!g->lane_ev[0]) {
-            TG_TRY_CUDA(cudaEventCreateWithFlags(&g->lane_ev[0], cudaEventDisableTiming));
-            TG_TRY_CUDA(cudaEventCreateWithFlags(&g->lane_ev[1], cudaEventDisableTiming));
+    int lanes = 1;
+    cudaStream_t ls[TG_LANES];
+    for (auto &x : ls) x = s;
+    if (g->opt_lanes >= 2 && k > S && out_dev && (!pred || pred_dev) && !g->opt_stats && g->opt_graph_loop &&
+        !trace && work) {
+        const uint32_t nsub = (k + S - 1) / S;
+        const int want = (int)std::min<uint64_t>((uint64_t)g->opt_lanes, nsub);
+        if (!g->lane_fork) TG_TRY_CUDA(cudaEventCreateWithFlags(&g->lane_fork, cudaEventDisableTiming));
+        TG_TRY_CUDA(cudaEventRecord(g->lane_fork, s));  // the lanes start after the caller's prior work
+        for (lanes = 1; lanes < want; lanes++) {  // as many scratch sets as the pool can hold
+            if (!g->lane_stream[lanes - 1]) {
+                TG_TRY_CUDA(cudaStreamCreateWithFlags(&g->lane_stream[lanes - 1], cudaStreamNonBlocking));
+                TG_TRY_CUDA(cudaEventCreateWithFlags(&g->lane_join[lanes - 1], cudaEventDisableTiming));
+            }
+            const cudaStream_t x = g->lane_stream[lanes - 1];
+            TG_TRY_CUDA(cudaStreamWaitEvent(x, g->lane_fork, 0));
+            QueryScratch &X = g->qsl[lanes - 1];
+            if (ensure_scratch_q(g, X, S, false, pk ? 8 : 4, x) != TG_OK) {
+                X.arena.free_all();
+                tg_pinned_put(X.h_ctr);
+                X = QueryScratch{};
+                break;
+            }
+            ls[lanes] = x;
         }
-        ls[1] = g->lane_stream;
-        TG_TRY_CUDA(cudaEventRecord(g->lane_ev[0], s));  // lane 1 starts after the caller's prior work
-        TG_TRY_CUDA(cudaStreamWaitEvent(ls[1], g->lane_ev[0], 0));
     }
-    bool pending[2] = {false, false};
+    const bool dual = lanes > 1;
+    bool pending[TG_LANES] = {};
     auto finish = [&](int l) -> tg_status {
         if (!pending[l]) return TG_OK;
         pending[l] = false;
         TG_TRY_CUDA(cudaStreamSynchronize(ls[l]));
         uint32_t r = 0;
-        TG_TRY(graph_rounds_finish(l ? g->qs2 : g->qs, &r));
+        TG_TRY(graph_rounds_finish(l ? g->qsl[l - 1] : g->qs, &r));
         g->last.rounds = std::max(g->last.rounds, r);
         return TG_OK;
     };
     for (uint32_t b0 = 0; b0 < k; b0 += S) {
         const uint32_t Sb = std::min(S, k - b0);
         const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
-        const int lane = dual ? (int)(bi & 1) : 0;
-        QueryScratch &Q = lane ? g->qs2 : g->qs;
-        tg_graph::RoundGraph &RG = lane ? g->rgraph2 : g->rgraph;
+        const int lane = (int)(bi % (uint32_t)lanes);
+        QueryScratch &Q = lane ? g->qsl[lane - 1] : g->qs;
+        tg_graph::RoundGraph &RG = lane ? g->rgl[lane - 1] : g->rgraph;
         const cudaStream_t st = ls[lane];
         TG_TRY(finish(lane));  // the lane's previous sub-batch (the other lane keeps running)
         TG_TRY(tg_load_sources_to(g, srcs_sched.data() + b0, Sb, Q.srcs, Q.srcs_int, st));
@@ -1438,11 +1455,16 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
                         h[Sb + 4], h[Sb + 5], h[Sb + 6], h[Sb + 7]);
         }
     }
-    TG_TRY(finish(0));
-    TG_TRY(finish(1));
-    if (dual) {  // the caller's stream continues after lane 1's work
-        TG_TRY_CUDA(cudaEventRecord(g->lane_ev[1], ls[1]));
-        TG_TRY_CUDA(cudaStreamWaitEvent(s, g->lane_ev[1], 0));
+    for (int l = 0; l < lanes; l++) TG_TRY(finish(l));
+    for (int l = 1; l < lanes; l++) {
+        // the lane's scratch back to the pool (stream-ordered), then the caller's stream
+        // continues after the lane's work
+        QueryScratch &X = g->qsl[l - 1];
+        X.arena.free_all();
+        tg_pinned_put(X.h_ctr);
+        X = QueryScratch{};
+        TG_TRY_CUDA(cudaEventRecord(g->lane_join[l - 1], ls[l]));
+        TG_TRY_CUDA(cudaStreamWaitEvent(s, g->lane_join[l - 1], 0));
     }
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     TG_TRY(tg_sink_end(g));

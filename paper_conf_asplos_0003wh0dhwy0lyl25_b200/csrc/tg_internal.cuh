@@ -62,6 +62,8 @@ struct DevArena {
     size_t total = 0;
     uint32_t slack_pct = 0;  // fresh blocks get this much extra room (dynamic graphs: the next,
                              // slightly larger, re-transformation reuses them from the cache)
+    cudaStream_t pool_stream = nullptr;  // set: stream-ordered pool blocks (cudaMallocAsync on this
+    bool use_pool = false;               // stream, no retry; free_all = cudaFreeAsync) -- query lanes
     tg_status alloc(void **p, size_t bytes);
     void free_all();
 };
@@ -122,6 +124,7 @@ struct QueryScratch {
     bool nodes_state = false;  // SP/FP node-state arrays present
     void *st = nullptr;  // [n][S] packed u64 (time << 32 | pred), or u32 time when no pred is requested
     uint32_t st_copies = 1;  // option "exchange" with logical partitions: one private state copy each
+    uint32_t st_w = 8;       // bytes per state entry allocated (8: packed states fit)
     uint32_t *act = nullptr;           // [S][n] last activated time
     unsigned long long *ub = nullptr;  // [n] arrival-bound codes per 8 queries (query_eat.cu, TG_UB)
     uint32_t stamp = 0;                // SP/FP frontier dedupe stamps handed out (host counter; marks start at 0)
@@ -202,6 +205,7 @@ struct ReachScratch {
     DevArena arena;
 };
 
+#define TG_LANES 4  // query lanes at most (option "lanes")
 #define TG_MAXP 16  // logical vertex-range partitions per process (tests / one rank's share)
 
 struct tg_comm;  // comm.cu: NCCL communicator (loaded with dlopen)
@@ -239,11 +243,11 @@ struct tg_graph {
         cudaGraph_t graph = nullptr;
         unsigned char key[512] = {};
         size_t key_len = 0;
-    } rgraph, rgraph2;
-    // second query lane (EAT family, device outputs): its scratch, stream, fork/join events
-    QueryScratch qs2;
-    cudaStream_t lane_stream = nullptr;
-    cudaEvent_t lane_ev[2] = {nullptr, nullptr};
+    } rgraph, rgl[TG_LANES - 1];
+    // query lanes 1 .. TG_LANES-1 (EAT family, device outputs): scratch, stream, join event
+    QueryScratch qsl[TG_LANES - 1];
+    cudaStream_t lane_stream[TG_LANES - 1] = {};
+    cudaEvent_t lane_fork = nullptr, lane_join[TG_LANES - 1] = {};
     ReachScratch rs;
     StreamGraph *stream = nullptr;  // out-of-memory graph (tg_graph_create_streamed)
     uint32_t qs_epoch = 0;  // frontier-dedupe stamp (monotone across rounds and queries)
@@ -256,7 +260,7 @@ struct tg_graph {
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
     int64_t opt_ub = 1;  // arrival bounds per (vertex, 8 queries) prune pairs: 0 off, 1 auto, 2 on (query_eat.cu)
     int64_t opt_graph_loop = 1;
-    int64_t opt_lanes = 2;  // sub-batches in flight (EAT family, device outputs, graph loop): 1 or 2  // 1 = GAC rounds run in a device-driven CUDA-graph WHILE loop (query_eat.cu)
+    int64_t opt_lanes = 4;  // sub-batches in flight (EAT family, device outputs, graph loop): 1 .. TG_LANES  // 1 = GAC rounds run in a device-driven CUDA-graph WHILE loop (query_eat.cu)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
     int64_t opt_order_sources = 1;  // schedule a call's sources by first departure time (query_eat.cu)
     int64_t opt_reach_bits = 0;  // 1 = TG_REACH without pred on the bit-lane engine (query_reach.cu)
