@@ -965,6 +965,18 @@ __global__ void k_round_next(RoundCtl *ctl, cudaGraphConditionalHandle h, uint32
 
 }  // namespace
 
+// Kernel profilers (ncu, compute-sanitizer: CUDA_INJECTION64_PATH) cannot see the kernel nodes
+// of a graph with conditional nodes, so under one the round loop stays host-driven; the
+// environment variable TG_GRAPH_LOOP=0 does the same.
+static bool graph_loop_allowed() {
+    static const bool ok = [] {
+        const char *inj = getenv("CUDA_INJECTION64_PATH");
+        const char *env = getenv("TG_GRAPH_LOOP");
+        return !(inj && inj[0]) && !(env && env[0] == '0');
+    }();
+    return ok;
+}
+
 static void rg_free(tg_graph::RoundGraph &G) {
     if (G.exec) cudaGraphExecDestroy(G.exec);
     if (G.graph) cudaGraphDestroy(G.graph);
@@ -1257,7 +1269,7 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.diag = Q.relax_cnt + S + 1;
         const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;
-        if (g->opt_graph_loop && !trace && !P.stats) {
+        if (g->opt_graph_loop && graph_loop_allowed() && !trace && !P.stats) {
             TG_TRY(graph_rounds<PK>(g, Q, RGp ? *RGp : g->rgraph, P, S, grid, s, rounds_out, async));
             return TG_OK;
         }
@@ -1332,8 +1344,19 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         if (alpha > C) { any_work = false; alpha = 0; omega = 0; }
         else { uint32_t a2 = (omega >= C) ? 0u : C - omega; omega = C - alpha; alpha = a2; }
     }
-    const uint32_t S = tg_pick_sub_batch(g, k, false);
-    TG_TRY(ensure_scratch(g, S, false));
+    // packed (arrival | pred) states only when the caller asked for preds (or forced)
+    const bool pk = pred != nullptr || g->opt_packed_state;
+    static const bool trace = getenv("TG_TRACE") != nullptr;
+    const bool work = any_work && g->m > 0 && alpha < omega;
+    // query lanes (below) need device outputs and the device-driven round loop
+    const bool lanes_ok = g->opt_lanes >= 2 && out_dev && (!pred || pred_dev) && !g->opt_stats &&
+                          g->opt_graph_loop && graph_loop_allowed() && !trace && work;
+    uint32_t S = tg_pick_sub_batch(g, k, false);
+    // a lone full sub-batch runs as two halves on two lanes (C2 64-source EAT 7.9 -> 6.8 ms;
+    // with several sub-batches 64 stays better: C4 1024 sources 1793 vs 1952 ms at 32)
+    if (lanes_ok && g->opt_sub_batch == 0 && S == k && k >= 64) S = ((k + 1) / 2 + 31) / 32 * 32;
+    // state entries at the width this call needs (u32 without preds): room for more lanes
+    TG_TRY(ensure_scratch_q(g, g->qs, S, false, pk ? 8 : 4));
     const uint64_t n = g->n;
     TG_TRY(tg_sink_begin(g, !out_dev, pred && !pred_dev));
     g->last = tg_query_stats{};
@@ -1344,8 +1367,6 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     }
     const uint64_t launches0 = g_tg_launches;
     const int mode = ld ? 1 : (p == TG_REACH ? 2 : 0);
-    // packed (arrival | pred) states only when the caller asked for preds (or forced)
-    const bool pk = pred != nullptr || g->opt_packed_state;
     // Sub-batch composition: sources are scheduled in order of their first departure time
     // >= alpha, so the queries sharing a sub-batch (and a 32-query frontier unit) start -- and
     // reach the graph's vertices -- at similar rounds; their activations share unit scans
@@ -1358,13 +1379,10 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     // streams, each running its device-driven round loop, so one sub-batch's kernels fill
     // the others' kernel tails and sparse rounds (C4 1024-source job, 2 lanes: 2088 ->
     // 1844 ms).  Device outputs only (host outputs stream through the single staging sink).
-    static const bool trace = getenv("TG_TRACE") != nullptr;
-    const bool work = any_work && g->m > 0 && alpha < omega;
     int lanes = 1;
     cudaStream_t ls[TG_LANES];
     for (auto &x : ls) x = s;
-    if (g->opt_lanes >= 2 && k > S && out_dev && (!pred || pred_dev) && !g->opt_stats && g->opt_graph_loop &&
-        !trace && work) {
+    if (lanes_ok && k > S) {
         const uint32_t nsub = (k + S - 1) / S;
         const int want = (int)std::min<uint64_t>((uint64_t)g->opt_lanes, nsub);
         if (!g->lane_fork) TG_TRY_CUDA(cudaEventCreateWithFlags(&g->lane_fork, cudaEventDisableTiming));

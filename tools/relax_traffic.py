@@ -2,7 +2,7 @@
 64-source query into profiles/round2/relax_traffic_<CFG>.json, the `traffic` of bench.py's
 roofline: DRAM bytes per bench step = per-query bytes x queries per step / 64.
 
-usage: python tools/relax_traffic.py LOG.csv CFG SUBBATCHES_PER_STEP"""
+usage: python tools/relax_traffic.py LOG.csv CFG CALLS_PER_STEP [K]"""
 import collections
 import csv
 import json
@@ -10,6 +10,7 @@ import os
 import sys
 
 log, cfg, per_step = sys.argv[1], sys.argv[2], float(sys.argv[3])
+kq = int(sys.argv[4]) if len(sys.argv) > 4 else 64
 rows = [r for r in csv.reader(open(log)) if len(r) > 10]
 hdr = rows[0]
 ix = {k: i for i, k in enumerate(hdr)}
@@ -40,8 +41,8 @@ out = {
                        "dram_GB": round((v["dram__bytes_read.sum"] + v["dram__bytes_write.sum"]) / 1e9, 3)}
                    for k, v in acc.items()},
     "source": (f"ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum over every "
-               f"k_eat_(activate|big|chain) launch of one 64-source EAT query (tools/prof_query.py --config {cfg}), "
-               f"serialised cold-cache replay; x{per_step:g} sub-batches per bench step"),
+               f"k_eat_(activate|big|chain) launch of one {kq}-source EAT call (tools/prof_query.py --config {cfg} "
+               f"--k {kq}), serialised cold-cache replay; x{per_step:g} such calls per bench step"),
 }
 dst = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "round2",
                    f"relax_traffic_{cfg}.json")
