@@ -965,14 +965,24 @@ __global__ void k_round_next(RoundCtl *ctl, cudaGraphConditionalHandle h, uint32
 
 }  // namespace
 
-// Kernel profilers (ncu, compute-sanitizer: CUDA_INJECTION64_PATH) cannot see the kernel nodes
-// of a graph with conditional nodes, so under one the round loop stays host-driven; the
-// environment variable TG_GRAPH_LOOP=0 does the same.
+// Kernel profilers (ncu, compute-sanitizer) cannot see the kernel nodes of a graph with
+// conditional nodes, so under one the round loop stays host-driven.  A profiler is detected
+// by its injection library in this process's mappings (or CUDA_INJECTION64_PATH); the
+// environment variable TG_GRAPH_LOOP=0 forces the host-driven loop too.
 static bool graph_loop_allowed() {
     static const bool ok = [] {
         const char *inj = getenv("CUDA_INJECTION64_PATH");
         const char *env = getenv("TG_GRAPH_LOOP");
-        return !(inj && inj[0]) && !(env && env[0] == '0');
+        const char *nsi = getenv("NV_NSIGHT_INJECTION_TRANSPORT_TYPE");  // set by ncu in its target
+        if ((inj && inj[0]) || (nsi && nsi[0]) || (env && env[0] == '0')) return false;
+        FILE *f = fopen("/proc/self/maps", "r");
+        if (!f) return true;
+        char line[4096];
+        bool tool = false;
+        while (!tool && fgets(line, sizeof(line), f))
+            tool = strstr(line, "injection") || strstr(line, "nsight-compute") || strstr(line, "sanitizer");
+        fclose(f);
+        return !tool;
     }();
     return ok;
 }
@@ -1349,8 +1359,10 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     static const bool trace = getenv("TG_TRACE") != nullptr;
     const bool work = any_work && g->m > 0 && alpha < omega;
     // query lanes (below) need device outputs and the device-driven round loop
-    const bool lanes_ok = g->opt_lanes >= 2 && out_dev && (!pred || pred_dev) && !g->opt_stats &&
-                          g->opt_graph_loop && graph_loop_allowed() && !trace && work;
+    // (host outputs too: each sub-batch's extract waits for its staging buffer's previous
+    // copy, wherever that ran -- the rounds of the lanes still overlap)
+    const bool lanes_ok = g->opt_lanes >= 2 && !g->opt_stats && g->opt_graph_loop && graph_loop_allowed() &&
+                          !trace && work;
     uint32_t S = tg_pick_sub_batch(g, k, false);
     // a lone full sub-batch runs as two halves on two lanes (C2 64-source EAT 7.9 -> 6.8 ms;
     // with several sub-batches 64 stays better: C4 1024 sources 1793 vs 1952 ms at 32)
@@ -1378,7 +1390,7 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     // Query lanes: consecutive sub-batches rotate over up to TG_LANES scratch sets and
     // streams, each running its device-driven round loop, so one sub-batch's kernels fill
     // the others' kernel tails and sparse rounds (C4 1024-source job, 2 lanes: 2088 ->
-    // 1844 ms).  Device outputs only (host outputs stream through the single staging sink).
+    // 1844 ms).
     int lanes = 1;
     cudaStream_t ls[TG_LANES];
     for (auto &x : ls) x = s;

@@ -557,7 +557,12 @@ def test_two_query_lanes(tg):
                 o2, pr = g.query(p, srcs, win, with_pred=True)
                 torch.cuda.synchronize()
                 res[(lanes, win, p)] = (tg.as_u32(o), tg.as_u32(o2), tg.as_u32(pr), g.last_stats()["rounds"])
-    for key in [k for k in res if k[0] > 1]:
+        # host outputs (pinned staging ring on a copy stream) with the lanes
+        win = tgsynth.CONFIGS["C2"]["windows"][0]
+        h = torch.empty((len(srcs), n), dtype=torch.int32).pin_memory()
+        g.query("eat", srcs, win, out=h)
+        res[(lanes, "host")] = tg.as_u32(h)
+    for key in [k for k in res if k[0] > 1 and k[1] != "host"]:
         a, b = res[key], res[(1,) + key[1:]]
         for x, y in zip(a[:3], b[:3]):
             np.testing.assert_array_equal(x, y)
@@ -568,6 +573,9 @@ def test_two_query_lanes(tg):
         vals = res[(2, win, "eat")][0]
         for r in (0, 63, 64, 127, 128, 199):
             np.testing.assert_array_equal(vals[r], oracle.eat(og, srcs[r], *win)[0])
+    for lanes in (2, 4):
+        np.testing.assert_array_equal(res[(lanes, "host")], res[(1, "host")])
+        np.testing.assert_array_equal(res[(lanes, "host")], res[(1, tgsynth.CONFIGS["C2"]["windows"][0], "eat")][0])
 
 
 # --------------------------------------------------------------------------- bit-lane reachability (f2)
