@@ -304,9 +304,11 @@ TG_API tg_status tg_graph_attach_comm(tg_graph *g, tg_comm *c, int mode);
  *                an edge skip the queries it cannot improve before any state read.
  *                0 = off, 1 (default) = on when the sub-batch state is >= 1 GiB, 2 = on.
  *                Results are identical either way.
- *   "graph_loop" 1 (default) = EAT/LD/REACH GAC rounds run as one CUDA graph with a
- *                conditional WHILE node (round number and stop test on the device);
- *                0 = host-driven rounds checked every "round_group" rounds
+ *   "graph_loop" GAC rounds (EAT/LD/REACH and SP/FP/LDS) as one CUDA graph with a
+ *                conditional WHILE node (round number and stop test on the device):
+ *                1 (default) = for graphs of >= 2^23 edges, 2 = always, 0 = never (host-
+ *                driven rounds checked every "round_group" rounds); query lanes need it.
+ *                Under a kernel profiler (ncu, compute-sanitizer) the rounds are host-driven
  *   "lanes"      1..4 (default 4): EAT/LD/REACH calls with several sub-batches and device
  *                outputs keep up to this many sub-batches in flight, one scratch set and
  *                stream each (as many sets as fit in device memory); 1 = one at a time */

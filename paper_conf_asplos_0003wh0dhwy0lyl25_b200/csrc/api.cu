@@ -474,7 +474,6 @@ void tg_graph_destroy(tg_graph *g) {
     cudaDeviceSynchronize();
     tg_sink_destroy(g);
     tg_stream_free(g);
-    tg_round_graph_free(g);
     g->qs.arena.free_all();
     tg_pinned_put(g->qs.h_ctr);
     for (auto &q : g->qsl) {
@@ -637,7 +636,7 @@ tg_status tg_set_option(tg_graph *g, const char *key, int64_t value) {
     }
     else if (k == "exchange") g->opt_exchange = value ? 1 : 0;
     else if (k == "packed_state") g->opt_packed_state = value ? 1 : 0;
-    else if (k == "graph_loop") g->opt_graph_loop = value ? 1 : 0;
+    else if (k == "graph_loop") g->opt_graph_loop = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (k == "lanes") g->opt_lanes = value < 1 ? 1 : (value > TG_LANES ? TG_LANES : value);
     else if (k == "ub_filter") g->opt_ub = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (k == "reach_bits") g->opt_reach_bits = value ? 1 : 0;

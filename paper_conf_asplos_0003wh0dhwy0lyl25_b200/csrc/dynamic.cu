@@ -193,7 +193,6 @@ extern "C" tg_status tg_graph_insert_edges(tg_graph *g, uint64_t k, const uint32
         tg_pinned_put(q.h_ctr);
         q = QueryScratch{};
     }
-    tg_round_graph_free(g);
     g->rs.arena.free_all();
     tg_pinned_put(g->rs.h_ctr);
     g->rs = ReachScratch{};

@@ -36,6 +36,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <vector>
 
 #include "tg_internal.cuh"
@@ -969,7 +970,12 @@ __global__ void k_round_next(RoundCtl *ctl, cudaGraphConditionalHandle h, uint32
 // conditional nodes, so under one the round loop stays host-driven.  A profiler is detected
 // by its injection library in this process's mappings (or CUDA_INJECTION64_PATH); the
 // environment variable TG_GRAPH_LOOP=0 forces the host-driven loop too.
-static bool graph_loop_allowed() {
+// Graphs below TG_GRAPH_LOOP_MIN_M edges keep the host-driven loop: their rounds are a few
+// microseconds, and a new handle's first loop pays an instantiation (C1 / C3 bench steps with
+// a fresh handle each: 3.9 / 8.4 ms host-driven vs 4.1-5.4 / 8.9-11.9 ms with the graph).
+bool tg_graph_loop_worth(const tg_graph *g) { return g->opt_graph_loop == 2 || g->m >= TG_GRAPH_LOOP_MIN_M; }
+
+bool tg_graph_loop_allowed() {
     static const bool ok = [] {
         const char *inj = getenv("CUDA_INJECTION64_PATH");
         const char *env = getenv("TG_GRAPH_LOOP");
@@ -987,15 +993,34 @@ static bool graph_loop_allowed() {
     return ok;
 }
 
-static void rg_free(tg_graph::RoundGraph &G) {
-    if (G.exec) cudaGraphExecDestroy(G.exec);
-    if (G.graph) cudaGraphDestroy(G.graph);
-    G = tg_graph::RoundGraph{};
+namespace {
+struct RGEntry {
+    int dev;
+    std::vector<unsigned char> key;
+    cudaGraph_t graph;
+    cudaGraphExec_t exec;
+};
+std::mutex g_rg_mu;
+std::vector<RGEntry> g_rg;
+constexpr size_t RG_MAX = 256;  // distinct loop shapes kept (never evicted: no graph in flight is destroyed)
+}  // namespace
+
+cudaGraphExec_t tg_rg_find(const unsigned char *key, size_t len) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(g_rg_mu);
+    for (const RGEntry &e : g_rg)
+        if (e.dev == dev && e.key.size() == len && std::memcmp(e.key.data(), key, len) == 0) return e.exec;
+    return nullptr;
 }
 
-void tg_round_graph_free(tg_graph *g) {
-    rg_free(g->rgraph);
-    for (auto &r : g->rgl) rg_free(r);
+bool tg_rg_add(const unsigned char *key, size_t len, cudaGraph_t graph, cudaGraphExec_t exec) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(g_rg_mu);
+    if (g_rg.size() >= RG_MAX) return false;
+    g_rg.push_back(RGEntry{dev, std::vector<unsigned char>(key, key + len), graph, exec});
+    return true;
 }
 
 // pool_stream: a query lane's scratch, from the stream-ordered pool on that stream (freed
@@ -1105,7 +1130,7 @@ tg_status tg_ensure_scratch(tg_graph *g, uint32_t S, bool nodes_state) { return 
 template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
                           cudaStream_t s, uint32_t *rounds_out, bool ub = false, QueryScratch *Qp = nullptr,
-                          tg_graph::RoundGraph *RGp = nullptr, bool async = false);
+                          bool async = false);
 
 // One GAC round's relax kernels; the stats counters are a template argument so that the
 // timed path carries no per-pair stats branch.
@@ -1143,63 +1168,73 @@ static uint32_t dir_max_t(const tg_graph *g, const ChainGraph &cg) {
 static tg_status graph_rounds_finish(QueryScratch &Q, uint32_t *rounds);
 
 template <bool PK>
-static tg_status graph_rounds(tg_graph *g, QueryScratch &Q, tg_graph::RoundGraph &RG, EatP P, uint32_t S,
-                              uint32_t grid, cudaStream_t s, uint32_t *rounds, bool async) {
+static tg_status graph_rounds(tg_graph *g, QueryScratch &Q, EatP P, uint32_t S, uint32_t grid, cudaStream_t s,
+                              uint32_t *rounds, bool async) {
     constexpr uint32_t LIMIT = 1000000;
     P.round = 0;  // device-side round (RoundCtl::round, reset by k_eat_init / k_ctl_reset)
     // the key: everything the captured launches depend on (parameters, shape, state width)
-    unsigned char key[sizeof(EatP) + 9];
-    static_assert(sizeof(key) <= sizeof(RG.key), "round-graph key");
+    unsigned char key[sizeof(EatP) + 10];
     std::memcpy(key, &P, sizeof(EatP));
     std::memcpy(key + sizeof(EatP), &S, 4);
     std::memcpy(key + sizeof(EatP) + 4, &grid, 4);
     key[sizeof(EatP) + 8] = PK ? 1 : 0;
-    if (!RG.exec || RG.key_len != sizeof(key) || std::memcmp(RG.key, key, sizeof(key)) != 0) {
-        rg_free(RG);
-        TG_TRY_CUDA(cudaGraphCreate(&RG.graph, 0));
+    key[sizeof(EatP) + 9] = 'E';  // the EAT family's loop
+    cudaGraphExec_t exec = tg_rg_find(key, sizeof(key));
+    cudaGraph_t graph = nullptr;
+    bool owned = false;  // a one-shot instantiation (the cache is full)
+    if (!exec) {
+        TG_TRY_CUDA(cudaGraphCreate(&graph, 0));
         cudaGraphConditionalHandle h;
-        TG_TRY_CUDA(cudaGraphConditionalHandleCreate(&h, RG.graph, 1, cudaGraphCondAssignDefault));
+        cudaError_t e = cudaGraphConditionalHandleCreate(&h, graph, 1, cudaGraphCondAssignDefault);
         cudaGraphNodeParams cp = {};
         cp.type = cudaGraphNodeTypeConditional;
         cp.conditional.handle = h;
         cp.conditional.type = cudaGraphCondTypeWhile;
         cp.conditional.size = 1;
         cudaGraphNode_t node;
-        TG_TRY_CUDA(cudaGraphAddNode(&node, RG.graph, nullptr, 0, &cp));
-        cudaGraph_t body = cp.conditional.phGraph_out[0];
-        cudaStream_t cs;  // capture needs a non-legacy stream
-        TG_TRY_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
-        cudaError_t e = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
+        if (e == cudaSuccess) e = cudaGraphAddNode(&node, graph, nullptr, 0, &cp);
         tg_status st = TG_OK;
         if (e == cudaSuccess) {
-            const int prof = g_tg_profile;
-            const uint64_t l0 = g_tg_launches;
-            g_tg_profile = 0;  // no event records inside the body
-            st = launch_round<PK, false>(P, S, grid, cs, nullptr);
-            if (st == TG_OK) k_round_next<<<1, 32, 0, cs>>>(Q.ctl, h, LIMIT);
-            g_tg_profile = prof;
-            g_tg_launches = l0;  // counted per executed round below
-            cudaGraph_t out = nullptr;
-            const cudaError_t e2 = cudaStreamEndCapture(cs, &out);
-            if (e == cudaSuccess) e = e2;
-            if (e == cudaSuccess) e = cudaGetLastError();
+            cudaGraph_t body = cp.conditional.phGraph_out[0];
+            cudaStream_t cs;  // capture needs a non-legacy stream
+            e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+            if (e == cudaSuccess) {
+                e = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
+                if (e == cudaSuccess) {
+                    const int prof = g_tg_profile;
+                    const uint64_t l0 = g_tg_launches;
+                    g_tg_profile = 0;  // no event records inside the body
+                    st = launch_round<PK, false>(P, S, grid, cs, nullptr);
+                    if (st == TG_OK) k_round_next<<<1, 32, 0, cs>>>(Q.ctl, h, LIMIT);
+                    g_tg_profile = prof;
+                    g_tg_launches = l0;  // counted per executed round below
+                    cudaGraph_t out = nullptr;
+                    const cudaError_t e2 = cudaStreamEndCapture(cs, &out);
+                    if (e == cudaSuccess) e = e2;
+                    if (e == cudaSuccess) e = cudaGetLastError();
+                }
+                cudaStreamDestroy(cs);
+            }
         }
-        cudaStreamDestroy(cs);
-        if (st != TG_OK) { rg_free(RG); return st; }
-        if (e == cudaSuccess) e = cudaGraphInstantiate(&RG.exec, RG.graph, 0);
-        if (e != cudaSuccess) {
-            rg_free(RG);
+        if (st == TG_OK && e == cudaSuccess) e = cudaGraphInstantiate(&exec, graph, 0);
+        if (st != TG_OK || e != cudaSuccess) {
+            cudaGraphDestroy(graph);
+            if (st != TG_OK) return st;
             tg_set_error(std::string("round graph: ") + cudaGetErrorString(e));
             return TG_ERR_CUDA;
         }
-        std::memcpy(RG.key, key, sizeof(key));
-        RG.key_len = sizeof(key);
+        owned = !tg_rg_add(key, sizeof(key), graph, exec);
     }
     cudaEvent_t ev0 = (g_tg_profile && g_tg_profile <= 2) ? tg_prof_begin(s) : nullptr;
-    TG_TRY_CUDA(cudaGraphLaunch(RG.exec, s));
+    TG_TRY_CUDA(cudaGraphLaunch(exec, s));
     if (ev0) tg_prof_end("k_eat_rounds (graph loop: k_eat_activate + k_eat_big + k_eat_chain per round)", s, ev0);
     TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
-    if (async) return TG_OK;  // two query lanes: graph_rounds_finish after the lane's stream is synchronised
+    if (owned) {  // one-shot: wait, then release
+        TG_TRY_CUDA(cudaStreamSynchronize(s));
+        cudaGraphExecDestroy(exec);
+        cudaGraphDestroy(graph);
+    }
+    if (async) return TG_OK;  // query lanes: graph_rounds_finish after the lane's stream is synchronised
     TG_TRY_CUDA(cudaStreamSynchronize(s));
     return graph_rounds_finish(Q, rounds);
 }
@@ -1216,7 +1251,7 @@ static tg_status graph_rounds_finish(QueryScratch &Q, uint32_t *rounds) {
 
 // Run the GAC rounds of one sub-batch on direction cg; returns rounds used.
 template <bool PK>
-static tg_status eat_rounds(tg_graph *g, QueryScratch &Q, tg_graph::RoundGraph &RG, const ChainGraph &cgr, uint32_t S,
+static tg_status eat_rounds(tg_graph *g, QueryScratch &Q, const ChainGraph &cgr, uint32_t S,
                             uint32_t alpha, uint32_t omega, bool any_work, cudaStream_t s, uint32_t *rounds_out,
                             bool async) {
     const uint64_t n = g->n;
@@ -1240,7 +1275,7 @@ static tg_status eat_rounds(tg_graph *g, QueryScratch &Q, tg_graph::RoundGraph &
     TG_LAUNCH(k_eat_init<PK>, (S + 255) / 256, 256, 0, s, Q.st, g->n, G, Q.srcs_int, S, alpha, Q.fb[1], Q.ctl,
               work ? 1 : 0);
     *rounds_out = 0;
-    if (work) TG_TRY(eat_loop<PK>(g, cgr, S, alpha, omega, s, rounds_out, ub, &Q, &RG, async));
+    if (work) TG_TRY(eat_loop<PK>(g, cgr, S, alpha, omega, s, rounds_out, ub, &Q, async));
     return TG_OK;
 }
 
@@ -1248,8 +1283,7 @@ static tg_status eat_rounds(tg_graph *g, QueryScratch &Q, tg_graph::RoundGraph &
 // round control reset; stops at the first round whose frontier was empty.
 template <bool PK>
 static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32_t alpha, uint32_t omega,
-                          cudaStream_t s, uint32_t *rounds_out, bool ub, QueryScratch *Qp, tg_graph::RoundGraph *RGp,
-                          bool async) {
+                          cudaStream_t s, uint32_t *rounds_out, bool ub, QueryScratch *Qp, bool async) {
     QueryScratch &Q = Qp ? *Qp : g->qs;
     const uint32_t G = (S + 31) / 32;
     uint32_t rounds = 0;
@@ -1279,8 +1313,8 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.diag = Q.relax_cnt + S + 1;
         const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;
-        if (g->opt_graph_loop && graph_loop_allowed() && !trace && !P.stats) {
-            TG_TRY(graph_rounds<PK>(g, Q, RGp ? *RGp : g->rgraph, P, S, grid, s, rounds_out, async));
+        if (g->opt_graph_loop && tg_graph_loop_allowed() && tg_graph_loop_worth(g) && !trace && !P.stats) {
+            TG_TRY(graph_rounds<PK>(g, Q, P, S, grid, s, rounds_out, async));
             return TG_OK;
         }
         if (async) { tg_set_error("async rounds need the graph loop"); return TG_ERR_STATE; }
@@ -1361,7 +1395,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     // query lanes (below) need device outputs and the device-driven round loop
     // (host outputs too: each sub-batch's extract waits for its staging buffer's previous
     // copy, wherever that ran -- the rounds of the lanes still overlap)
-    const bool lanes_ok = g->opt_lanes >= 2 && !g->opt_stats && g->opt_graph_loop && graph_loop_allowed() &&
+    const bool lanes_ok = g->opt_lanes >= 2 && !g->opt_stats && g->opt_graph_loop && tg_graph_loop_allowed() &&
+                          tg_graph_loop_worth(g) &&
                           !trace && work;
     uint32_t S = tg_pick_sub_batch(g, k, false);
     // a lone full sub-batch runs as two halves on two lanes (C2 64-source EAT 7.9 -> 6.8 ms;
@@ -1432,7 +1467,6 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
         const uint32_t bi = b0 / S;  // sub-batch index (staging buffer bi & 1 for host outputs)
         const int lane = (int)(bi % (uint32_t)lanes);
         QueryScratch &Q = lane ? g->qsl[lane - 1] : g->qs;
-        tg_graph::RoundGraph &RG = lane ? g->rgl[lane - 1] : g->rgraph;
         const cudaStream_t st = ls[lane];
         TG_TRY(finish(lane));  // the lane's previous sub-batch (the other lane keeps running)
         TG_TRY(tg_load_sources_to(g, srcs_sched.data() + b0, Sb, Q.srcs, Q.srcs_int, st));
@@ -1445,8 +1479,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
             rows = Q.rows;
         }
         uint32_t rounds = 0;
-        if (pk) TG_TRY(eat_rounds<true>(g, Q, RG, cgr, Sb, alpha, omega, any_work, st, &rounds, dual));
-        else TG_TRY(eat_rounds<false>(g, Q, RG, cgr, Sb, alpha, omega, any_work, st, &rounds, dual));
+        if (pk) TG_TRY(eat_rounds<true>(g, Q, cgr, Sb, alpha, omega, any_work, st, &rounds, dual));
+        else TG_TRY(eat_rounds<false>(g, Q, cgr, Sb, alpha, omega, any_work, st, &rounds, dual));
         if (dual) pending[lane] = true;
         else g->last.rounds = std::max(g->last.rounds, rounds);
         g->last.sub_batches++;

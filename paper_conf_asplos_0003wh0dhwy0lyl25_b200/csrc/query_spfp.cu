@@ -25,6 +25,9 @@
 #include <cstdlib>
 #include <vector>
 
+#include <cstring>
+#include <string>
+
 #include "tg_internal.cuh"
 
 namespace cg = cooperative_groups;
@@ -58,6 +61,7 @@ struct SpP {
     int use_sc;
     RoundCtl *ctl;
     uint32_t round, stamp;  // round of this launch and its dedupe stamp (host counters)
+    uint32_t dev_round;     // 1: graph loop -- round = RoundCtl::round, stamp = RoundCtl::stamp + round
     unsigned long long *fr0, *fr1;
     uint4 *bigq;
     uint64_t bigcap;
@@ -68,6 +72,7 @@ struct SpP {
 };
 
 struct RoundV {
+    uint32_t r;
     uint32_t stamp;
     const unsigned long long *fin;
     uint32_t fin_n;
@@ -77,8 +82,9 @@ struct RoundV {
 
 __device__ __forceinline__ RoundV round_view(const SpP &P) {
     RoundV R;
-    const uint32_t r = P.round;
-    R.stamp = P.stamp;
+    const uint32_t r = P.dev_round ? *(volatile const uint32_t *)&P.ctl->round : P.round;
+    R.r = r;
+    R.stamp = P.dev_round ? *(volatile const uint32_t *)&P.ctl->stamp + r : P.stamp;
     R.fin = (r & 1) ? P.fr1 : P.fr0;
     R.fout = (r & 1) ? P.fr0 : P.fr1;
     R.fin_n = *(volatile uint32_t *)&P.ctl->cnt[r & 3][0];
@@ -92,9 +98,9 @@ __device__ __forceinline__ RoundV round_view(const SpP &P) {
 // (its input count is written during round r+1) and round r+1's work-queue counts.
 // The host reads round r+1's input count after round r; it is cleared again only in
 // round r+3.
-__device__ __forceinline__ void clear_later_rounds(const SpP &P) {
+__device__ __forceinline__ void clear_later_rounds(const SpP &P, const RoundV &R) {
     if (blockIdx.x != 0) return;
-    const uint32_t r = P.round;
+    const uint32_t r = R.r;
     if (threadIdx.x < 4) P.ctl->cnt[(r + 2) & 3][threadIdx.x] = 0;
     else if (threadIdx.x < 6) P.ctl->cnt[(r + 1) & 3][threadIdx.x - 3] = 0;
 }
@@ -207,7 +213,7 @@ __device__ __forceinline__ void spfp_edge(const SpP &P, const RoundV &R, uint32_
 template <int MODE, bool ST>
 __global__ void __launch_bounds__(QT) k_spfp_activate(SpP P) {
     const RoundV R = round_view(P);
-    clear_later_rounds(P);
+    clear_later_rounds(P, R);
     const uint32_t F = R.fin_n;
     const int lane = threadIdx.x & 31;
     const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -373,9 +379,23 @@ __global__ void __launch_bounds__(QT) k_spfp_big(SpP P) {
 
 // VInitial: the source's departure nodes tau >= alpha get 0 (SP) / LS = tau (FP).
 // round control for a new loop (before k_spfp_init pushes into buffer 1)
-__global__ void k_spfp_ctl_init(RoundCtl *ctl) {
+__global__ void k_spfp_ctl_init(RoundCtl *ctl, uint32_t stamp_base) {
     for (int i = 0; i < 4; i++)
         for (int j = 0; j < 4; j++) ctl->cnt[i][j] = 0;
+    ctl->round = 1;
+    ctl->stamp = stamp_base;  // graph loop: round r's stamp = stamp_base + r
+}
+
+// Graph loop: ends round r; the loop stops when the next round's input is empty.
+__global__ void k_spfp_round_next(RoundCtl *ctl, cudaGraphConditionalHandle h, uint32_t limit) {
+    if (threadIdx.x != 0) return;
+    const uint32_t r = ctl->round;
+    if (ctl->cnt[(r + 1) & 3][0] == 0 || r >= limit) {
+        ctl->last = r;
+        cudaGraphSetConditional(h, 0);
+    } else {
+        ctl->round = r + 1;
+    }
 }
 
 template <int MODE>
@@ -422,6 +442,76 @@ __global__ void k_spfp_extract(const uint32_t *__restrict__ vout, uint32_t n, co
 
 }  // namespace
 
+// The rounds of one SP/FP/LDS sub-batch as one CUDA graph with a conditional WHILE node
+// (as the EAT family's, query_eat.cu): round number and stamp on the device, the loop ends
+// when the next round's frontier is empty.  Cached on the handle by launch parameters.
+template <int MODE>
+static tg_status spfp_graph_rounds(tg_graph *g, QueryScratch &Q, const SpP &P, uint32_t grid, cudaStream_t s,
+                                   uint32_t *rounds) {
+    constexpr uint32_t LIMIT = 10000000;
+    unsigned char key[sizeof(SpP) + 9];
+    std::memcpy(key, &P, sizeof(SpP));
+    std::memcpy(key + sizeof(SpP), &grid, 4);
+    const int32_t mode = MODE;
+    std::memcpy(key + sizeof(SpP) + 4, &mode, 4);
+    key[sizeof(SpP) + 8] = 'S';  // the SP/FP/LDS loop
+    cudaGraphExec_t exec = tg_rg_find(key, sizeof(key));
+    cudaGraph_t graph = nullptr;
+    bool owned = false;
+    if (!exec) {
+        TG_TRY_CUDA(cudaGraphCreate(&graph, 0));
+        cudaGraphConditionalHandle h;
+        cudaError_t e = cudaGraphConditionalHandleCreate(&h, graph, 1, cudaGraphCondAssignDefault);
+        cudaGraphNodeParams cp = {};
+        cp.type = cudaGraphNodeTypeConditional;
+        cp.conditional.handle = h;
+        cp.conditional.type = cudaGraphCondTypeWhile;
+        cp.conditional.size = 1;
+        cudaGraphNode_t node;
+        if (e == cudaSuccess) e = cudaGraphAddNode(&node, graph, nullptr, 0, &cp);
+        if (e == cudaSuccess) {
+            cudaGraph_t body = cp.conditional.phGraph_out[0];
+            cudaStream_t cs;
+            e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+            if (e == cudaSuccess) {
+                e = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
+                if (e == cudaSuccess) {
+                    k_spfp_activate<MODE, false><<<grid, QT, 0, cs>>>(P);
+                    k_spfp_wait<MODE, false><<<grid, QT, 0, cs>>>(P);
+                    k_spfp_big<MODE, false><<<grid, QT, 0, cs>>>(P);
+                    k_spfp_round_next<<<1, 32, 0, cs>>>(Q.ctl, h, LIMIT);
+                    cudaGraph_t out = nullptr;
+                    const cudaError_t e2 = cudaStreamEndCapture(cs, &out);
+                    e = e2 != cudaSuccess ? e2 : cudaGetLastError();
+                }
+                cudaStreamDestroy(cs);
+            }
+        }
+        if (e == cudaSuccess) e = cudaGraphInstantiate(&exec, graph, 0);
+        if (e != cudaSuccess) {
+            cudaGraphDestroy(graph);
+            tg_set_error(std::string("SP/FP round graph: ") + cudaGetErrorString(e));
+            return TG_ERR_CUDA;
+        }
+        owned = !tg_rg_add(key, sizeof(key), graph, exec);
+    }
+    cudaEvent_t ev0 = (g_tg_profile && g_tg_profile <= 2) ? tg_prof_begin(s) : nullptr;
+    TG_TRY_CUDA(cudaGraphLaunch(exec, s));
+    if (ev0) tg_prof_end("k_spfp_rounds (graph loop: k_spfp_activate + k_spfp_wait + k_spfp_big per round)", s, ev0);
+    TG_TRY_CUDA(cudaMemcpyAsync(Q.h_ctr, Q.ctl, sizeof(RoundCtl), cudaMemcpyDeviceToHost, s));
+    TG_TRY_CUDA(cudaStreamSynchronize(s));
+    if (owned) {
+        cudaGraphExecDestroy(exec);
+        cudaGraphDestroy(graph);
+    }
+    const RoundCtl *hc = (const RoundCtl *)Q.h_ctr;
+    const uint32_t last = hc->last;
+    g_tg_launches += 4ull * last;
+    if (hc->cnt[(last + 1) & 3][0] != 0) { tg_set_error("SP/FP rounds did not converge"); return TG_ERR_CUDA; }
+    *rounds = last;
+    return TG_OK;
+}
+
 template <int MODE>
 static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t omega, cudaStream_t s,
                              uint32_t *rounds_out) {
@@ -446,16 +536,27 @@ static tg_status spfp_rounds(tg_graph *g, uint32_t Sb, uint32_t alpha, uint32_t 
     P.bigq = Q.bigq; P.bigcap = Q.bigcap;
     P.waitq = Q.chq; P.waitcap = Q.chcap;
     P.cnt = Q.relax_cnt; P.stats = (int)g->opt_stats;
-    TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl);
-    // rounds and dedupe stamps are host counters passed with each launch; stamps only
-    // grow (marks of earlier rounds and loops never match)
+    // rounds and dedupe stamps are host counters passed with each launch (graph loop: on
+    // the device, round r's stamp = the base + r); stamps only grow (marks of earlier
+    // rounds and loops never match)
+    const uint32_t stamp0 = ++Q.stamp;
+    TG_LAUNCH(k_spfp_ctl_init, 1, 1, 0, s, Q.ctl, stamp0);
     {
         P.round = 0;  // k_spfp_init pushes with round 0's view: output buffer 1, count cnt[1][0]
-        P.stamp = ++Q.stamp;
+        P.stamp = stamp0;
         dim3 grid(64, Sb);  // a hub source has many departure nodes
         TG_LAUNCH(k_spfp_init<MODE>, grid, 256, 0, s, P, Q.srcs_int, Sb);
     }
     const uint32_t grid = tg_grid_persistent(8);
+    static const bool trace0 = getenv("TG_TRACE") != nullptr;
+    if (g->opt_graph_loop && tg_graph_loop_allowed() && tg_graph_loop_worth(g) && !trace0 && !P.stats) {
+        P.round = 0;
+        P.stamp = 0;
+        P.dev_round = 1;
+        TG_TRY(spfp_graph_rounds<MODE>(g, Q, P, grid, s, rounds_out));
+        Q.stamp = stamp0 + *rounds_out + 2;  // the loop used stamp0 + 1 .. stamp0 + rounds + 1
+        return TG_OK;
+    }
     const int group = (int)std::max<int64_t>(1, g->opt_round_group);
     uint32_t rounds = 0;
     uint32_t r = 1;

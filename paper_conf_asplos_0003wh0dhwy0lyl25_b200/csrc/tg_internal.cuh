@@ -236,14 +236,6 @@ struct tg_graph {
     int comm_mode = 0;              // 0 replicated (source sharding), 1 vertex range
     DevArena arena;        // input copies + chain structures
     QueryScratch qs;
-    // EAT-family round loop captured as a CUDA graph with a conditional WHILE node
-    // (query_eat.cu): the last instantiation, keyed by its kernel parameters
-    struct RoundGraph {
-        cudaGraphExec_t exec = nullptr;
-        cudaGraph_t graph = nullptr;
-        unsigned char key[512] = {};
-        size_t key_len = 0;
-    } rgraph, rgl[TG_LANES - 1];
     // query lanes 1 .. TG_LANES-1 (EAT family, device outputs): scratch, stream, join event
     QueryScratch qsl[TG_LANES - 1];
     cudaStream_t lane_stream[TG_LANES - 1] = {};
@@ -259,7 +251,7 @@ struct tg_graph {
     int opt_mirror = 1;
     int64_t opt_exchange = 0;  // 1 = vertex-range partitions exchange states every round (cross-rank algorithm)
     int64_t opt_ub = 1;  // arrival bounds per (vertex, 8 queries) prune pairs: 0 off, 1 auto, 2 on (query_eat.cu)
-    int64_t opt_graph_loop = 1;
+    int64_t opt_graph_loop = 1;  // 0 host-driven rounds, 1 graph loop for graphs >= TG_GRAPH_LOOP_MIN_M edges, 2 always
     int64_t opt_lanes = 4;  // sub-batches in flight (EAT family, device outputs, graph loop): 1 .. TG_LANES  // 1 = GAC rounds run in a device-driven CUDA-graph WHILE loop (query_eat.cu)
     int64_t opt_packed_state = 0;  // 1 = packed (arrival|pred) u64 EAT-family state even without pred (tests)
     int64_t opt_order_sources = 1;  // schedule a call's sources by first departure time (query_eat.cu)
@@ -314,7 +306,18 @@ tg_status tg_validate_launch(const uint32_t *u, const uint32_t *v, const uint32_
 tg_status tg_validate_finish(tg_graph *g, const uint32_t *h);  // h: the 5 accumulated words
 tg_status tg_build_streamed(tg_graph *g);
 void tg_stream_free(tg_graph *g);
-void tg_round_graph_free(tg_graph *g);  // query_eat.cu: the cached round-loop graph
+bool tg_graph_loop_allowed();           // query_eat.cu: no kernel profiler attached, TG_GRAPH_LOOP != 0
+#ifndef TG_GRAPH_LOOP_MIN_M
+#define TG_GRAPH_LOOP_MIN_M (1ull << 23)  // edges: smaller graphs keep host-driven round loops
+#endif
+struct tg_graph;
+bool tg_graph_loop_worth(const tg_graph *g);  // query_eat.cu
+// Process-wide cache of instantiated round-loop graphs (query_eat.cu), keyed by the bytes of
+// their launch parameters and the device: a new handle whose buffers come back from the
+// block cache at the same addresses reuses the instantiation.
+cudaGraphExec_t tg_rg_find(const unsigned char *key, size_t len);
+// Takes ownership; false (the caller destroys them after use) when the cache is full.
+bool tg_rg_add(const unsigned char *key, size_t len, cudaGraph_t graph, cudaGraphExec_t exec);
 tg_status tg_run_eat_streamed(tg_graph *g, const uint32_t *sources, uint32_t k, tg_window w, uint32_t *out,
                               uint32_t *pred, bool out_dev, bool pred_dev, int mode, cudaStream_t s);
 tg_status tg_build_partition(tg_graph *g, ChainGraph *fwd, ChainGraph *mir, uint32_t vb, uint32_t ve, cudaStream_t s,

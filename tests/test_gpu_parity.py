@@ -520,7 +520,7 @@ def test_arrival_bound_filter_c2_small(tg):
         _check_values(tg, g, og, "ld", srcs[:16], win)
 
 
-@pytest.mark.parametrize("graph_loop", [0, 1])
+@pytest.mark.parametrize("graph_loop", [0, 2])
 def test_round_loop_modes(tg, graph_loop):
     """GAC rounds driven by the host (checks every round_group rounds) or by the device in
     a CUDA-graph WHILE loop (the default): same rows and preds; packed and u32 states
@@ -536,6 +536,9 @@ def test_round_loop_modes(tg, graph_loop):
             _check_rows(tg, g, og, p, srcs, win)
             rounds.append(g.last_stats()["rounds"])
             _check_values(tg, g, og, p, srcs, win)
+        for p in ("sp", "fp"):  # the SP/FP node-state engine's loop (same two modes)
+            _check_rows(tg, g, og, p, srcs[:6], win)
+            rounds.append(g.last_stats()["rounds"])
     assert min(rounds) >= 1
 
 
@@ -550,7 +553,7 @@ def test_two_query_lanes(tg):
     srcs = tgsynth.config_sources("C2", ge, k=200)
     res = {}
     for lanes in (1, 2, 4):
-        g = _gpu_graph(tg, n, u, v, t, d, lanes=lanes)
+        g = _gpu_graph(tg, n, u, v, t, d, lanes=lanes, graph_loop=2)
         for win in tgsynth.CONFIGS["C2"]["windows"]:
             for p in ("eat", "ld", "reach"):
                 o = g.query(p, srcs, win)
