@@ -1393,11 +1393,10 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
     static const bool trace = getenv("TG_TRACE") != nullptr;
     const bool work = any_work && g->m > 0 && alpha < omega;
     // query lanes (below) need device outputs and the device-driven round loop
-    // (host outputs too: each sub-batch's extract waits for its staging buffer's previous
-    // copy, wherever that ran -- the rounds of the lanes still overlap)
-    const bool lanes_ok = g->opt_lanes >= 2 && !g->opt_stats && g->opt_graph_loop && tg_graph_loop_allowed() &&
-                          tg_graph_loop_worth(g) &&
-                          !trace && work;
+    // (device outputs only: with host outputs the staging sink serialises the sub-batches on
+    // the copies, and C2's e2e leg measured 41 -> 82 ms per step with lanes)
+    const bool lanes_ok = g->opt_lanes >= 2 && out_dev && (!pred || pred_dev) && !g->opt_stats &&
+                          g->opt_graph_loop && tg_graph_loop_allowed() && tg_graph_loop_worth(g) && !trace && work;
     uint32_t S = tg_pick_sub_batch(g, k, false);
     // a lone full sub-batch runs as two halves on two lanes (C2 64-source EAT 7.9 -> 6.8 ms;
     // with several sub-batches 64 stays better: C4 1024 sources 1793 vs 1952 ms at 32)

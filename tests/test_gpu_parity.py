@@ -560,7 +560,7 @@ def test_two_query_lanes(tg):
                 o2, pr = g.query(p, srcs, win, with_pred=True)
                 torch.cuda.synchronize()
                 res[(lanes, win, p)] = (tg.as_u32(o), tg.as_u32(o2), tg.as_u32(pr), g.last_stats()["rounds"])
-        # host outputs (pinned staging ring on a copy stream) with the lanes
+        # host outputs (pinned staging ring on a copy stream; one lane)
         win = tgsynth.CONFIGS["C2"]["windows"][0]
         h = torch.empty((len(srcs), n), dtype=torch.int32).pin_memory()
         g.query("eat", srcs, win, out=h)
