@@ -309,7 +309,12 @@ __device__ __forceinline__ void unit_range(const EatP &P, const RoundV &R, uint3
         }
         // mask of queries for which edge pb+k is newly usable (lane k keeps its own):
         // each query lane's range as a row of block bits, transposed across the warp
-        uint32_t mask = tg_warp_transpose32(lo < hi ? tg_block_bits(lo, hi, pb) : 0u);
+        const uint32_t rowbits = lo < hi ? tg_block_bits(lo, hi, pb) : 0u;
+        if (ST) {  // diag[7]: blocks whose query ranges all cover it whole or not at all
+            const bool uni = __all_sync(0xffffffffu, rowbits == 0u || rowbits == 0xFFFFFFFFu);
+            if (uni && lane == 0) atomicAdd(P.diag + 7, 1ull);
+        }
+        uint32_t mask = tg_warp_transpose32(rowbits);
         if (p >= pend || (uint32_t)sl.y > P.omega) mask = 0;  // past the window end: never usable
 #if TG_UB
         // one-edge chains: the queries of an 8-query block whose arrival bound at the head
@@ -1514,8 +1519,8 @@ tg_status tg_run_eat_family(tg_graph *g, tg_problem p, const uint32_t *sources, 
             static const bool trace = getenv("TG_TRACE") != nullptr;
             if (trace)
                 fprintf(stderr, "[tg] diag S=%u: union edges %llu, unit ranges %llu, pairs %llu, activations %llu, "
-                        "frontier bits %llu, past filter %llu, pruned by bounds %llu\n", Sb, h[Sb + 1], h[Sb + 2], h[Sb + 3],
-                        h[Sb + 4], h[Sb + 5], h[Sb + 6], h[Sb + 7]);
+                        "frontier bits %llu, past filter %llu, pruned by bounds %llu, uniform blocks %llu\n", Sb, h[Sb + 1],
+                        h[Sb + 2], h[Sb + 3], h[Sb + 4], h[Sb + 5], h[Sb + 6], h[Sb + 7], h[Sb + 8]);
         }
     }
     for (int l = 0; l < lanes; l++) TG_TRY(finish(l));
