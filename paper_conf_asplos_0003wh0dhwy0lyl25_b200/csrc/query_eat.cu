@@ -65,6 +65,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_DEFER
 #define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
 #endif
+#ifndef TG_DEFER_BIG
+#define TG_DEFER_BIG 32                 // the threshold for sub-batch states >= 1 GiB (with query lanes, C4: -8 %)
+#endif
 #ifndef TG_DEFER_FROM
 #define TG_DEFER_FROM 3                 // first round in which units may be deferred
 #endif
@@ -97,7 +100,8 @@ struct EatP {
     uint32_t ub_sh;          // code c <-> bound alpha + (c << ub_sh)
     uint32_t *act, *bits;
     uint32_t *touched;  // stats: slots relaxed by any query of the sub-batch
-    uint32_t *defer;    // TG_DEFER experiment: units deferred once (bit per unit)
+    uint32_t *defer;    // TG_DEFER: units deferred once (bit per unit)
+    uint32_t defer_t;   // units with fewer new queries than this wait one round
     uint64_t bit_words;
     uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
     uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
@@ -428,7 +432,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         if (word && P.defer && P.S >= 64 && R.r >= TG_DEFER_FROM) {  // full sub-batches only
             const uint32_t bit = 1u << (ui & 31);
             uint32_t *dw = P.defer + (ui >> 5);
-            if (__popc(word) < TG_DEFER) {
+            if ((uint32_t)__popc(word) < P.defer_t) {
                 if (!(atomicOr(dw, bit) & bit)) {
                     atomicOr(R.fout + ui, word);
                     word = 0;
@@ -1300,6 +1304,9 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.st = Q.st; P.act = Q.act; P.bits = Q.bits; P.bit_words = Q.bit_words;
         P.n = g->n; P.S = S; P.G = G; P.alpha = alpha; P.omega = omega;
         P.ub0 = 0; P.ub1 = g->n * G;
+        // deferral threshold: states far beyond the L2 (C4's 4.3 GB) gain from merging more
+        // events (1795 -> 1649 ms with query lanes); C2's 256 MB state does not (21.7 -> 22.3)
+        P.defer_t = (uint64_t)S * g->n * 4 >= (1ull << 30) ? TG_DEFER_BIG : TG_DEFER;
         if (ub) {
             // codes over [alpha, min(omega, largest arrival)], where every state but INF
             // lies: the smallest shift that maps the far end to <= 254
