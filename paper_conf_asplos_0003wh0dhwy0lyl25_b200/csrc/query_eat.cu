@@ -65,6 +65,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_DEFER
 #define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
 #endif
+#ifndef TG_DEFER_MAX
+#define TG_DEFER_MAX 1                  // consecutive rounds a unit may wait
+#endif
 #ifndef TG_DEFER_BIG
 #define TG_DEFER_BIG 32                 // the threshold for sub-batch states >= 1 GiB (with query lanes, C4: -8 %)
 #endif
@@ -102,6 +105,7 @@ struct EatP {
     uint32_t *touched;  // stats: slots relaxed by any query of the sub-batch
     uint32_t *defer;    // TG_DEFER: units deferred once (bit per unit)
     uint32_t defer_t;   // units with fewer new queries than this wait one round
+    uint64_t defer_words;  // words of one deferral bitmap (TG_DEFER_MAX >= 2: a second one follows)
     uint64_t bit_words;
     uint32_t n, S, G;  // G = query groups of 32 per vertex (frontier unit = (vertex, group))
     uint32_t ub0, ub1; // frontier units this engine activates ([vb*G, ve*G) of its vertex range)
@@ -432,15 +436,30 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         if (word && P.defer && P.S >= 64 && R.r >= TG_DEFER_FROM) {  // full sub-batches only
             const uint32_t bit = 1u << (ui & 31);
             uint32_t *dw = P.defer + (ui >> 5);
+#if TG_DEFER_MAX >= 2
+            uint32_t *dw2 = dw + P.defer_words;  // second consecutive deferral
+#endif
             if ((uint32_t)__popc(word) < P.defer_t) {
                 if (!(atomicOr(dw, bit) & bit)) {
                     atomicOr(R.fout + ui, word);
                     word = 0;
+#if TG_DEFER_MAX >= 2
+                } else if (!(atomicOr(dw2, bit) & bit)) {
+                    atomicOr(R.fout + ui, word);
+                    word = 0;
                 } else {
                     atomicAnd(dw, ~bit);
+                    atomicAnd(dw2, ~bit);
+#else
+                } else {
+                    atomicAnd(dw, ~bit);
+#endif
                 }
             } else if (__ldcg(dw) & bit) {
                 atomicAnd(dw, ~bit);
+#if TG_DEFER_MAX >= 2
+                if (__ldcg(dw2) & bit) atomicAnd(dw2, ~bit);
+#endif
             }
         }
         pending = __ballot_sync(0xffffffffu, word != 0);
@@ -1062,7 +1081,7 @@ static tg_status ensure_scratch_q(tg_graph *g, QueryScratch &Q, uint32_t S, bool
     Q.vwords = (uint32_t)((S + 31) / 32);  // query groups per vertex
     TG_TRY(A.alloc((void **)&Q.fb[0], n * Q.vwords * 4));
     TG_TRY(A.alloc((void **)&Q.fb[1], n * Q.vwords * 4));
-    if (TG_DEFER) TG_TRY(A.alloc((void **)&Q.defer, (n * Q.vwords + 31) / 32 * 4 + 4));
+    if (TG_DEFER) TG_TRY(A.alloc((void **)&Q.defer, ((n * Q.vwords + 31) / 32 + 1) * 4 * TG_DEFER_MAX));
     if (nodes_state) {
         const uint64_t mark_len = S * nnodes;
         TG_TRY(A.alloc((void **)&Q.mark, std::max<uint64_t>(mark_len, 1) * 4));
@@ -1270,7 +1289,7 @@ static tg_status eat_rounds(tg_graph *g, QueryScratch &Q, const ChainGraph &cgr,
     const uint32_t G = (S + 31) / 32;
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[0], 0, n * G * 4, s));
     TG_TRY_CUDA(cudaMemsetAsync(Q.fb[1], 0, n * G * 4, s));
-    if (TG_DEFER) TG_TRY_CUDA(cudaMemsetAsync(Q.defer, 0, (n * G + 31) / 32 * 4 + 4, s));
+    if (TG_DEFER) TG_TRY_CUDA(cudaMemsetAsync(Q.defer, 0, ((n * G + 31) / 32 + 1) * 4 * TG_DEFER_MAX, s));
     if (g->opt_stats) {
         TG_TRY_CUDA(cudaMemsetAsync(Q.relax_cnt, 0, S * 8 + 8 + 64, s));
         TG_TRY_CUDA(cudaMemsetAsync(Q.touched, 0, Q.bit_words * 4, s));
@@ -1322,6 +1341,7 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.bigq = Q.bigq; P.bigcap = Q.bigcap; P.chq = Q.chq; P.chcap = Q.chcap; P.relax_cnt = Q.relax_cnt;
         P.touched = Q.touched;
         P.defer = Q.defer;
+        P.defer_words = (g->n * G + 31) / 32 + 1;
         P.diag = Q.relax_cnt + S + 1;
         const uint32_t grid = tg_grid_persistent(TG_ACT_MINB);
         static const bool trace = getenv("TG_TRACE") != nullptr;
