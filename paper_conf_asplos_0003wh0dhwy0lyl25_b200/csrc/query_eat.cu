@@ -65,6 +65,9 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #ifndef TG_DEFER
 #define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
 #endif
+#ifndef TG_DEFER_MIN_S
+#define TG_DEFER_MIN_S 32               // sub-batches smaller than this never defer (C3's 16-query batches: +18 %)
+#endif
 #ifndef TG_DEFER_MAX
 #define TG_DEFER_MAX 1                  // consecutive rounds a unit may wait
 #endif
@@ -433,7 +436,7 @@ __global__ void __launch_bounds__(QT, TG_ACT_MINB) k_eat_activate(EatP P) {
         // experiment: a unit with few new queries in a bulk round waits one round (its
         // word moves to the next frontier) so that more of its group's queries share one
         // scan of its edges; a unit is deferred at most once in a row
-        if (word && P.defer && P.S >= 64 && R.r >= TG_DEFER_FROM) {  // full sub-batches only
+        if (word && P.defer && P.S >= TG_DEFER_MIN_S && R.r >= TG_DEFER_FROM) {  // full sub-batches only
             const uint32_t bit = 1u << (ui & 31);
             uint32_t *dw = P.defer + (ui >> 5);
 #if TG_DEFER_MAX >= 2
@@ -1325,7 +1328,10 @@ static tg_status eat_loop(tg_graph *g, const ChainGraph &cgr, uint32_t S, uint32
         P.ub0 = 0; P.ub1 = g->n * G;
         // deferral threshold: states far beyond the L2 (C4's 4.3 GB) gain from merging more
         // events (1795 -> 1649 ms with query lanes); C2's 256 MB state does not (21.7 -> 22.3)
-        P.defer_t = (uint64_t)S * g->n * 4 >= (1ull << 30) ? TG_DEFER_BIG : TG_DEFER;
+        // (32-query sub-batches -- a lone 64-query batch split over two lanes -- defer only with
+        // such states: C4 168 -> 163 ms, C2 6.9 -> 7.2 ms)
+        const bool big_state = (uint64_t)S * g->n * 4 >= (1ull << 30);
+        P.defer_t = big_state ? TG_DEFER_BIG : (S >= 64 ? TG_DEFER : 0u);
         if (ub) {
             // codes over [alpha, min(omega, largest arrival)], where every state but INF
             // lies: the smallest shift that maps the far end to <= 254
