@@ -381,6 +381,8 @@ def run_ours(a, rank, world, local_rank):
         relax_ms += union[1] if union else 0.0
         relax_launches = sum(kprof[x][0] for x in relax_names)
         dom = max(kprof.items(), key=lambda kv: kv[1][1])
+        if union:  # overlapping lanes: the round loops' wall time, not their summed durations
+            dom = ("k_eat_rounds (graph loops of the query lanes, union of their intervals)", union)
         # SURVEY 8(d), batched with source lanes, at the state width the timed path moves
         # (u32 arrivals: pred = NULL): every slot relaxed by some query of a sub-batch is read
         # once (16 B slot + 4 B occurrence), every relaxation touches 4 B of state:
@@ -434,6 +436,8 @@ def run_ours(a, rank, world, local_rank):
             "profiled_kernels": "all" if plevel == 1 else "relaxation kernels only (CUDA events per launch)",
             "kernels_ms_per_step": {x: round(v[1] / a.steps, 4) for x, v in
                                     sorted(kprof.items(), key=lambda kv: -kv[1][1])[:12]},
+            "kernels_ms_note": ("summed per-launch durations; the query lanes' round loops overlap, so their sum "
+                                "exceeds the step" if union else "summed per-launch durations"),
         }
 
     if persistent is not None:
