@@ -47,9 +47,9 @@ namespace {
 
 constexpr int QT = 256;                 // threads per block
 // Unions longer than big_t edges are cut into big_t-edge chunks for k_eat_big, big_t =
-// 8 x the mean out-degree within [BIG_T_MIN, BIG_T_MAX]: denser graphs amortise a chunk's
-// record over more edges (C4, degree 32: 256 -> job -1.8 %; C2, degree 16: 128, 512 would
-// cost +16 %).  Queue capacities are sized for the smallest chunk.
+// TG_BIG_T_F x the mean out-degree within [BIG_T_MIN, BIG_T_MAX]: denser graphs amortise a
+// chunk's record over more edges (C4, degree 32: 512; C2, degree 16: 256 -- with query lanes
+// both are as fast as or faster than 8x).  Queue capacities are sized for the smallest chunk.
 constexpr uint32_t BIG_T_MIN = 128, BIG_T_MAX = 512;
 #ifndef TG_BIG_T_F
 #define TG_BIG_T_F 16  // chunk edges per unit of mean out-degree (with query lanes: C4 1671 -> 1659 ms; 8 before them)
