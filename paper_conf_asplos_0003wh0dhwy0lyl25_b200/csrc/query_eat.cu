@@ -63,7 +63,7 @@ static uint32_t pick_big_t(const tg_graph *g) {
 }
 constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in the activating thread
 #ifndef TG_MLP
-#define TG_MLP 4                        // state reads in flight per lane in the pair loop
+#define TG_MLP 2                        // state reads in flight per lane in the pair loop (4 before query lanes)
 #endif
 #ifndef TG_DEFER
 #define TG_DEFER 16                     // units with fewer new queries wait one round (0 = off; C4 job -3.5 %)
@@ -94,7 +94,7 @@ constexpr uint32_t INLINE_WALK = 8;     // walks up to this many slots stay in t
 #endif
 constexpr uint32_t UB_WORDS = TG_UBQ == 4 ? 2 : 1;  // u64 code words per vertex
 #ifndef TG_ACT_MINB
-#define TG_ACT_MINB 6                   // resident blocks per SM requested for the relax kernels (8, 7, 5, 4 measured slower)
+#define TG_ACT_MINB 7                   // resident blocks per SM for the relax kernels (with query lanes: C4 1644 -> 1590 ms with MLP 2; 6 before)
 #endif
 
 struct EatP {
